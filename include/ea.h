@@ -1,0 +1,197 @@
+/*
+ * ea.h -- C ABI of the B200-native elastic-averaging step of AvgPipe
+ * (Chen, Xu, Qian, Zhou, "Elastic Averaging for Efficient Pipelined DNN
+ * Training", PPoPP'23).  Citations "P:<line> §<sec>" are to the paper text.
+ *
+ * What the library computes (per pipeline stage s, per iteration; §3.2):
+ *
+ *   N parallel pipelines each hold a replica x_i of every stage; a
+ *   reference ("center") model x~ is co-partitioned with them.  For
+ *   every element j, with x~ = x~_t and all right-hand sides at step t:
+ *
+ *     Step 1  local update of a user-specified optimizer -- here SGD
+ *                     with momentum, PyTorch convention (buffer starts at 0,
+ *                     dampening 0):
+ *                       g' = g_i + lambda*x_i;  m_i <- mu*m_i + g';
+ *                       Delta_i = -lr * (nesterov ? g' + mu*m_i : m_i)
+ *     Step 2  dilution in the ratio (1-alpha):alpha plus the local update:
+ *                       x_i <- (1-alpha)*x_i + alpha*x~ + Delta_i
+ *     Step 3/4  send and accumulate the contribution
+ *                       R = sum_i r_i,  r_i = rho*Delta_i + beta*(x_i - x~)
+ *     Step 5  normalise and apply:  x~ <- x~ + R / N
+ *
+ *   (alpha, beta, rho) = (1/N, 0, 1) is the paper's own mode ("stays the
+ *   average"); (alpha, 0, N*alpha) is EASGD's center pull (refs [35],
+ *   [18]); see DESIGN.md "Readings" c1-c14 for every reading of the prose.
+ *
+ * Layouts (ea_config.layout):
+ *   EA_COLOCATED  all N replicas of each hosted stage live on this GPU (the
+ *                 paper's placement: one GPU per stage).  One
+ *                 fused kernel per ea_step; no communication.
+ *   EA_SPREAD     one replica per GPU per stage; world == N ranks; the center
+ *                 of each stage is sharded 1/N over the ranks.  ea_step runs
+ *                 the fused local kernel, an NCCL reduce-scatter of the
+ *                 contributions into the owning shard, the shard update and an
+ *                 in-place NCCL all-gather, all on a library-owned side stream
+ *                 (the reference process "so as to not block the parallel
+ *                 pipelines").
+ *
+ * Data: fp32, flat, contiguous, device-resident, 16-byte aligned.  The caller
+ * owns x_i, g_i and x~ (e.g. torch tensors); the library owns momentum,
+ * scratch, streams, events and the NCCL communicator.
+ *
+ * Errors: every call returns an ea_status; nothing throws or aborts.  On
+ * EA_EINVAL nothing was enqueued.  ea_last_error(h) returns a message for the
+ * last failing call on h (thread-local message for h == NULL / ea_init).
+ * Threading: a handle is not thread-safe; use one per (process, device).
+ */
+#ifndef AVGPIPE_EA_H_
+#define AVGPIPE_EA_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define EA_ABI_VERSION 1
+#define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
+#define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
+
+typedef enum {
+  EA_OK = 0,
+  EA_EINVAL = 1,  /* bad argument: null/misaligned pointer, N<1, alpha not in [0,1], ... */
+  EA_ECUDA = 2,   /* CUDA launch / runtime error (also async, reported at ea_sync) */
+  EA_ENCCL = 3,   /* NCCL error (init, enqueue, or async at ea_sync) */
+  EA_ESTATE = 4,  /* call not valid in the handle's current state/layout */
+  EA_ENOMEM = 5   /* device or host allocation failed */
+} ea_status;
+
+typedef enum { EA_COLOCATED = 0, EA_SPREAD = 1 } ea_layout;
+
+typedef struct {
+  int32_t n_pipelines;          /* N >= 1 parallel pipelines */
+  int32_t n_stages;             /* stages hosted by this process, >= 1 */
+  const int64_t* stage_params;  /* n_stages entries, P_s >= 1 (copied by ea_init) */
+  float alpha;                  /* dilution rate in [0,1], P:112 (default 1/N) */
+  float beta;                   /* center pull (EASGD); 0 in the paper's mode */
+  float rho;                    /* weight of Delta_i in the contribution; 1 in the paper's mode */
+  float lr;                     /* SGD learning rate eta */
+  float momentum;               /* mu in [0,1) */
+  float weight_decay;           /* lambda >= 0 (L2, added to the gradient) */
+  int32_t nesterov;             /* 0/1 */
+  int32_t layout;               /* ea_layout */
+  int32_t rank;                 /* EA_SPREAD: 0 <= rank < world; ignored otherwise */
+  int32_t world;                /* EA_SPREAD: must equal n_pipelines; ignored otherwise */
+  int32_t device;               /* CUDA device ordinal the handle binds to */
+} ea_config;
+
+typedef struct ea_ctx* ea_handle;
+
+/* One op of the micro-batch order (Algorithm 1): kind 0 = forward,
+ * 1 = backward; micro_batch is 0-based. */
+typedef struct {
+  int32_t kind;
+  int32_t micro_batch;
+} ea_op;
+
+/* ABI version compiled into the library (EA_ABI_VERSION). */
+int32_t ea_abi_version(void);
+
+/* Fill id[EA_UNIQUE_ID_BYTES] with a fresh NCCL unique id (call on rank 0 and
+ * broadcast it, e.g. over a torch process group).  EA_ENCCL on failure. */
+ea_status ea_get_unique_id(uint8_t* id);
+
+/* Create a handle.  Validates cfg (EA_EINVAL, nothing allocated), binds
+ * cfg->device, allocates zero-initialised momentum for every hosted stage and
+ * replica (N per stage co-located, 1 per stage spread) and, for EA_SPREAD,
+ * the side stream, events, contribution scratch and the NCCL communicator
+ * built from nccl_id (world ranks; ignored and may be NULL for EA_COLOCATED;
+ * NULL for EA_SPREAD is EA_EINVAL).  *out is NULL on failure. */
+ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out);
+
+/* Number of fp32 elements the center buffer of `stage` must hold:
+ * P_s for EA_COLOCATED; P_pad = round_up(P_s, 32*N) for EA_SPREAD (the
+ * padding must be zero-initialised by the caller and stays zero).
+ * Returns -1 for a bad handle or stage. */
+int64_t ea_center_capacity(ea_handle h, int32_t stage);
+
+/* Number of center elements owned by this rank (EA_SPREAD: P_pad/N; the
+ * shard starts at element rank*P_pad/N).  EA_COLOCATED: P_s.  -1 on error. */
+int64_t ea_shard_elems(ea_handle h, int32_t stage);
+
+/* One elastic-averaging iteration of `stage` (0-based, < n_stages).
+ *   replica_ptrs: EA_COLOCATED: N device pointers x_0..x_{N-1}, each P_s
+ *                 floats, updated in place; EA_SPREAD: 1 pointer (this
+ *                 rank's replica).
+ *   grad_ptrs:    matching gradient pointers (read only).
+ *   center_ptr:   x~ of the stage (ea_center_capacity floats), updated in place.
+ *   stream:       caller's stream (cudaStream_t); NULL = legacy default stream.
+ * EA_COLOCATED: one fused kernel on `stream`.  EA_SPREAD: the side stream
+ * waits for `stream`, runs kernel -> reduce-scatter -> shard update ->
+ * all-gather; `stream` then waits only for the kernel (x_i ready), so the
+ * next forward can start while the center is being exchanged.  Call
+ * ea_sync before reading x~ on another stream.  All ranks must call
+ * ea_step for the same stages in the same order (NCCL ordering).
+ * Pointers must stay valid until the work completes. */
+ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
+                  const float* const* grad_ptrs, float* center_ptr, void* stream);
+
+/* Make `stream` wait until every center update enqueued so far is complete,
+ * then report any asynchronous CUDA/NCCL error seen so far.  Does not block
+ * the host. */
+ea_status ea_sync(ea_handle h, void* stream);
+
+/* ---- Phases of the EA_SPREAD step, for callers that run their own
+ * collective (and for single-GPU verification of the decomposition). ---- */
+
+/* Local phase of EA_SPREAD on `stream`: updates x (this rank's replica) and
+ * this rank's momentum in place and writes the contribution
+ * r = rho*Delta + beta*(x - x~) into contrib[0..P_s) and zeros into
+ * contrib[P_s..P_pad).  center_ptr is read only. */
+ea_status ea_spread_local(ea_handle h, int32_t stage, float* replica_ptr, const float* grad_ptr,
+                          const float* center_ptr, float* contrib, void* stream);
+
+/* Shard phase of EA_SPREAD on `stream`: center_shard[k] += reduced[k] / N for
+ * k < ea_shard_elems (reduced = this rank's shard of sum_i r_i). */
+ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const float* reduced,
+                          void* stream);
+
+/* ---- Optimizer state (checkpoint / resume) ---- */
+
+/* *momentum_dev = device pointer to the momentum of (stage, replica): P_s
+ * floats, owned by the library, valid until ea_destroy.  EA_SPREAD: replica
+ * must be 0. */
+ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, float** momentum_dev);
+
+/* Copy P_s floats from device pointer momentum_src into the momentum of
+ * (stage, replica), ordered on `stream`. */
+ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, const float* momentum_src,
+                       void* stream);
+
+/* Replace the hyper-parameters (e.g. a learning-rate schedule); same
+ * validation as ea_init.  Takes effect for steps enqueued afterwards. */
+ea_status ea_set_hyper(ea_handle h, float alpha, float beta, float rho, float lr, float momentum,
+                       float weight_decay, int32_t nesterov);
+
+/* Wait for outstanding work, free everything the library owns, destroy the
+ * communicator.  NULL is a no-op. */
+ea_status ea_destroy(ea_handle h);
+
+/* Message of the last failing call on h (h == NULL: this thread's last
+ * ea_init / handle-less failure).  Never NULL; "" if none. */
+const char* ea_last_error(ea_handle h);
+
+/* Advance-forward-propagation order of one batch on one stage (Algorithm 1,
+ * P:140-162, plus the implied cool-down -- DESIGN.md c15).  K stages, M
+ * micro-batches, stage 0-based (< K), advance = forwards run in advance
+ * (clamped to [0, M]; K-1-stage is 1F1B, M is AFAB).  Writes 2M ops to out
+ * (cap >= 2M) and returns 2M; returns -EA_EINVAL for K < 1, M < 0, stage out
+ * of range, cap < 2M or out == NULL (with M > 0).  Host only; no GPU needed. */
+int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* AVGPIPE_EA_H_ */
