@@ -1,0 +1,373 @@
+#!/usr/bin/env python
+"""Benchmark of the elastic-averaging step (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+One "step" = one elastic-averaging iteration over every stage of the
+workload (rows a1-a8 of SURVEY §8): N=1 runs configs[1] (C2: ResNet-50-sized
+25M params, K=4 stages, N=4 pipelines, all replicas co-located on the GPU);
+N>1 (torchrun, one rank per GPU) runs the spread layout with N pipelines
+(C3 for 2/4 GPUs, C4 for 8) -- one replica of every stage per GPU, the
+center sharded and exchanged by NCCL reduce-scatter / all-gather.
+
+value = replica-params/s = (pipelines x params) / step time, whole job,
+inputs resident in HBM, timed with CUDA events (max over ranks).  `e2e`
+repeats the measurement through the same API with the gradients coming
+from pinned HOST memory and the new center read back every step.
+`--impl reference` times the float64 CPU oracle (the only reference that
+exists: the paper ships no code) on a bounded per-step sample.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "elastic-avg step params/sec and HBM/NVLink GB/s (% roofline) at 1/2/4/8 B200"
+UNIT = "replica-params/s"
+MODE = "combined"   # rho=1, beta=N*alpha, alpha=1/N; every mode moves the same bytes
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=1000)
+    ap.add_argument("--warmup", type=int, default=20)
+    ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
+    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl"), default="auto")
+    ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=10.0)
+    ap.add_argument("--config", default=None, help="override workload key (synth.CONFIGS)")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- env
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return rank, world, local
+
+
+def measured_peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        d = json.load(open(path))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy burst)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+NVLINK_PEAK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md)
+
+
+class ClockSampler:
+    """NVML clocks + throttle reasons sampled DURING the timed region."""
+    REASONS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap", 0x8: "hw_slowdown",
+               0x10: "sync_boost", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x100: "display_clock_setting"}
+
+    def __init__(self, index: int, period_s: float = 0.02):
+        self.samples, self.reasons, self.ok = [], set(), False
+        self.max_mhz = None
+        self.period = period_s
+        self._stop = threading.Event()
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            self.nv = pynvml
+            self.h = pynvml.nvmlDeviceGetHandleByIndex(index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = repr(e)
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                bits = self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h)
+                for b, name in self.REASONS.items():
+                    if bits & b:
+                        self.reasons.add(name)
+            except Exception:
+                pass
+            self._stop.wait(self.period)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *exc):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok or not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons),
+                    "samples": len(self.samples)}
+        s = sorted(self.samples)
+        return {"sm_mhz": s[len(s) // 2], "sm_max_mhz": self.max_mhz, "reasons": sorted(self.reasons - {"gpu_idle"}),
+                "samples": len(s)}
+
+
+def workload_key(gpus: int, override):
+    if override:
+        return override
+    return {1: "C2", 2: "C3N2", 4: "C3N4", 8: "C4"}.get(gpus, "C4")
+
+
+# ----------------------------------------------------------------------------- our arm
+def bytes_colocated(n, p):
+    """Algorithmic HBM bytes of one co-located launch: read x~ and x_i, g_i,
+    m_i of every replica, write x_i, m_i and x~ (fp32): (20 N + 8) P."""
+    return (20 * n + 8) * p
+
+
+def bytes_spread_local(p):
+    """HBM bytes of the spread local kernel: read x, g, m, x~; write x, m, r: 28 P."""
+    return 28 * p
+
+
+def run_ours(args, rank, world, local):
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ppopp_chen0qz23_b200 import synth
+    from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
+    from paper_conf_ppopp_chen0qz23_b200 import parallel
+
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    key = workload_key(world, args.config)
+    cfg = synth.CONFIGS[key]
+    n = cfg.n_pipelines if world == 1 else world
+    sizes = cfg.stage_sizes
+    a, b, r = synth.mode_coeffs(MODE, n)
+    stream = torch.cuda.current_stream(dev)
+    spread = world > 1
+    if spread:
+        dist.init_process_group("nccl", device_id=dev)
+        uid = parallel.broadcast_unique_id()
+        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
+                             layout="spread", rank=rank, world=world, device=local, nccl_id=uid)
+        state = []
+        for s, p in enumerate(sizes):
+            reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s + parallel.replica_of(rank, s, n))
+            cc = torch.zeros(h.center_capacity(s), device=dev)
+            cc[:p] = c0
+            state.append((reps, grads, cc))
+    else:
+        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
+                             device=local, kernel_variant=args.variant)
+        state = [synth.device_state(n, p, dev, seed=s) for s, p in enumerate(sizes)]
+        state = [(reps, grads, c) for (reps, c, grads) in state]
+    order = parallel.stage_order(len(sizes))
+
+    def one_step(evs=None):
+        for s in order:
+            reps, grads, c = state[s]
+            if evs is not None:
+                evs[s][0].record(stream)
+            h.step(s, reps, grads, c, stream=stream)
+            if evs is not None:
+                evs[s][1].record(stream)
+        if spread:
+            h.sync(stream)
+
+    for _ in range(args.warmup):
+        one_step()
+    torch.cuda.synchronize()
+    if spread:
+        dist.barrier()
+    # per-launch events for the dominant kernel (co-located: every ea_step is one kernel)
+    ev = None
+    if not spread:
+        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in sizes]
+              for _ in range(args.steps)]
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local) as clk:
+        torch.cuda.synchronize()
+        t0.record(stream)
+        for k in range(args.steps):
+            one_step(None if ev is None else ev[k])
+        t1.record(stream)
+        torch.cuda.synchronize()
+    ms = t0.elapsed_time(t1) / args.steps
+    if spread:
+        tt = torch.tensor([ms], device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        ms = float(tt.item())
+    total_params = sum(sizes)
+    value = n * total_params / (ms * 1e-3)
+    peak, peak_src = measured_peaks()
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "f32", "data": "synthetic (seeded: x0~N(0,0.02^2), replicas +N(0,1e-3^2), "
+                                                        "grads~N(0,1e-2^2); torch.Generator on device)"}
+    ws_bytes = (n * 3 + 1) * 4 * total_params if not spread else 5 * 4 * total_params
+    out["config"] = {"workload": cfg.name, "n_pipelines": n, "n_stages": len(sizes), "params": total_params,
+                     "stage_params": sizes, "layout": "spread" if spread else "colocated", "mode": MODE,
+                     "optimizer": "sgd-momentum(0.9)", "kernel": args.variant,
+                     "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
+    if not spread:
+        step_bytes = sum(bytes_colocated(n, p) for p in sizes)
+        kern_ms = [ev[k][s][0].elapsed_time(ev[k][s][1]) for k in range(args.steps) for s in range(len(sizes))]
+        # per launch, averaged over the (equal-sized) stages
+        per_launch_bytes = step_bytes / len(sizes)
+        avg_ms = sum(kern_ms) / len(kern_ms)
+        achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
+        out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
+        out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                           "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
+                           "kernel": "colocated_" + ("laneshfl" if args.variant == "laneshfl" else "regloop"),
+                           "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
+                           "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
+        out["gpu_launches"] = args.steps * len(sizes)
+    else:
+        step_bytes = sum(bytes_spread_local(p) for p in sizes)
+        nv_bytes = sum(2 * (n - 1) / n * 4 * h.center_capacity(s) for s in range(len(sizes)))
+        out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
+        nv_gbs = nv_bytes / (ms * 1e-3) / 1e9
+        out["roofline"] = {"bound": "nvlink", "achieved": nv_gbs, "peak": NVLINK_PEAK_GBS, "unit": "GB/s",
+                           "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None,
+                           "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / "
+                                   "step time; peak = measured peer copy per direction"}
+        out["gpu_launches"] = args.steps * 2 * len(sizes)
+    out["clocks"] = clk.summary()
+    if not spread and not args.no_e2e:
+        out["e2e"] = e2e_colocated(h, state, sizes, n, args, stream, dev, order)
+    elif spread:
+        out["e2e"] = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        out["cpu_baseline"] = cpu_baseline(cfg, n, seconds=args.cpu_seconds)
+    h.close()
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    if spread:
+        dist.destroy_process_group()
+
+
+def traffic_from_profiles(workload):
+    path = os.path.join(ROOT, "profiles", "traffic.json")
+    if not os.path.exists(path):
+        return None
+    d = json.load(open(path))
+    return d.get(workload, {}).get("dram_bytes_per_launch")
+
+
+def e2e_colocated(h, state, sizes, n, args, stream, dev, order):
+    """Same step through the same API, gradients copied from pinned host memory
+    before each stage's update and the new center copied back after it."""
+    import torch
+    host_g = [[g.cpu().pin_memory() for g in grads] for (_, grads, _) in state]
+    host_c = [torch.empty(p, dtype=torch.float32).pin_memory() for p in sizes]
+    dev_g = [[torch.empty_like(g) for g in grads] for (_, grads, _) in state]
+
+    def step():
+        for s in order:
+            reps, _, c = state[s]
+            for i in range(n):
+                dev_g[s][i].copy_(host_g[s][i], non_blocking=True)
+            h.step(s, reps, dev_g[s], c, stream=stream)
+            host_c[s].copy_(c, non_blocking=True)
+
+    for _ in range(3):
+        step()
+    torch.cuda.synchronize()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for _ in range(args.e2e_steps):
+        step()
+    t1.record(stream)
+    torch.cuda.synchronize()
+    ms = t0.elapsed_time(t1) / args.e2e_steps
+    return {"value": n * sum(sizes) / (ms * 1e-3), "unit": UNIT, "ms_per_step": ms,
+            "h2d_bytes_per_step": 4 * n * sum(sizes), "d2h_bytes_per_step": 4 * sum(sizes),
+            "path": "binding ElasticAveraging.step; pinned host grads -> device, center -> pinned host"}
+
+
+# ----------------------------------------------------------------------------- oracle (CPU) legs
+def _oracle_sample(n, p_sample, seed=0):
+    import numpy as np
+    from paper_conf_ppopp_chen0qz23_b200 import synth
+    reps, c = synth.host_state(n, p_sample, seed=synth.WEIGHT_SEED + seed)
+    gs = synth.GradStream(n, p_sample).next()
+    return reps, [np.zeros(p_sample, dtype=np.float32) for _ in range(n)], c, gs
+
+
+def cpu_baseline(cfg, n, seconds=10.0):
+    """The float64 oracle, as it stands (single-threaded numpy), on a bounded
+    sample: one full stage of the workload, repeated until `seconds` pass."""
+    from oracle.ea_oracle import Hyper, ea_step
+    from paper_conf_ppopp_chen0qz23_b200 import synth
+    p = cfg.stage_sizes[0]
+    a, b, r = synth.mode_coeffs(MODE, n)
+    hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
+    xs, ms, c, g = _oracle_sample(n, p)
+    steps, t0 = 0, time.perf_counter()
+    while True:
+        xs, ms, c = ea_step(xs, ms, c, g, hp)
+        steps += 1
+        el = time.perf_counter() - t0
+        if el >= seconds:
+            break
+    return {"value": n * p * steps / el, "unit": UNIT, "cores": 1, "kind": "oracle",
+            "sample": f"{steps} oracle steps of one {p}-element stage x N={n} (float64 numpy, 1 thread), "
+                      f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0))}
+
+
+def run_reference(args, rank, world):
+    """--impl reference: the float64 oracle on host cores; rank 0 only."""
+    if rank != 0:
+        return
+    from oracle.ea_oracle import Hyper, ea_step
+    from paper_conf_ppopp_chen0qz23_b200 import synth
+    key = workload_key(world, args.config)
+    cfg = synth.CONFIGS[key]
+    n = cfg.n_pipelines if world == 1 else world
+    a, b, r = synth.mode_coeffs(MODE, n)
+    hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
+    p_sample = 1 << 16      # per-step bounded sample: 65,536 elements x N replicas
+    xs, ms, c, g = _oracle_sample(n, p_sample)
+    for _ in range(args.warmup):
+        xs, ms, c = ea_step(xs, ms, c, g, hp)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        xs, ms, c = ea_step(xs, ms, c, g, hp)
+    el = time.perf_counter() - t0
+    ms_step = el / args.steps * 1e3
+    value = n * p_sample / (el / args.steps)
+    sample = f"each step: {p_sample} elements x N={n} replicas of {cfg.name} (float64 numpy, 1 thread)"
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
+           "config": {"workload": cfg.name, "n_pipelines": n, "params_per_step_sample": p_sample, "mode": MODE},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+           "gpu_launches": 0}
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse()
+    rank, world, local = dist_env()
+    if world != args.gpus and rank == 0:
+        print(f"note: WORLD_SIZE={world} but --gpus={args.gpus}; using WORLD_SIZE", file=sys.stderr)
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    run_ours(args, rank, world, local)
+
+
+if __name__ == "__main__":
+    main()

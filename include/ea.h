@@ -54,6 +54,12 @@
 extern "C" {
 #endif
 
+#if defined(__GNUC__)
+#define EA_API __attribute__((visibility("default")))
+#else
+#define EA_API
+#endif
+
 #define EA_ABI_VERSION 1
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
@@ -84,6 +90,11 @@ typedef struct {
   int32_t rank;                 /* EA_SPREAD: 0 <= rank < world; ignored otherwise */
   int32_t world;                /* EA_SPREAD: must equal n_pipelines; ignored otherwise */
   int32_t device;               /* CUDA device ordinal the handle binds to */
+  int32_t kernel_variant;       /* EA_COLOCATED kernel: 0 = library default, 1 = register-
+                                   resident replica loop, 2 = lane-per-replica with the center
+                                   tile staged by cp.async.bulk and warp-shuffle reduction
+                                   (N <= 8; larger N uses 1).  Same results up to fp32
+                                   summation order (DESIGN.md c14). */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;
@@ -96,29 +107,33 @@ typedef struct {
 } ea_op;
 
 /* ABI version compiled into the library (EA_ABI_VERSION). */
-int32_t ea_abi_version(void);
+EA_API int32_t ea_abi_version(void);
 
 /* Fill id[EA_UNIQUE_ID_BYTES] with a fresh NCCL unique id (call on rank 0 and
  * broadcast it, e.g. over a torch process group).  EA_ENCCL on failure. */
-ea_status ea_get_unique_id(uint8_t* id);
+EA_API ea_status ea_get_unique_id(uint8_t* id);
 
 /* Create a handle.  Validates cfg (EA_EINVAL, nothing allocated), binds
  * cfg->device, allocates zero-initialised momentum for every hosted stage and
  * replica (N per stage co-located, 1 per stage spread) and, for EA_SPREAD,
- * the side stream, events, contribution scratch and the NCCL communicator
- * built from nccl_id (world ranks; ignored and may be NULL for EA_COLOCATED;
- * NULL for EA_SPREAD is EA_EINVAL).  *out is NULL on failure. */
-ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out);
+ * the side stream, events, contribution scratch and -- if nccl_id is not
+ * NULL -- the NCCL communicator of `world` ranks built from nccl_id (a
+ * collective call: every rank must call ea_init).  EA_SPREAD with nccl_id ==
+ * NULL is the external-collective mode: ea_step returns EA_ESTATE and the
+ * caller drives ea_spread_local / its own reduce-scatter / ea_spread_apply /
+ * its own all-gather.  nccl_id is ignored for EA_COLOCATED.  *out is NULL on
+ * failure. */
+EA_API ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out);
 
 /* Number of fp32 elements the center buffer of `stage` must hold:
  * P_s for EA_COLOCATED; P_pad = round_up(P_s, 32*N) for EA_SPREAD (the
  * padding must be zero-initialised by the caller and stays zero).
  * Returns -1 for a bad handle or stage. */
-int64_t ea_center_capacity(ea_handle h, int32_t stage);
+EA_API int64_t ea_center_capacity(ea_handle h, int32_t stage);
 
 /* Number of center elements owned by this rank (EA_SPREAD: P_pad/N; the
  * shard starts at element rank*P_pad/N).  EA_COLOCATED: P_s.  -1 on error. */
-int64_t ea_shard_elems(ea_handle h, int32_t stage);
+EA_API int64_t ea_shard_elems(ea_handle h, int32_t stage);
 
 /* One elastic-averaging iteration of `stage` (0-based, < n_stages).
  *   replica_ptrs: EA_COLOCATED: N device pointers x_0..x_{N-1}, each P_s
@@ -134,13 +149,13 @@ int64_t ea_shard_elems(ea_handle h, int32_t stage);
  * ea_sync before reading x~ on another stream.  All ranks must call
  * ea_step for the same stages in the same order (NCCL ordering).
  * Pointers must stay valid until the work completes. */
-ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
+EA_API ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
                   const float* const* grad_ptrs, float* center_ptr, void* stream);
 
 /* Make `stream` wait until every center update enqueued so far is complete,
  * then report any asynchronous CUDA/NCCL error seen so far.  Does not block
  * the host. */
-ea_status ea_sync(ea_handle h, void* stream);
+EA_API ea_status ea_sync(ea_handle h, void* stream);
 
 /* ---- Phases of the EA_SPREAD step, for callers that run their own
  * collective (and for single-GPU verification of the decomposition). ---- */
@@ -149,12 +164,12 @@ ea_status ea_sync(ea_handle h, void* stream);
  * this rank's momentum in place and writes the contribution
  * r = rho*Delta + beta*(x - x~) into contrib[0..P_s) and zeros into
  * contrib[P_s..P_pad).  center_ptr is read only. */
-ea_status ea_spread_local(ea_handle h, int32_t stage, float* replica_ptr, const float* grad_ptr,
+EA_API ea_status ea_spread_local(ea_handle h, int32_t stage, float* replica_ptr, const float* grad_ptr,
                           const float* center_ptr, float* contrib, void* stream);
 
 /* Shard phase of EA_SPREAD on `stream`: center_shard[k] += reduced[k] / N for
  * k < ea_shard_elems (reduced = this rank's shard of sum_i r_i). */
-ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const float* reduced,
+EA_API ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const float* reduced,
                           void* stream);
 
 /* ---- Optimizer state (checkpoint / resume) ---- */
@@ -162,25 +177,25 @@ ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const
 /* *momentum_dev = device pointer to the momentum of (stage, replica): P_s
  * floats, owned by the library, valid until ea_destroy.  EA_SPREAD: replica
  * must be 0. */
-ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, float** momentum_dev);
+EA_API ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, float** momentum_dev);
 
 /* Copy P_s floats from device pointer momentum_src into the momentum of
  * (stage, replica), ordered on `stream`. */
-ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, const float* momentum_src,
+EA_API ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, const float* momentum_src,
                        void* stream);
 
 /* Replace the hyper-parameters (e.g. a learning-rate schedule); same
  * validation as ea_init.  Takes effect for steps enqueued afterwards. */
-ea_status ea_set_hyper(ea_handle h, float alpha, float beta, float rho, float lr, float momentum,
+EA_API ea_status ea_set_hyper(ea_handle h, float alpha, float beta, float rho, float lr, float momentum,
                        float weight_decay, int32_t nesterov);
 
 /* Wait for outstanding work, free everything the library owns, destroy the
  * communicator.  NULL is a no-op. */
-ea_status ea_destroy(ea_handle h);
+EA_API ea_status ea_destroy(ea_handle h);
 
 /* Message of the last failing call on h (h == NULL: this thread's last
  * ea_init / handle-less failure).  Never NULL; "" if none. */
-const char* ea_last_error(ea_handle h);
+EA_API const char* ea_last_error(ea_handle h);
 
 /* Advance-forward-propagation order of one batch on one stage (Algorithm 1,
  * P:140-162, plus the implied cool-down -- DESIGN.md c15).  K stages, M
@@ -188,7 +203,7 @@ const char* ea_last_error(ea_handle h);
  * (clamped to [0, M]; K-1-stage is 1F1B, M is AFAB).  Writes 2M ops to out
  * (cap >= 2M) and returns 2M; returns -EA_EINVAL for K < 1, M < 0, stage out
  * of range, cap < 2M or out == NULL (with M > 0).  Host only; no GPU needed. */
-int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
+EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
 
 #ifdef __cplusplus
 }

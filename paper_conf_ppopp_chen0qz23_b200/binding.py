@@ -1,0 +1,264 @@
+"""Thin ctypes binding of ``include/ea.h`` (argument marshalling only).
+
+Every step of the elastic-averaging path runs inside ``libavgpipe_ea.so``
+(hand-written sm_100a kernels + NCCL).  This module converts torch tensors,
+streams and Python scalars into the C ABI's pointers and sizes, raises on a
+non-zero ``ea_status`` with the library's message, and never computes
+anything itself.  There is no fallback: if the library is missing, every
+entry point raises ``LibraryNotBuilt``.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import List, Optional, Sequence, Tuple
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libavgpipe_ea.so")
+
+EA_OK, EA_EINVAL, EA_ECUDA, EA_ENCCL, EA_ESTATE, EA_ENOMEM = range(6)
+EA_COLOCATED, EA_SPREAD = 0, 1
+STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA_ESTATE", 5: "EA_ENOMEM"}
+LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
+VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2}
+UNIQUE_ID_BYTES = 128
+ABI_VERSION = 1
+
+
+class LibraryNotBuilt(RuntimeError):
+    pass
+
+
+class EAError(RuntimeError):
+    def __init__(self, status: int, message: str):
+        super().__init__(f"{STATUS_NAMES.get(status, status)}: {message}")
+        self.status = status
+
+
+class EAConfig(ctypes.Structure):
+    _fields_ = [
+        ("n_pipelines", ctypes.c_int32),
+        ("n_stages", ctypes.c_int32),
+        ("stage_params", ctypes.POINTER(ctypes.c_int64)),
+        ("alpha", ctypes.c_float),
+        ("beta", ctypes.c_float),
+        ("rho", ctypes.c_float),
+        ("lr", ctypes.c_float),
+        ("momentum", ctypes.c_float),
+        ("weight_decay", ctypes.c_float),
+        ("nesterov", ctypes.c_int32),
+        ("layout", ctypes.c_int32),
+        ("rank", ctypes.c_int32),
+        ("world", ctypes.c_int32),
+        ("device", ctypes.c_int32),
+        ("kernel_variant", ctypes.c_int32),
+    ]
+
+
+class EAOp(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("micro_batch", ctypes.c_int32)]
+
+
+# name -> (restype, argtypes); mirrors include/ea.h one to one.
+_VP = ctypes.c_void_p
+_FPP = ctypes.POINTER(ctypes.c_void_p)
+SIGNATURES = {
+    "ea_abi_version": (ctypes.c_int32, []),
+    "ea_get_unique_id": (ctypes.c_int, [ctypes.c_void_p]),
+    "ea_init": (ctypes.c_int, [ctypes.POINTER(EAConfig), ctypes.c_void_p, ctypes.POINTER(_VP)]),
+    "ea_center_capacity": (ctypes.c_int64, [_VP, ctypes.c_int32]),
+    "ea_shard_elems": (ctypes.c_int64, [_VP, ctypes.c_int32]),
+    "ea_step": (ctypes.c_int, [_VP, ctypes.c_int32, _FPP, _FPP, _VP, _VP]),
+    "ea_sync": (ctypes.c_int, [_VP, _VP]),
+    "ea_spread_local": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP, _VP, _VP]),
+    "ea_spread_apply": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP]),
+    "ea_get_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, ctypes.POINTER(_VP)]),
+    "ea_set_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, _VP, _VP]),
+    "ea_set_hyper": (ctypes.c_int, [_VP, ctypes.c_float, ctypes.c_float, ctypes.c_float, ctypes.c_float,
+                                    ctypes.c_float, ctypes.c_float, ctypes.c_int32]),
+    "ea_destroy": (ctypes.c_int, [_VP]),
+    "ea_last_error": (ctypes.c_char_p, [_VP]),
+    "ea_schedule": (ctypes.c_int32, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
+                                     ctypes.POINTER(EAOp), ctypes.c_int32]),
+}
+
+_lib = None
+
+
+def load_library(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load (once) and type the C ABI.  Raises LibraryNotBuilt if absent."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise LibraryNotBuilt(f"{path} not found: run `python -m paper_conf_ppopp_chen0qz23_b200.build` "
+                              "(or __graft_entry__.build()); there is no CPU fallback")
+    try:
+        import torch  # noqa: F401  -- map torch's libnccl.so.2 first so one NCCL is loaded
+    except Exception:
+        pass
+    lib = ctypes.CDLL(path, mode=ctypes.RTLD_GLOBAL)
+    for name, (res, args) in SIGNATURES.items():
+        fn = getattr(lib, name)
+        fn.restype = res
+        fn.argtypes = args
+    if lib.ea_abi_version() != ABI_VERSION:
+        raise LibraryNotBuilt(f"ABI version mismatch: library {lib.ea_abi_version()} vs binding {ABI_VERSION}")
+    _lib = lib
+    return lib
+
+
+def last_error(handle=None) -> str:
+    return (load_library().ea_last_error(handle) or b"").decode()
+
+
+def _check(status: int, handle=None):
+    if status != EA_OK:
+        raise EAError(status, last_error(handle))
+
+
+def get_unique_id() -> bytes:
+    buf = (ctypes.c_uint8 * UNIQUE_ID_BYTES)()
+    _check(load_library().ea_get_unique_id(buf))
+    return bytes(buf)
+
+
+def schedule(K: int, M: int, stage: int, advance: int) -> List[Tuple[str, int]]:
+    """Advance-forward order of `stage` (0-based) as [('F'|'B', micro_batch)]."""
+    lib = load_library()
+    cap = max(2 * M, 0)
+    out = (EAOp * max(cap, 1))()
+    n = lib.ea_schedule(K, M, stage, advance, out, cap)
+    if n < 0:
+        raise EAError(-n, f"ea_schedule(K={K}, M={M}, stage={stage}, advance={advance}) rejected")
+    return [("F" if out[i].kind == 0 else "B", out[i].micro_batch) for i in range(n)]
+
+
+def _stream_ptr(stream) -> Optional[int]:
+    import torch
+    if stream is None:
+        stream = torch.cuda.current_stream()
+    return stream.cuda_stream
+
+
+def _ptr(t, what: str) -> int:
+    import torch
+    if not isinstance(t, torch.Tensor) or t.dtype != torch.float32 or not t.is_cuda or not t.is_contiguous():
+        raise TypeError(f"{what} must be a contiguous float32 CUDA tensor")
+    return t.data_ptr()
+
+
+class ElasticAveraging:
+    """Handle over ``ea_init`` for the stages this process hosts.
+
+    stage_params: P_s per hosted stage.  alpha defaults to 1/N.
+    layout "colocated": all N replicas of a stage on this GPU; "spread": one
+    replica per rank, world == N, center sharded (needs ``nccl_id``)."""
+
+    def __init__(self, stage_params: Sequence[int], n_pipelines: int, *, alpha: Optional[float] = None,
+                 beta: float = 0.0, rho: float = 1.0, lr: float = 0.05, momentum: float = 0.0,
+                 weight_decay: float = 0.0, nesterov: bool = False, layout: str = "colocated", rank: int = 0,
+                 world: int = 1, device: Optional[int] = None, kernel_variant: str = "auto",
+                 nccl_id: Optional[bytes] = None):
+        import torch
+        self._lib = load_library()
+        self.n = int(n_pipelines)
+        self.stage_params = [int(p) for p in stage_params]
+        self.layout = layout
+        if device is None:
+            device = torch.cuda.current_device()
+        self.device = int(device)
+        self._sp = (ctypes.c_int64 * len(self.stage_params))(*self.stage_params)
+        cfg = EAConfig(self.n, len(self.stage_params), self._sp,
+                       1.0 / self.n if alpha is None else float(alpha), float(beta), float(rho), float(lr),
+                       float(momentum), float(weight_decay), int(bool(nesterov)), LAYOUTS[layout], int(rank),
+                       int(world), self.device, VARIANTS[kernel_variant])
+        self.rank, self.world = int(rank), int(world)
+        idbuf = None
+        if nccl_id is not None:
+            if len(nccl_id) != UNIQUE_ID_BYTES:
+                raise ValueError("nccl_id must be 128 bytes")
+            idbuf = (ctypes.c_uint8 * UNIQUE_ID_BYTES).from_buffer_copy(nccl_id)
+        h = ctypes.c_void_p()
+        _check(self._lib.ea_init(ctypes.byref(cfg), idbuf, ctypes.byref(h)))
+        self._h = h
+
+    # -- queries
+    def center_capacity(self, stage: int) -> int:
+        v = self._lib.ea_center_capacity(self._h, stage)
+        if v < 0:
+            raise EAError(EA_EINVAL, f"bad stage {stage}")
+        return v
+
+    def shard_elems(self, stage: int) -> int:
+        v = self._lib.ea_shard_elems(self._h, stage)
+        if v < 0:
+            raise EAError(EA_EINVAL, f"bad stage {stage}")
+        return v
+
+    # -- the step
+    def step(self, stage: int, replicas, grads, center, stream=None):
+        reps = list(replicas)
+        gs = list(grads)
+        rp = (ctypes.c_void_p * max(len(reps), 1))(*[_ptr(t, "replica") for t in reps])
+        gp = (ctypes.c_void_p * max(len(gs), 1))(*[_ptr(t, "grad") for t in gs])
+        want = self.n if self.layout == "colocated" else 1
+        if len(reps) != want or len(gs) != want:
+            raise ValueError(f"need {want} replica and gradient tensors, got {len(reps)}/{len(gs)}")
+        _check(self._lib.ea_step(self._h, stage, rp, gp, _ptr(center, "center"), _stream_ptr(stream)), self._h)
+
+    def sync(self, stream=None):
+        _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)
+
+    def spread_local(self, stage: int, replica, grad, center, contrib, stream=None):
+        _check(self._lib.ea_spread_local(self._h, stage, _ptr(replica, "replica"), _ptr(grad, "grad"),
+                                         _ptr(center, "center"), _ptr(contrib, "contrib"), _stream_ptr(stream)),
+               self._h)
+
+    def spread_apply(self, stage: int, center_shard, reduced, stream=None):
+        _check(self._lib.ea_spread_apply(self._h, stage, _ptr(center_shard, "center_shard"),
+                                         _ptr(reduced, "reduced"), _stream_ptr(stream)), self._h)
+
+    # -- optimizer state
+    def momentum(self, stage: int, replica: int):
+        """A torch view of the library-owned momentum of (stage, replica)."""
+        import torch
+        ptr = ctypes.c_void_p()
+        _check(self._lib.ea_get_state(self._h, stage, replica, ctypes.byref(ptr)), self._h)
+        return _device_view(ptr.value, self.stage_params[stage], self.device)
+
+    def set_momentum(self, stage: int, replica: int, src, stream=None):
+        _check(self._lib.ea_set_state(self._h, stage, replica, _ptr(src, "momentum"), _stream_ptr(stream)),
+               self._h)
+
+    def set_hyper(self, *, alpha, beta, rho, lr, momentum, weight_decay=0.0, nesterov=False):
+        _check(self._lib.ea_set_hyper(self._h, alpha, beta, rho, lr, momentum, weight_decay, int(bool(nesterov))),
+               self._h)
+
+    def close(self):
+        if getattr(self, "_h", None) is not None and self._h.value:
+            self._lib.ea_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *exc):
+        self.close()
+
+
+def _device_view(ptr: int, n: int, device: int):
+    """Zero-copy float32 torch view of library-owned device memory."""
+    import torch
+
+    class _Arr:
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "<f4", "data": (ptr, False), "version": 3,
+                                    "strides": None}
+
+    return torch.as_tensor(_Arr(), device=f"cuda:{device}")

@@ -1,0 +1,49 @@
+"""Parity helpers: run the CUDA path (through the C ABI) and the float64
+oracle on the same seeded inputs and compare with the c13 metric.
+
+c13: for each tensor T,
+    max_j |T_gpu[j] - T_ref[j]| / max(|T_ref[j]|, rms(T_ref))  <=  1e-5
+after the run.  The rms floor is what makes the north star's "max relative
+error 1e-5" attainable in fp32 at all: a pure elementwise ratio is dominated by
+elements that pass near zero (DESIGN.md derives the budget: ~100 steps x a few
+fp32 roundings of 6e-8 each -> ~1.5e-6 measured in an fp32 numpy model).
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from oracle.ea_oracle import Hyper, ea_step
+from paper_conf_ppopp_chen0qz23_b200 import synth
+
+TOL = 1e-5
+
+
+def rel_err(gpu: np.ndarray, ref: np.ndarray) -> float:
+    gpu = np.asarray(gpu, dtype=np.float64)
+    ref = np.asarray(ref, dtype=np.float64)
+    if ref.size == 0:
+        return 0.0
+    floor = float(np.sqrt(np.mean(ref * ref)))
+    denom = np.maximum(np.abs(ref), floor if floor > 0 else 1e-30)
+    return float(np.max(np.abs(gpu - ref) / denom))
+
+
+def to_np(t) -> np.ndarray:
+    return t.detach().cpu().numpy()
+
+
+def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nesterov=False):
+    a, b, r = synth.mode_coeffs(mode, n, alpha)
+    return Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=momentum, weight_decay=wd, nesterov=nesterov)
+
+
+class OracleStage:
+    """float64 oracle state of one stage."""
+
+    def __init__(self, reps, center):
+        self.xs = [np.asarray(x, dtype=np.float64) for x in reps]
+        self.ms = [np.zeros_like(self.xs[0]) for _ in reps]
+        self.c = np.asarray(center, dtype=np.float64)
+
+    def step(self, grads, hp):
+        self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)

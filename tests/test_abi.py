@@ -1,0 +1,153 @@
+"""C-ABI library: loads, exports every symbol include/ea.h declares, validates
+arguments before touching CUDA, and its host-only schedule generator (row a9)
+matches the oracle bit-exactly.  No GPU needed."""
+import ctypes
+import os
+import random
+import re
+import subprocess
+
+import pytest
+
+from oracle.schedule import advance_forward_schedule
+from paper_conf_ppopp_chen0qz23_b200 import binding
+from paper_conf_ppopp_chen0qz23_b200.build import build
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "ea.h")
+
+
+@pytest.fixture(scope="module")
+def lib():
+    build()
+    return binding.load_library()
+
+
+def header_functions():
+    text = open(HEADER).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(ea_[a-z_]+)\s*\(", text)))
+
+
+def test_header_lists_the_north_star_calls():
+    fns = header_functions()
+    for name in ("ea_init", "ea_step", "ea_sync", "ea_destroy", "ea_schedule", "ea_get_state", "ea_set_state",
+                 "ea_center_capacity", "ea_get_unique_id", "ea_last_error"):
+        assert name in fns
+
+
+def test_every_header_symbol_exported(lib):
+    out = subprocess.run(["nm", "-D", "--defined-only", binding.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r"\bT (ea_\w+)", out))
+    missing = [f for f in header_functions() if f not in exported]
+    assert not missing, missing
+    # and the binding types exactly those
+    assert set(binding.SIGNATURES) == set(header_functions())
+    # nothing else leaks (visibility=hidden)
+    assert exported == set(header_functions())
+
+
+def test_abi_version(lib):
+    assert lib.ea_abi_version() == binding.ABI_VERSION
+
+
+def test_config_struct_layout_matches_header():
+    # ea_config: 2 x int32, pointer, 6 floats, 6 int32  (x86-64 alignment)
+    assert ctypes.sizeof(binding.EAConfig) == 8 + 8 + 6 * 4 + 6 * 4
+    assert binding.EAConfig.stage_params.offset == 8
+    assert ctypes.sizeof(binding.EAOp) == 8
+
+
+def _cfg(**kw):
+    sp = (ctypes.c_int64 * 2)(1000, 1001)
+    base = dict(n_pipelines=2, n_stages=2, stage_params=sp, alpha=0.5, beta=0.0, rho=1.0, lr=0.05, momentum=0.9,
+                weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0)
+    base.update(kw)
+    c = binding.EAConfig(**base)
+    c._keep = sp
+    return c
+
+
+@pytest.mark.parametrize("kw,needle", [
+    (dict(n_pipelines=0), "n_pipelines"),
+    (dict(n_stages=0), "n_stages"),
+    (dict(alpha=1.5), "alpha"),
+    (dict(alpha=-0.1), "alpha"),
+    (dict(momentum=1.0), "momentum"),
+    (dict(weight_decay=-1.0), "weight_decay"),
+    (dict(nesterov=2), "nesterov"),
+    (dict(nesterov=1, momentum=0.0), "nesterov"),
+    (dict(layout=7), "layout"),
+    (dict(layout=1, world=3), "world"),
+    (dict(layout=1, world=2, rank=2), "rank"),
+    (dict(kernel_variant=9), "kernel_variant"),
+    (dict(n_pipelines=65), "N must be"),
+    (dict(lr=float("nan")), "finite"),
+])
+def test_init_rejects_bad_config(lib, kw, needle):
+    h = ctypes.c_void_p(123)
+    st = lib.ea_init(ctypes.byref(_cfg(**kw)), None, ctypes.byref(h))
+    assert st == binding.EA_EINVAL
+    assert h.value is None
+    assert needle in binding.last_error(None)
+
+
+def test_init_rejects_nonpositive_stage(lib):
+    sp = (ctypes.c_int64 * 2)(1000, 0)
+    c = _cfg(stage_params=sp)
+    h = ctypes.c_void_p()
+    assert lib.ea_init(ctypes.byref(c), None, ctypes.byref(h)) == binding.EA_EINVAL
+    assert lib.ea_init(None, None, ctypes.byref(h)) == binding.EA_EINVAL
+    assert lib.ea_init(ctypes.byref(c), None, None) == binding.EA_EINVAL
+
+
+def test_null_handle_paths(lib):
+    assert lib.ea_center_capacity(None, 0) == -1
+    assert lib.ea_shard_elems(None, 0) == -1
+    assert lib.ea_step(None, 0, None, None, None, None) == binding.EA_EINVAL
+    assert lib.ea_sync(None, None) == binding.EA_EINVAL
+    assert lib.ea_destroy(None) == binding.EA_OK
+    assert lib.ea_set_hyper(None, 0.5, 0, 1, 0.1, 0.9, 0, 0) == binding.EA_EINVAL
+    assert isinstance(lib.ea_last_error(None), bytes)
+
+
+@pytest.mark.skipif(__import__("torch").cuda.is_available(), reason="checks the no-GPU error path")
+def test_valid_config_without_gpu_reports_cuda_error(lib):
+    h = ctypes.c_void_p()
+    st = lib.ea_init(ctypes.byref(_cfg()), None, ctypes.byref(h))
+    assert st in (binding.EA_ECUDA, binding.EA_EINVAL)
+    assert h.value is None
+
+
+# ----------------------------------------------------------------- schedule (a9)
+def _oracle(K, M, stage, a):
+    return advance_forward_schedule(K, M, stage + 1, a)
+
+
+def test_schedule_bit_exact_exhaustive(lib):
+    for K in range(1, 9):
+        for M in range(0, 33):
+            for stage in range(K):
+                for a in range(-1, M + 2):
+                    assert binding.schedule(K, M, stage, a) == _oracle(K, M, stage, a), (K, M, stage, a)
+
+
+def test_schedule_bit_exact_sampled_large(lib):
+    rnd = random.Random(0)
+    for _ in range(3000):
+        K = rnd.randint(1, 16)
+        M = rnd.randint(0, 128)
+        stage = rnd.randrange(K)
+        a = rnd.randint(-2, M + 2)
+        assert binding.schedule(K, M, stage, a) == _oracle(K, M, stage, a)
+
+
+def test_schedule_rejects_bad_args(lib):
+    out = (binding.EAOp * 16)()
+    assert lib.ea_schedule(0, 4, 0, 1, out, 16) == -binding.EA_EINVAL
+    assert lib.ea_schedule(2, -1, 0, 1, out, 16) == -binding.EA_EINVAL
+    assert lib.ea_schedule(2, 4, 2, 1, out, 16) == -binding.EA_EINVAL
+    assert lib.ea_schedule(2, 4, -1, 1, out, 16) == -binding.EA_EINVAL
+    assert lib.ea_schedule(2, 9, 0, 1, out, 16) == -binding.EA_EINVAL      # cap < 2M
+    assert lib.ea_schedule(2, 4, 0, 1, None, 8) == -binding.EA_EINVAL
+    assert lib.ea_schedule(2, 0, 0, 1, None, 0) == 0

@@ -1,0 +1,269 @@
+"""GPU parity: the CUDA path through the C ABI vs the float64 oracle.
+
+Element by element on seeded synthetic inputs (paper_conf_ppopp_chen0qz23_b200.synth),
+c13 metric <= 1e-5 on every x_i, m_i and x~ (tests/_parity.py):
+  * C1 (2 pipelines x 2 stages, 1M params per stage) + the ragged-tail stage
+    P_s = 1,000,003, 100 steps, all three modes, both co-located kernels;
+  * N in {1, 3, 5, 8, 12}, ragged/tiny/empty-vector sizes, Nesterov, weight
+    decay, alpha in {0, 1};
+  * the spread decomposition (local kernel -> reduce-scatter -> shard update
+    -> all-gather) with N virtual ranks on one GPU, and the integrated NCCL
+    path at world = 1;
+  * optimizer-state get/set (checkpoint/resume) and set_hyper.
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ppopp_chen0qz23_b200 import synth
+from paper_conf_ppopp_chen0qz23_b200.binding import EAError, ElasticAveraging, get_unique_id
+from tests._parity import TOL, OracleStage, hyper, rel_err, to_np
+
+pytestmark = pytest.mark.gpu
+
+VARIANTS = ("regloop", "laneshfl")
+
+
+def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nesterov=False, wd=0.0, lr=synth.LR,
+                   momentum=synth.MOMENTUM, seed=0):
+    hp = hyper(n, mode, alpha=alpha, lr=lr, momentum=momentum, wd=wd, nesterov=nesterov)
+    dev = torch.device("cuda:0")
+    oracle, gstreams = [], []
+    gpu = {v: [] for v in variants}
+    handles = {}
+    for s, p in enumerate(sizes):
+        reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + 97 * seed + s)
+        oracle.append(OracleStage(reps, c))
+        gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + 97 * seed + s))
+        for v in variants:
+            gpu[v].append(([torch.from_numpy(x).to(dev) for x in reps], torch.from_numpy(c).to(dev)))
+    for v in variants:
+        handles[v] = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr,
+                                      momentum=hp.momentum, weight_decay=hp.weight_decay, nesterov=hp.nesterov,
+                                      kernel_variant=v)
+    gbuf = [[torch.empty(p, device=dev) for _ in range(n)] for p in sizes]
+    for t in range(steps):
+        for s in range(len(sizes)):
+            g = gstreams[s].next()
+            for i in range(n):
+                gbuf[s][i].copy_(torch.from_numpy(g[i]))
+            for v in variants:
+                reps, c = gpu[v][s]
+                handles[v].step(s, reps, gbuf[s], c)
+            oracle[s].step(g, hp)
+    torch.cuda.synchronize()
+    worst = 0.0
+    for v in variants:
+        for s in range(len(sizes)):
+            reps, c = gpu[v][s]
+            o = oracle[s]
+            errs = [rel_err(to_np(c), o.c)]
+            for i in range(n):
+                errs.append(rel_err(to_np(reps[i]), o.xs[i]))
+                errs.append(rel_err(to_np(handles[v].momentum(s, i)), o.ms[i]))
+            e = max(errs)
+            worst = max(worst, e)
+            assert e <= TOL, f"variant={v} stage={s} (P={sizes[s]}) rel err {e:.3e} > {TOL}"
+        handles[v].close()
+    return worst
+
+
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_c1_100_steps_with_ragged_tail(mode):
+    """C1 sizes, the P_s = 1,000,003 tail stage, 100 steps (north-star gate)."""
+    _run_colocated(2, [1_000_000, 1_000_003], 100, mode)
+
+
+@pytest.mark.parametrize("n", [1, 3, 5, 8, 12])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_replica_counts(n, mode):
+    _run_colocated(n, [65_539, 4097], 30, mode)
+
+
+@pytest.mark.parametrize("p", [1, 2, 3, 4, 5, 7, 31, 127, 1029, 4096 * 8 + 3])
+def test_tiny_and_ragged_sizes(p):
+    _run_colocated(3, [p], 12, "combined")
+    _run_colocated(4, [p], 5, "paper")
+
+
+@pytest.mark.parametrize("nesterov,wd", [(True, 0.0), (False, 1e-2), (True, 5e-3)])
+def test_nesterov_and_weight_decay(nesterov, wd):
+    _run_colocated(4, [300_001], 40, "combined", nesterov=nesterov, wd=wd)
+
+
+@pytest.mark.parametrize("alpha", [0.0, 1.0, 0.37])
+def test_alpha_edges(alpha):
+    _run_colocated(3, [100_003], 25, "easgd", alpha=alpha)
+    _run_colocated(3, [100_003], 25, "paper", alpha=alpha)
+
+
+def test_plain_sgd_momentum_zero():
+    _run_colocated(2, [10_000], 20, "paper", momentum=0.0)
+
+
+# ------------------------------------------------------------------ spread
+def _placement(rank, stage, n):
+    from paper_conf_ppopp_chen0qz23_b200.parallel import replica_of
+    return replica_of(rank, stage, n)
+
+
+@pytest.mark.parametrize("n", [2, 3, 4, 8])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_spread_decomposition_virtual_ranks(n, mode):
+    """N ranks on one GPU, external-collective mode: the real local and shard
+    kernels, with the reduce-scatter / all-gather done by the test."""
+    sizes = [200_003, 64]
+    steps = 20
+    hp = hyper(n, mode)
+    dev = torch.device("cuda:0")
+    hs = [ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                           layout="spread", rank=r, world=n) for r in range(n)]
+    oracle, gstreams, xs, centers = [], [], [], []
+    for s, p in enumerate(sizes):
+        reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
+        oracle.append(OracleStage(reps, c))
+        gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
+        cap = hs[0].center_capacity(s)
+        assert cap % (32 * n) == 0 and cap >= p
+        assert hs[0].shard_elems(s) * n == cap
+        cs = []
+        for r in range(n):
+            cr = torch.zeros(cap, device=dev)
+            cr[:p] = torch.from_numpy(c)
+            cs.append(cr)
+        centers.append(cs)
+        xs.append([torch.from_numpy(reps[_placement(r, s, n)]).to(dev) for r in range(n)])
+    for t in range(steps):
+        for s in reversed(range(len(sizes))):   # global stage order K-1 .. 0
+            p = sizes[s]
+            cap = hs[0].center_capacity(s)
+            shard = cap // n
+            g = gstreams[s].next()
+            contribs = []
+            for r in range(n):
+                gr = torch.from_numpy(g[_placement(r, s, n)]).to(dev)
+                cb = torch.full((cap,), float("nan"), device=dev)    # padding must be written as 0
+                hs[r].spread_local(s, xs[s][r], gr, centers[s][r], cb)
+                contribs.append(cb)
+            total = torch.stack(contribs).sum(0)                     # reduce-scatter (sum)
+            for r in range(n):
+                hs[r].spread_apply(s, centers[s][r][r * shard:(r + 1) * shard], total[r * shard:(r + 1) * shard])
+            for r in range(n):                                        # all-gather
+                for q in range(n):
+                    if q != r:
+                        centers[s][q][r * shard:(r + 1) * shard].copy_(centers[s][r][r * shard:(r + 1) * shard])
+            oracle[s].step(g, hp)
+    torch.cuda.synchronize()
+    for s, p in enumerate(sizes):
+        o = oracle[s]
+        for r in range(n):
+            i = _placement(r, s, n)
+            assert rel_err(to_np(xs[s][r]), o.xs[i]) <= TOL
+            assert rel_err(to_np(hs[r].momentum(s, 0)), o.ms[i]) <= TOL
+            assert rel_err(to_np(centers[s][r][:p]), o.c) <= TOL
+            assert torch.all(centers[s][r][p:] == 0), "center padding must stay zero"
+    for h in hs:
+        h.close()
+
+
+def test_spread_nccl_world1_and_stream_order():
+    """Integrated EA_SPREAD path (NCCL reduce-scatter / all-gather on the
+    library's side stream) at world = 1, driven from a non-default stream."""
+    sizes = [100_003, 5]
+    hp = hyper(1, "combined")
+    dev = torch.device("cuda:0")
+    h = ElasticAveraging(sizes, 1, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                         layout="spread", rank=0, world=1, nccl_id=get_unique_id())
+    stream = torch.cuda.Stream()
+    oracle, gstreams, xs, cs = [], [], [], []
+    for s, p in enumerate(sizes):
+        reps, c = synth.host_state(1, p, seed=synth.WEIGHT_SEED + s)
+        oracle.append(OracleStage(reps, c))
+        gstreams.append(synth.GradStream(1, p, seed=synth.GRAD_SEED + s))
+        cap = h.center_capacity(s)
+        cc = torch.zeros(cap, device=dev)
+        cc[:p] = torch.from_numpy(c)
+        cs.append(cc)
+        xs.append(torch.from_numpy(reps[0]).to(dev))
+    with torch.cuda.stream(stream):
+        for t in range(15):
+            for s in reversed(range(len(sizes))):
+                g = gstreams[s].next()
+                gd = torch.from_numpy(g[0]).to(dev, non_blocking=False)
+                h.step(s, [xs[s]], [gd], cs[s], stream=stream)
+                oracle[s].step(g, hp)
+        h.sync(stream)
+    stream.synchronize()
+    for s, p in enumerate(sizes):
+        assert rel_err(to_np(xs[s]), oracle[s].xs[0]) <= TOL
+        assert rel_err(to_np(cs[s][:p]), oracle[s].c) <= TOL
+        assert rel_err(to_np(h.momentum(s, 0)), oracle[s].ms[0]) <= TOL
+    with pytest.raises(EAError):
+        h.step(0, [xs[0][1:]], [xs[0][1:]], cs[0])   # misaligned pointers -> EA_EINVAL
+    h.close()
+
+
+def test_spread_external_mode_rejects_ea_step():
+    h = ElasticAveraging([1000], 2, layout="spread", rank=0, world=2)
+    x = torch.zeros(1000, device="cuda:0")
+    c = torch.zeros(h.center_capacity(0), device="cuda:0")
+    with pytest.raises(EAError, match="EA_ESTATE"):
+        h.step(0, [x], [x], c)
+    h.close()
+
+
+# ------------------------------------------------------------------ state & errors
+def test_state_roundtrip_and_set_hyper():
+    """Checkpoint the library-owned momentum, resume in a fresh handle, and
+    change the learning rate mid-run: must equal an uninterrupted oracle run."""
+    n, p = 3, 50_001
+    dev = torch.device("cuda:0")
+    hp1 = hyper(n, "combined")
+    hp2 = hyper(n, "combined", lr=0.01)
+    reps, c = synth.host_state(n, p)
+    o = OracleStage(reps, c)
+    gs = synth.GradStream(n, p)
+    xs = [torch.from_numpy(x).to(dev) for x in reps]
+    cc = torch.from_numpy(c).to(dev)
+    kw = dict(alpha=hp1.alpha, beta=hp1.beta, rho=hp1.rho, momentum=hp1.momentum)
+    h = ElasticAveraging([p], n, lr=hp1.lr, **kw)
+    for t in range(5):
+        g = gs.next()
+        h.step(0, xs, [torch.from_numpy(a).to(dev) for a in g], cc)
+        o.step(g, hp1)
+    saved = [h.momentum(0, i).clone() for i in range(n)]
+    h.close()
+    h2 = ElasticAveraging([p], n, lr=hp1.lr, **kw)
+    for i in range(n):
+        h2.set_momentum(0, i, saved[i])
+    h2.set_hyper(alpha=hp2.alpha, beta=hp2.beta, rho=hp2.rho, lr=hp2.lr, momentum=hp2.momentum)
+    for t in range(5):
+        g = gs.next()
+        h2.step(0, xs, [torch.from_numpy(a).to(dev) for a in g], cc)
+        o.step(g, hp2)
+    torch.cuda.synchronize()
+    assert rel_err(to_np(cc), o.c) <= TOL
+    for i in range(n):
+        assert rel_err(to_np(xs[i]), o.xs[i]) <= TOL
+        assert rel_err(to_np(h2.momentum(0, i)), o.ms[i]) <= TOL
+    h2.close()
+
+
+def test_bad_pointers_rejected_before_enqueue():
+    n, p = 2, 1000
+    h = ElasticAveraging([p], n)
+    x = [torch.zeros(p + 4, device="cuda:0") for _ in range(n)]
+    c = torch.zeros(p, device="cuda:0")
+    with pytest.raises(EAError, match="EA_EINVAL"):
+        h.step(0, [t[1:] for t in x], [t[:p] for t in x], c)          # 4-byte offset -> misaligned
+    with pytest.raises(EAError, match="EA_EINVAL"):
+        h.step(1, [t[:p] for t in x], [t[:p] for t in x], c)          # stage out of range
+    host = torch.zeros(p).pin_memory()
+    import ctypes
+    from paper_conf_ppopp_chen0qz23_b200 import binding
+    lib = binding.load_library()
+    arr = (ctypes.c_void_p * 2)(host.data_ptr(), host.data_ptr())
+    st = lib.ea_step(h._h, 0, arr, arr, c.data_ptr(), None)
+    assert st == binding.EA_EINVAL                                     # host memory is not device memory
+    h.sync()
+    h.close()
