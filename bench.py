@@ -41,6 +41,7 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
     ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl"), default="auto")
+    ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -162,7 +163,7 @@ def run_ours(args, rank, world, local):
                              layout="spread", rank=rank, world=world, device=local, nccl_id=uid)
         state = []
         for s, p in enumerate(sizes):
-            reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s + parallel.replica_of(rank, s, n))
+            reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s)   # same center on every rank
             cc = torch.zeros(h.center_capacity(s), device=dev)
             cc[:p] = c0
             state.append((reps, grads, cc))
@@ -173,7 +174,17 @@ def run_ours(args, rank, world, local):
         state = [(reps, grads, c) for (reps, c, grads) in state]
     order = parallel.stage_order(len(sizes))
 
+    batched = not spread and not args.per_stage
+
     def one_step(evs=None):
+        if batched:    # all stages in ONE launch (ea_step_many)
+            if evs is not None:
+                evs[0][0].record(stream)
+            h.step_many(order, [state[s][0] for s in order], [state[s][1] for s in order],
+                        [state[s][2] for s in order], stream=stream)
+            if evs is not None:
+                evs[0][1].record(stream)
+            return
         for s in order:
             reps, grads, c = state[s]
             if evs is not None:
@@ -192,8 +203,8 @@ def run_ours(args, rank, world, local):
     # per-launch events for the dominant kernel (co-located: every ea_step is one kernel)
     ev = None
     if not spread:
-        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in sizes]
-              for _ in range(args.steps)]
+        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+               for _ in (range(1) if batched else sizes)] for _ in range(args.steps)]
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
@@ -221,18 +232,20 @@ def run_ours(args, rank, world, local):
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
     if not spread:
         step_bytes = sum(bytes_colocated(n, p) for p in sizes)
-        kern_ms = [ev[k][s][0].elapsed_time(ev[k][s][1]) for k in range(args.steps) for s in range(len(sizes))]
-        # per launch, averaged over the (equal-sized) stages
-        per_launch_bytes = step_bytes / len(sizes)
+        launches_per_step = 1 if batched else len(sizes)
+        kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(launches_per_step)]
+        # per launch (batched: all stages; per-stage: averaged over the equal-sized stages)
+        per_launch_bytes = step_bytes / launches_per_step
         avg_ms = sum(kern_ms) / len(kern_ms)
         achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
-                           "kernel": "colocated_" + ("laneshfl" if args.variant == "laneshfl" else "regloop"),
+                           "kernel": "colocated_" + ("regloop" if args.variant == "regloop" else "laneshfl"),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
-        out["gpu_launches"] = args.steps * len(sizes)
+        out["gpu_launches"] = args.steps * launches_per_step
+        out["config"]["launch"] = "ea_step_many (1 launch/step)" if batched else "ea_step per stage"
     else:
         step_bytes = sum(bytes_spread_local(p) for p in sizes)
         nv_bytes = sum(2 * (n - 1) / n * 4 * h.center_capacity(s) for s in range(len(sizes)))

@@ -152,6 +152,17 @@ EA_API int64_t ea_shard_elems(ea_handle h, int32_t stage);
 EA_API ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
                   const float* const* grad_ptrs, float* center_ptr, void* stream);
 
+/* Several stages in one call, in the given order (e.g. all stages hosted
+ * here once the last backward is done).  stages: `count` distinct stage
+ * indices; replica_ptrs / grad_ptrs: count*R pointers, stage-major (R = N
+ * co-located, 1 spread); center_ptrs: `count` pointers.  EA_COLOCATED with
+ * N <= 8 updates up to 8 stages with ONE kernel launch whose persistent grid
+ * splits the concatenated work of all of them evenly; otherwise the stages
+ * are stepped one after another exactly as by ea_step.  Every argument is
+ * validated before anything is enqueued. */
+EA_API ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                              const float* const* grad_ptrs, float* const* center_ptrs, void* stream);
+
 /* Make `stream` wait until every center update enqueued so far is complete,
  * then report any asynchronous CUDA/NCCL error seen so far.  Does not block
  * the host. */

@@ -69,6 +69,7 @@ SIGNATURES = {
     "ea_center_capacity": (ctypes.c_int64, [_VP, ctypes.c_int32]),
     "ea_shard_elems": (ctypes.c_int64, [_VP, ctypes.c_int32]),
     "ea_step": (ctypes.c_int, [_VP, ctypes.c_int32, _FPP, _FPP, _VP, _VP]),
+    "ea_step_many": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP, _VP]),
     "ea_sync": (ctypes.c_int, [_VP, _VP]),
     "ea_spread_local": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP, _VP, _VP]),
     "ea_spread_apply": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP]),
@@ -206,6 +207,26 @@ class ElasticAveraging:
         if len(reps) != want or len(gs) != want:
             raise ValueError(f"need {want} replica and gradient tensors, got {len(reps)}/{len(gs)}")
         _check(self._lib.ea_step(self._h, stage, rp, gp, _ptr(center, "center"), _stream_ptr(stream)), self._h)
+
+    def step_many(self, stages, replicas, grads, centers, stream=None):
+        """Several stages in one call (one launch co-located, N <= 8).
+        replicas[j] / grads[j]: the tensors of stages[j]; centers[j] its center."""
+        stages = [int(s) for s in stages]
+        want = self.n if self.layout == "colocated" else 1
+        if not (len(replicas) == len(grads) == len(centers) == len(stages)):
+            raise ValueError("stages, replicas, grads, centers must have the same length")
+        rp, gp = [], []
+        for j in range(len(stages)):
+            if len(replicas[j]) != want or len(grads[j]) != want:
+                raise ValueError(f"stage {stages[j]}: need {want} replica and gradient tensors")
+            rp += [_ptr(t, "replica") for t in replicas[j]]
+            gp += [_ptr(t, "grad") for t in grads[j]]
+        k = max(len(stages), 1)
+        st = (ctypes.c_int32 * k)(*stages)
+        ra = (ctypes.c_void_p * max(len(rp), 1))(*rp)
+        ga = (ctypes.c_void_p * max(len(gp), 1))(*gp)
+        ca = (ctypes.c_void_p * k)(*[_ptr(c, "center") for c in centers])
+        _check(self._lib.ea_step_many(self._h, len(stages), st, ra, ga, ca, _stream_ptr(stream)), self._h)
 
     def sync(self, stream=None):
         _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)

@@ -223,9 +223,9 @@ int64_t ea_shard_elems(ea_handle h, int32_t stage) {
   return h->cfg.layout == EA_SPREAD ? h->p_pad[stage] / h->cfg.n_pipelines : h->p[stage];
 }
 
-ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
-                  float* center_ptr, void* stream) {
-  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+// Validates one stage's pointers (nothing enqueued on failure).
+static ea_status check_stage_ptrs(ea_ctx* h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
+                                  const float* center_ptr) {
   if (stage < 0 || stage >= h->cfg.n_stages) { set_err(h, "stage %d out of range", stage); return EA_EINVAL; }
   if (!replica_ptrs || !grad_ptrs) { set_err(h, "replica_ptrs / grad_ptrs is NULL"); return EA_EINVAL; }
   const int reps = replicas_here(h);
@@ -237,38 +237,68 @@ ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const 
   for (int i = 0; i < reps; ++i) {
     if (!replica_ptrs[i] || !grad_ptrs[i] || !aligned16(replica_ptrs[i]) || !aligned16(grad_ptrs[i]) ||
         !is_device_ptr(replica_ptrs[i], dev) || !is_device_ptr(grad_ptrs[i], dev)) {
-      set_err(h, "replica/grad pointer %d must be a 16-byte aligned device pointer on device %d", i, dev);
+      set_err(h, "stage %d: replica/grad pointer %d must be a 16-byte aligned device pointer on device %d", stage, i,
+              dev);
       return EA_EINVAL;
     }
   }
-  cudaError_t e = cudaSetDevice(dev);
-  if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
-  const int64_t ps = h->p[stage];
+  return EA_OK;
+}
 
-  if (h->cfg.layout == EA_COLOCATED) {
-    ea::ReplicaTable t;
-    for (int i = 0; i < reps; ++i) {
-      t.x[i] = replica_ptrs[i];
-      t.g[i] = grad_ptrs[i];
-      t.m[i] = h->mom[stage] + h->stride[stage] * i;
+// Co-located: `count` validated stages in as few launches as possible.
+static ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                                  const float* const* grad_ptrs, float* const* center_ptrs, cudaStream_t s) {
+  const int n = h->cfg.n_pipelines;
+  cudaError_t e = cudaSuccess;
+  if (n > ea::kMaxFusedN) {  // wide N: one launch per stage
+    for (int j = 0; j < count; ++j) {
+      const int st = stages[j];
+      ea::ReplicaTable t;
+      for (int i = 0; i < n; ++i) {
+        t.x[i] = replica_ptrs[j * n + i];
+        t.g[i] = grad_ptrs[j * n + i];
+        t.m[i] = h->mom[st] + h->stride[st] * i;
+      }
+      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, h->num_sms, s);
+      if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
     }
-    e = ea::launch_colocated(t, reps, center_ptr, ps, h->hp, h->variant, h->num_sms, s);
-    if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
     return EA_OK;
   }
+  for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
+    ea::StageBatch b;
+    b.nstages = 0;
+    for (int j = j0; j < count && j < j0 + ea::kMaxLaunchStages; ++j) {
+      const int st = stages[j];
+      ea::StageRefs& r = b.st[b.nstages++];
+      for (int i = 0; i < ea::kMaxFusedN; ++i) {
+        const bool on = i < n;
+        r.x[i] = on ? replica_ptrs[j * n + i] : nullptr;
+        r.g[i] = on ? grad_ptrs[j * n + i] : nullptr;
+        r.m[i] = on ? h->mom[st] + h->stride[st] * i : nullptr;
+      }
+      r.c = center_ptrs[j];
+      r.p = h->p[st];
+    }
+    e = ea::launch_colocated_batch(b, n, h->hp, h->variant, h->num_sms, s);
+    if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
+  }
+  return EA_OK;
+}
 
-  // EA_SPREAD: side stream: local kernel -> RS -> shard update -> in-place AG (rows a6-a8).
+// Spread: one stage's exchange on the side stream (rows a6-a8).
+static ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr,
+                             cudaStream_t s) {
   if (!h->comm) {
     set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
     return EA_ESTATE;
   }
+  cudaError_t e;
   const int n = h->cfg.n_pipelines;
   const int64_t pad = h->p_pad[stage], shard = pad / n;
   float* own = center_ptr + shard * h->cfg.rank;
   if ((e = cudaEventRecord(h->ev_in, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   if ((e = cudaStreamWaitEvent(h->side, h->ev_in, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  e = ea::launch_spread_local(replica_ptrs[0], grad_ptrs[0], h->mom[stage], center_ptr, h->contrib, ps, pad, h->hp,
+  e = ea::launch_spread_local(replica, grad, h->mom[stage], center_ptr, h->contrib, h->p[stage], pad, h->hp,
                               h->num_sms, h->side);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
   if ((e = cudaEventRecord(h->ev_local, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
@@ -281,6 +311,45 @@ ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const 
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
   // The caller's stream waits only for x_i (the next forward may start now).
   if ((e = cudaStreamWaitEvent(s, h->ev_local, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  return EA_OK;
+}
+
+ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
+                  float* center_ptr, void* stream) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  ea_status st = check_stage_ptrs(h, stage, replica_ptrs, grad_ptrs, center_ptr);
+  if (st != EA_OK) return st;
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->cfg.layout == EA_COLOCATED) return colocated_launch(h, 1, &stage, replica_ptrs, grad_ptrs, &center_ptr, s);
+  return spread_step(h, stage, replica_ptrs[0], grad_ptrs[0], center_ptr, s);
+}
+
+ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                       const float* const* grad_ptrs, float* const* center_ptrs, void* stream) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  if (count < 0 || (count > 0 && (!stages || !replica_ptrs || !grad_ptrs || !center_ptrs))) {
+    set_err(h, "ea_step_many: bad count or NULL array");
+    return EA_EINVAL;
+  }
+  const int reps = replicas_here(h);
+  for (int j = 0; j < count; ++j) {
+    for (int k = 0; k < j; ++k)
+      if (stages[k] == stages[j]) { set_err(h, "ea_step_many: stage %d listed twice", stages[j]); return EA_EINVAL; }
+    ea_status st = check_stage_ptrs(h, stages[j], replica_ptrs + (size_t)j * reps, grad_ptrs + (size_t)j * reps,
+                                    center_ptrs[j]);
+    if (st != EA_OK) return st;
+  }
+  if (count == 0) return EA_OK;
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  if (h->cfg.layout == EA_COLOCATED) return colocated_launch(h, count, stages, replica_ptrs, grad_ptrs, center_ptrs, s);
+  for (int j = 0; j < count; ++j) {
+    ea_status st = spread_step(h, stages[j], replica_ptrs[j], grad_ptrs[j], center_ptrs[j], s);
+    if (st != EA_OK) return st;
+  }
   return EA_OK;
 }
 

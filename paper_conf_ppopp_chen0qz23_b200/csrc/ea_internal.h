@@ -19,9 +19,27 @@ struct Hyper {
   float inv_n;     // 1/N (step 5 normalisation)
 };
 
-constexpr int kMaxReplicas = 64;
+constexpr int kMaxReplicas = 64;      // EA_MAX_REPLICAS
+constexpr int kMaxFusedN = 8;         // replicas handled by the compile-time-N kernels
+constexpr int kMaxLaunchStages = 8;   // stages fused into one launch
 
-// Pointer table of one co-located stage: N replicas, gradients, momenta.
+// One co-located stage as the kernels see it.
+struct StageRefs {
+  float* x[kMaxFusedN];
+  const float* g[kMaxFusedN];
+  float* m[kMaxFusedN];
+  float* c;
+  int64_t p;  // elements
+};
+
+// Up to kMaxLaunchStages stages updated by ONE launch (same N): the work of
+// all stages is concatenated and split evenly over the persistent grid.
+struct StageBatch {
+  StageRefs st[kMaxLaunchStages];
+  int nstages;
+};
+
+// Pointer table of one stage with up to kMaxReplicas replicas (N > 8 path).
 struct ReplicaTable {
   float* x[kMaxReplicas];
   const float* g[kMaxReplicas];
@@ -29,16 +47,20 @@ struct ReplicaTable {
 };
 
 enum KernelVariant : int {
-  kVariantAuto = 0,      // library picks (default: register-resident replica loop)
+  kVariantAuto = 0,      // library picks (see launch_colocated_batch)
   kVariantRegLoop = 1,   // one thread per float4 of center, loops over N replicas in registers
   kVariantLaneShfl = 2,  // lanes = (replica, float4 chunk); center tile staged by cp.async.bulk
                          // into shared memory; replica reduction by warp shuffles
 };
 
-// Co-located fused step (rows a1-a5): updates x_i, m_i for all replicas and
-// x~ in place.  p elements per vector; every pointer 16-byte aligned.
-cudaError_t launch_colocated(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
-                             int variant, int num_sms, cudaStream_t s);
+// Co-located fused step (rows a1-a5) for a batch of stages with the same N
+// (N <= kMaxFusedN): updates x_i, m_i and x~ of every stage in place, one launch.
+cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int variant, int num_sms,
+                                   cudaStream_t s);
+
+// Co-located step for one stage with any N <= kMaxReplicas (N > 8 path).
+cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
+                                  int num_sms, cudaStream_t s);
 
 // Spread local step (rows a1-a4 for one replica): updates x, m in place and
 // writes r = rho*Delta + beta*(x - x~) into contrib[0..p), zeros into

@@ -1,0 +1,84 @@
+"""Full-size parity on sampled outputs (the oracle is elementwise over j, so it
+can compute any sample of elements one by one).
+
+* C2 (BASELINE configs[1]: 25M params, K=4, N=4) in bench.py's launch
+  configuration (ea_step_many, default kernel): 3 steps, 200k sampled
+  elements per stage plus the first/last elements, checked after every step.
+* A stage larger than 2^31 elements (int64 indexing) with N=1 and N=2.
+"""
+import numpy as np
+import pytest
+import torch
+
+from oracle.ea_oracle import Hyper, ea_step
+from paper_conf_ppopp_chen0qz23_b200 import synth
+from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
+from tests._parity import TOL, rel_err
+
+pytestmark = pytest.mark.gpu
+
+
+def _sample_idx(p, k, rng):
+    idx = rng.choice(p, size=min(k, p), replace=False)
+    edge = np.r_[np.arange(min(8, p)), np.arange(max(p - 8, 0), p)]
+    return torch.from_numpy(np.unique(np.r_[idx, edge]).astype(np.int64))
+
+
+def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000):
+    dev = torch.device("cuda:0")
+    a, b, r = synth.mode_coeffs(mode, n)
+    hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
+    h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
+                         kernel_variant=variant)
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(7)
+    rng = np.random.default_rng(0)
+    state = []
+    for s, p in enumerate(sizes):
+        reps, c, grads = synth.device_state(n, p, dev, seed=s)
+        state.append((reps, c, grads, _sample_idx(p, k, rng).to(dev)))
+    order = list(reversed(range(len(sizes))))
+    f64 = lambda t, idx: t[idx].double().cpu().numpy()
+    for t in range(steps):
+        before = []
+        for s, (reps, c, grads, idx) in enumerate(state):
+            for g in grads:
+                g.normal_(0.0, synth.GRAD_STD, generator=gen)
+            before.append(([f64(x, idx) for x in reps], [f64(h.momentum(s, i), idx) for i in range(n)],
+                           f64(c, idx), [f64(g, idx) for g in grads]))
+        if many:
+            h.step_many(order, [state[s][0] for s in order], [state[s][2] for s in order],
+                        [state[s][1] for s in order])
+        else:
+            for s in order:
+                h.step(s, state[s][0], state[s][2], state[s][1])
+        torch.cuda.synchronize()
+        for s, (reps, c, grads, idx) in enumerate(state):
+            xs, ms, cc, gs = before[s]
+            ox, om, oc = ea_step(xs, ms, cc, gs, hp)
+            assert rel_err(f64(c, idx), oc) <= TOL, (s, t)
+            for i in range(n):
+                assert rel_err(f64(reps[i], idx), ox[i]) <= TOL, (s, t, i)
+                assert rel_err(f64(h.momentum(s, i), idx), om[i]) <= TOL, (s, t, i)
+    h.close()
+
+
+@pytest.mark.parametrize("variant", ["auto", "regloop"])
+def test_c2_full_size_sampled(variant):
+    cfg = synth.CONFIGS["C2"]
+    _run_sampled(cfg.n_pipelines, cfg.stage_sizes, 3, variant)
+
+
+def test_c2_full_size_per_stage_launches():
+    cfg = synth.CONFIGS["C2"]
+    _run_sampled(cfg.n_pipelines, cfg.stage_sizes, 2, "auto", many=False)
+
+
+@pytest.mark.parametrize("n,p", [(1, (1 << 31) + 5), (2, (1 << 30) + 3)])
+def test_beyond_int32_elements(n, p):
+    free, _ = torch.cuda.mem_get_info()
+    need = (3 * n + 1) * 4 * p * 1.2
+    if free < need:
+        pytest.skip(f"needs {need / 1e9:.0f} GB")
+    _run_sampled(n, [p], 1, "auto", k=100_000)
+    torch.cuda.empty_cache()

@@ -25,7 +25,7 @@ VARIANTS = ("regloop", "laneshfl")
 
 
 def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nesterov=False, wd=0.0, lr=synth.LR,
-                   momentum=synth.MOMENTUM, seed=0):
+                   momentum=synth.MOMENTUM, seed=0, many=False):
     hp = hyper(n, mode, alpha=alpha, lr=lr, momentum=momentum, wd=wd, nesterov=nesterov)
     dev = torch.device("cuda:0")
     oracle, gstreams = [], []
@@ -42,15 +42,21 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
                                       momentum=hp.momentum, weight_decay=hp.weight_decay, nesterov=hp.nesterov,
                                       kernel_variant=v)
     gbuf = [[torch.empty(p, device=dev) for _ in range(n)] for p in sizes]
+    order = list(reversed(range(len(sizes))))
     for t in range(steps):
         for s in range(len(sizes)):
             g = gstreams[s].next()
             for i in range(n):
                 gbuf[s][i].copy_(torch.from_numpy(g[i]))
-            for v in variants:
-                reps, c = gpu[v][s]
-                handles[v].step(s, reps, gbuf[s], c)
+            if not many:
+                for v in variants:
+                    reps, c = gpu[v][s]
+                    handles[v].step(s, reps, gbuf[s], c)
             oracle[s].step(g, hp)
+        if many:      # every stage in one ea_step_many call (one launch per <= 8 stages)
+            for v in variants:
+                handles[v].step_many(order, [gpu[v][s][0] for s in order], [gbuf[s] for s in order],
+                                     [gpu[v][s][1] for s in order])
     torch.cuda.synchronize()
     worst = 0.0
     for v in variants:
@@ -72,6 +78,32 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
 def test_c1_100_steps_with_ragged_tail(mode):
     """C1 sizes, the P_s = 1,000,003 tail stage, 100 steps (north-star gate)."""
     _run_colocated(2, [1_000_000, 1_000_003], 100, mode)
+
+
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_c1_step_many_one_launch(mode):
+    """C1 + tail stage, all stages in ONE launch per step (ea_step_many)."""
+    _run_colocated(2, [1_000_000, 1_000_003], 100, mode, many=True)
+
+
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 8, 12])
+def test_step_many_mixed_sizes_and_chunks(n):
+    """10 stages of mixed/ragged sizes: > kMaxLaunchStages (8) -> 2 launches;
+    tiny stages shorter than one tile or one float4."""
+    sizes = [100_003, 64, 3, 65_536, 7, 1, 4099, 250_000, 33, 12_345]
+    _run_colocated(n, sizes, 12, "combined", many=True)
+
+
+def test_step_many_rejects_duplicates_and_bad_stage():
+    h = ElasticAveraging([1000, 1000], 2)
+    x = [torch.zeros(1000, device="cuda:0") for _ in range(2)]
+    c = torch.zeros(1000, device="cuda:0")
+    with pytest.raises(EAError, match="twice"):
+        h.step_many([0, 0], [x, x], [x, x], [c, c])
+    with pytest.raises(EAError, match="EA_EINVAL"):
+        h.step_many([0, 2], [x, x], [x, x], [c, c])
+    h.step_many([], [], [], [])
+    h.close()
 
 
 @pytest.mark.parametrize("n", [1, 3, 5, 8, 12])
