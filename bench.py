@@ -40,7 +40,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl"), default="auto")
+    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
     ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
@@ -241,7 +241,7 @@ def run_ours(args, rank, world, local):
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
-                           "kernel": "colocated_" + ("regloop" if args.variant == "regloop" else "laneshfl"),
+                           "kernel": "colocated_" + ("laneshfl" if args.variant == "auto" else args.variant),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * launches_per_step
@@ -257,6 +257,8 @@ def run_ours(args, rank, world, local):
                                    "step time; peak = measured peer copy per direction"}
         out["gpu_launches"] = args.steps * 2 * len(sizes)
     out["clocks"] = clk.summary()
+    if not spread:
+        out["copy_gbs_same_box"] = same_box_copy_gbs(dev)
     if not spread and not args.no_e2e:
         out["e2e"] = e2e_colocated(h, state, sizes, n, args, stream, dev, order)
     elif spread:
@@ -268,6 +270,26 @@ def run_ours(args, rank, world, local):
         print(json.dumps(out), flush=True)
     if spread:
         dist.destroy_process_group()
+
+
+def same_box_copy_gbs(dev, nbytes=2 << 30, reps=10):
+    """torch copy_ of 2 GiB (read + write bytes / best time): this box's copy
+    bandwidth, for context next to MEASURED_PEAKS.json (same recipe)."""
+    import torch
+    a = torch.empty(nbytes // 2, dtype=torch.bfloat16, device=dev)
+    b = torch.empty_like(a)
+    best = None
+    for _ in range(reps + 2):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        b.copy_(a)
+        e1.record()
+        e1.synchronize()
+        t = e0.elapsed_time(e1)
+        best = t if best is None else min(best, t)
+    del a, b
+    torch.cuda.empty_cache()
+    return 2 * nbytes / (best * 1e-3) / 1e9
 
 
 def traffic_from_profiles(workload):

@@ -90,11 +90,12 @@ typedef struct {
   int32_t rank;                 /* EA_SPREAD: 0 <= rank < world; ignored otherwise */
   int32_t world;                /* EA_SPREAD: must equal n_pipelines; ignored otherwise */
   int32_t device;               /* CUDA device ordinal the handle binds to */
-  int32_t kernel_variant;       /* EA_COLOCATED kernel: 0 = library default, 1 = register-
-                                   resident replica loop, 2 = lane-per-replica with the center
-                                   tile staged by cp.async.bulk and warp-shuffle reduction
-                                   (N <= 8; larger N uses 1).  Same results up to fp32
-                                   summation order (DESIGN.md c14). */
+  int32_t kernel_variant;       /* EA_COLOCATED kernel (N <= 8; larger N has one kernel):
+                                   0 = library default, 1 = register-resident replica loop,
+                                   2 = lane-per-replica, center tile staged by cp.async.bulk,
+                                   warp-shuffle reduction, 3 = bulk-copy pipeline (every input
+                                   tile by cp.async.bulk into an mbarrier ring).  Same results
+                                   up to fp32 summation order (DESIGN.md c14). */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;

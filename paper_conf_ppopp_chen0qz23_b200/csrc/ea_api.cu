@@ -145,7 +145,7 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (c.world != c.n_pipelines) { set_err(nullptr, "EA_SPREAD needs world == n_pipelines"); return EA_EINVAL; }
     if (c.rank < 0 || c.rank >= c.world) { set_err(nullptr, "rank %d out of [0,%d)", c.rank, c.world); return EA_EINVAL; }
   }
-  if (c.kernel_variant < 0 || c.kernel_variant > 2) { set_err(nullptr, "kernel_variant must be 0, 1 or 2"); return EA_EINVAL; }
+  if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
   ea_status st = check_hyper(nullptr, c.alpha, c.beta, c.rho, c.lr, c.momentum, c.weight_decay, c.nesterov);
   if (st != EA_OK) return st;
   int ndev = 0;

@@ -51,6 +51,8 @@ enum KernelVariant : int {
   kVariantRegLoop = 1,   // one thread per float4 of center, loops over N replicas in registers
   kVariantLaneShfl = 2,  // lanes = (replica, float4 chunk); center tile staged by cp.async.bulk
                          // into shared memory; replica reduction by warp shuffles
+  kVariantBulkPipe = 3,  // every input tile streamed by cp.async.bulk into a multi-stage smem
+                         // ring (producer warp + mbarriers); consumers store from registers
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N

@@ -12,8 +12,9 @@
 // byte, far below the fp32 ridge, so every kernel here is HBM-bound and is
 // written for bytes in flight: 128-bit coalesced accesses, no shared-memory
 // round trips for data that is used once, persistent grids (#SMs x resident
-// blocks) over which the work of ALL stages of a launch is split evenly, so
-// no SM idles in a ragged last wave.  Tensor cores are not used (no contraction).
+// blocks) sweeping the stages of a launch in waves with the ragged remainder
+// split evenly (wave_item), so no SM idles in a partial last wave.  Tensor
+// cores are not used (no contraction).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -126,6 +127,53 @@ __device__ __forceinline__ void block_range(int64_t total, int64_t& lo, int64_t&
   hi = total * (blockIdx.x + 1) / gridDim.x;
 }
 
+// Wave schedule over the stages of a launch.  Chunks of C float4: in stage s
+// the grid sweeps full waves (chunk w*G + b for block b, so the G blocks of
+// a wave touch one contiguous window of every stream -- DRAM-page friendly),
+// then the ragged remainder R < G*C is split evenly over all G blocks (no
+// block idles in a partial last wave).  Every block walks the same sequence
+// of (stage, wave) items, so the cursor is warp- and block-uniform.
+struct WaveCursor {
+  int s;
+  int64_t w;
+};
+
+template <class NvecOf>
+__device__ __forceinline__ bool wave_item_f(int nstages, NvecOf nvec_of, int64_t C, WaveCursor& cur, int& s_out,
+                                            int64_t& v0, int64_t& nv) {
+  const int64_t G = gridDim.x, bid = blockIdx.x;
+  while (cur.s < nstages) {
+    const int64_t nvec = nvec_of(cur.s);
+    const int64_t waves = nvec / (G * C);
+    if (cur.w < waves) {
+      v0 = (cur.w * G + bid) * C;
+      nv = C;
+      s_out = cur.s;
+      ++cur.w;
+      return true;
+    }
+    if (cur.w == waves) {
+      const int64_t r0 = waves * G * C, R = nvec - r0;
+      const int64_t a = r0 + R * bid / G, e = r0 + R * (bid + 1) / G;
+      ++cur.w;
+      if (e > a) {
+        v0 = a;
+        nv = e - a;
+        s_out = cur.s;
+        return true;
+      }
+    }
+    ++cur.s;
+    cur.w = 0;
+  }
+  return false;
+}
+
+__device__ __forceinline__ bool wave_item(const StageBatch& b, int64_t C, WaveCursor& cur, int& s_out, int64_t& v0,
+                                          int64_t& nv) {
+  return wave_item_f(b.nstages, [&](int s) { return b.st[s].p / 4; }, C, cur, s_out, v0, nv);
+}
+
 // ============================================================================
 // Variant 1: register-resident replica loop.
 // One thread owns U float4 of a center; it issues all (3N+1)*U 128-bit loads
@@ -133,8 +181,7 @@ __device__ __forceinline__ void block_range(int64_t total, int64_t& lo, int64_t&
 // replica pointers may alias as far as the compiler knows, so the loads are
 // hoisted by hand), shares the center value across the N replicas in
 // registers, reduces the N contributions in registers and writes x_i, m_i
-// and x~ once.  Work unit: kUnitVec float4 (512 B); the units of all stages
-// of the launch are concatenated and split evenly over the persistent grid.
+// and x~ once.  Work unit: kThreads*U float4 per block, scheduled by wave_item.
 // ============================================================================
 constexpr int kUnitVec = 32;
 
@@ -181,22 +228,10 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
 template <int N, int U, int HINT>
 __global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b, const Hyper hp) {
   const Mem<HINT> mem;
-  int64_t begin[kMaxLaunchStages + 1];
-  begin[0] = 0;
-  for (int s = 0; s < b.nstages; ++s) begin[s + 1] = begin[s] + (b.st[s].p / 4 + kUnitVec - 1) / kUnitVec;
-  int64_t lo, hi;
-  block_range(begin[b.nstages], lo, hi);
-  int s = 0;
-  for (int64_t pos = lo; pos < hi;) {
-    while (pos >= begin[s + 1]) ++s;
-    const int64_t end = hi < begin[s + 1] ? hi : begin[s + 1];
-    const int64_t nvec = b.st[s].p / 4;
-    const int64_t va = (pos - begin[s]) * kUnitVec;
-    int64_t ve = (end - begin[s]) * kUnitVec;
-    if (ve > nvec) ve = nvec;
-    regloop_range<N, U, HINT>(b.st[s], va, ve, hp, mem);
-    pos = end;
-  }
+  WaveCursor cur{0, 0};
+  int s;
+  int64_t v0, nv;
+  while (wave_item(b, (int64_t)kThreads * U, cur, s, v0, nv)) regloop_range<N, U, HINT>(b.st[s], v0, v0 + nv, hp, mem);
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
     for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
 }
@@ -334,12 +369,6 @@ __global__ void __launch_bounds__(kThreads) colocated_laneshfl(const StageBatch 
   const int rep = lane / CH, chunk = lane % CH;
   const bool active = rep < N;
 
-  int64_t begin[kMaxLaunchStages + 1];
-  begin[0] = 0;
-  for (int s = 0; s < b.nstages; ++s) begin[s + 1] = begin[s] + (b.st[s].p / 4 + kTileVec - 1) / kTileVec;
-  int64_t lo, hi;
-  block_range(begin[b.nstages], lo, hi);
-
   if (threadIdx.x == 0) {
     mbar_init(&s_bar[0], 1);
     mbar_init(&s_bar[1], 1);
@@ -347,32 +376,26 @@ __global__ void __launch_bounds__(kThreads) colocated_laneshfl(const StageBatch 
   }
   __syncthreads();
 
-  auto locate = [&](int64_t tile, int& s, int64_t& v0, int64_t& nv) {
-    while (tile >= begin[s + 1]) ++s;
-    const int64_t nvec = b.st[s].p / 4;
-    v0 = (tile - begin[s]) * kTileVec;
-    nv = (nvec - v0) < kTileVec ? (nvec - v0) : kTileVec;
-  };
-  auto issue = [&](int64_t tile, int buf) {
-    int s = 0;
-    int64_t v0, nv;
-    locate(tile, s, v0, nv);
+  auto issue = [&](int s, int64_t v0, int64_t nv, int buf) {
     const uint32_t bytes = static_cast<uint32_t>(nv * 16);
     mbar_expect_tx(&s_bar[buf], bytes);
     bulk_g2s(&s_center[buf][0], b.st[s].c + 4 * v0, bytes, &s_bar[buf]);
   };
 
-  if (threadIdx.x == 0 && lo < hi) issue(lo, 0);
+  WaveCursor cur{0, 0};
+  int s, s_next;
+  int64_t v0, nv, v0_next, nv_next;
+  bool have = wave_item(b, kTileVec, cur, s, v0, nv);
+  if (threadIdx.x == 0 && have) issue(s, v0, nv, 0);
   uint32_t phase[2] = {0u, 0u};
-  int buf = 0, s = 0;
+  int buf = 0;
 
-  for (int64_t tile = lo; tile < hi; ++tile) {
-    if (threadIdx.x == 0 && tile + 1 < hi) {
+  while (have) {
+    const bool have_next = wave_item(b, kTileVec, cur, s_next, v0_next, nv_next);
+    if (threadIdx.x == 0 && have_next) {
       fence_proxy_async();  // buffer buf^1 was last read through the generic proxy
-      issue(tile + 1, buf ^ 1);
+      issue(s_next, v0_next, nv_next, buf ^ 1);
     }
-    int64_t v0, nv;
-    locate(tile, s, v0, nv);
     const StageRefs& st = b.st[s];
     float* xi = nullptr;
     const float* gi = nullptr;
@@ -418,9 +441,118 @@ __global__ void __launch_bounds__(kThreads) colocated_laneshfl(const StageBatch 
     }
     __syncthreads();  // everyone done reading s_center[buf] before it is refilled
     buf ^= 1;
+    have = have_next;
+    s = s_next;
+    v0 = v0_next;
+    nv = nv_next;
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
     for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
+}
+
+// ============================================================================
+// Variant 3: bulk-copy load pipeline (TMA engine feeds shared memory).
+//
+// One producer warp (one elected thread) streams every input of a tile --
+// x~ and x_i, g_i, m_i of all N replicas, (3N+1) 1-D cp.async.bulk copies of
+// kBulkTile float4 each -- into a kBulkStages-deep ring of shared-memory
+// slots, completing on a per-slot "full" mbarrier with the byte count.  Eight
+// consumer warps read a slot (one float4 column per thread: the x~ value is
+// shared by the N replica rows in registers), update in registers, write x_i,
+// m_i and x~ straight to HBM with 128-bit stores, and release the slot on its
+// "empty" mbarrier (one arrive per consumer warp).  Requests reach the memory
+// system as (3N+1) x 4 KB bulk reads per tile instead of 16-byte loads, and the
+// loads of up to kBulkStages tiles are in flight per SM with no registers
+// held for them.  Tiles follow the same wave schedule as the other variants.
+// ============================================================================
+constexpr int kBulkConsumerWarps = 8;
+constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
+
+template <int N>
+struct BulkGeom {
+  // float4 per array per tile: keep one slot <= ~56 KB
+  static constexpr int kTile = (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128;
+  static constexpr int kSlotVec = (3 * N + 1) * kTile;  // float4 per slot
+  static constexpr int kStages = (kSlotVec * 16 * 4 <= 200 * 1024) ? 4 : 3;
+  static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
+};
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+template <int N, int HINT>
+__global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
+  using G = BulkGeom<N>;
+  constexpr int T = G::kTile, S = G::kStages;
+  extern __shared__ __align__(128) float4 smem[];
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * G::kSlotVec);
+  uint64_t* empty = full + S;
+  const Mem<HINT> mem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], kBulkConsumerWarps);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+
+  if (warp == kBulkConsumerWarps) {
+    // ---------------- producer: one thread issues every bulk copy
+    if (lane == 0) {
+      WaveCursor cur{0, 0};
+      int s;
+      int64_t v0, nv;
+      for (int k = 0; wave_item(b, T, cur, s, v0, nv); ++k) {
+        const int slot = k % S;
+        mbar_wait(&empty[slot], ((k / S) & 1) ^ 1);
+        float4* base = smem + slot * G::kSlotVec;
+        const uint32_t bytes = static_cast<uint32_t>(nv * 16);
+        const StageRefs& st = b.st[s];
+        mbar_expect_tx(&full[slot], bytes * (3 * N + 1));
+        bulk_g2s(base, st.c + 4 * v0, bytes, &full[slot]);
+#pragma unroll
+        for (int i = 0; i < N; ++i) {
+          bulk_g2s(base + (1 + 3 * i) * T, st.x[i] + 4 * v0, bytes, &full[slot]);
+          bulk_g2s(base + (2 + 3 * i) * T, st.g[i] + 4 * v0, bytes, &full[slot]);
+          bulk_g2s(base + (3 + 3 * i) * T, st.m[i] + 4 * v0, bytes, &full[slot]);
+        }
+      }
+    }
+  } else {
+    // ---------------- consumers
+    WaveCursor cur{0, 0};
+    int s;
+    int64_t v0, nv;
+    for (int k = 0; wave_item(b, T, cur, s, v0, nv); ++k) {
+      const int slot = k % S;
+      mbar_wait(&full[slot], (k / S) & 1);
+      const float4* base = smem + slot * G::kSlotVec;
+      const StageRefs& st = b.st[s];
+      for (int lv = threadIdx.x; lv < nv; lv += 32 * kBulkConsumerWarps) {
+        const float4 c = base[lv];
+        float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+        const int64_t v = v0 + lv;
+#pragma unroll
+        for (int i = 0; i < N; ++i) {
+          float4 x = base[(1 + 3 * i) * T + lv];
+          const float4 g = base[(2 + 3 * i) * T + lv];
+          float4 m = base[(3 + 3 * i) * T + lv];
+          add4(acc, ea_vec(x, g, m, c, hp));
+          mem.st(st.x[i] + 4 * v, x);
+          mem.st(st.m[i] + 4 * v, m);
+        }
+        mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
+      }
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&empty[slot]);  // release: this warp's smem reads are done
+    }
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+      for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
+  }
 }
 
 // ============================================================================
@@ -433,10 +565,12 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
                                                          float* __restrict__ contrib, int64_t nvec, int64_t p,
                                                          int64_t p_pad, const Hyper hp) {
   const Mem<0> mem;
-  int64_t lo, hi;
-  block_range((nvec + kUnitVec - 1) / kUnitVec, lo, hi);
-  const int64_t va = lo * kUnitVec, ve = hi * kUnitVec < nvec ? hi * kUnitVec : nvec;
-  for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
+  WaveCursor cur{0, 0};
+  int sidx;
+  int64_t va0, nv0;
+  while (wave_item_f(1, [&](int) { return nvec; }, (int64_t)kThreads * U, cur, sidx, va0, nv0)) {
+    const int64_t va = va0, ve = va0 + nv0;
+    for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
     float4 xv[U], gv[U], mv[U], cv[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -458,6 +592,7 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
         mem.st(contrib + 4 * v, r);
       }
     }
+  }
   }
   // scalar tail of the vector part and the zero padding of the contribution
   const int64_t gtid = (int64_t)blockIdx.x * kThreads + threadIdx.x;
@@ -507,14 +642,29 @@ int l2_hint() {
   return v;
 }
 
-template <int N, int HINT>
-cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  constexpr int U = N <= 2 ? 4 : (N <= 4 ? 2 : 1);
+template <int N, int HINT, int U>
+cudaError_t launch_regloop_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   int64_t units = 0;
-  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kUnitVec - 1) / kUnitVec;
+  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kThreads * U - 1) / (kThreads * U);
   auto k = colocated_regloop<N, U, HINT>;
   k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
   return cudaGetLastError();
+}
+
+// Unroll knob for measurement: AVGPIPE_EA_REGLOOP_U=1 forces U=1 for N<=4.
+int regloop_u1() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_REGLOOP_U");
+    return (e && e[0] == '1') ? 1 : 0;
+  }();
+  return v;
+}
+
+template <int N, int HINT>
+cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  constexpr int U = N <= 2 ? 4 : (N <= 4 ? 2 : 1);
+  if (U > 1 && regloop_u1()) return launch_regloop_u<N, HINT, 1>(b, hp, num_sms, s);
+  return launch_regloop_u<N, HINT, U>(b, hp, num_sms, s);
 }
 
 template <int N, int HINT>
@@ -522,14 +672,32 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
   constexpr int kTileVec = LaneGeom<N>::kTileVec;
   int64_t units = 0;
   for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kTileVec - 1) / kTileVec;
+  if (units < 1) units = 1;
   auto k = colocated_laneshfl<N, HINT>;
   k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
+  return cudaGetLastError();
+}
+
+template <int N, int HINT>
+cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  using G = BulkGeom<N>;
+  auto k = colocated_bulkpipe<N, HINT>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
+  if (e != cudaSuccess) return e;
+  int64_t units = 0;
+  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + G::kTile - 1) / G::kTile;
+  int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
+  if (grid > units) grid = units;
+  if (grid < 1) grid = 1;
+  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp);
   return cudaGetLastError();
 }
 
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int variant, int num_sms, cudaStream_t s) {
   const bool hint = l2_hint() != 0;
+  if (variant == kVariantBulkPipe)
+    return hint ? launch_bulkpipe<N, 1>(b, hp, num_sms, s) : launch_bulkpipe<N, 0>(b, hp, num_sms, s);
   if (variant == kVariantRegLoop)
     return hint ? launch_regloop<N, 1>(b, hp, num_sms, s) : launch_regloop<N, 0>(b, hp, num_sms, s);
   return hint ? launch_laneshfl<N, 1>(b, hp, num_sms, s) : launch_laneshfl<N, 0>(b, hp, num_sms, s);

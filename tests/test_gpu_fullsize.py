@@ -63,7 +63,7 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
     h.close()
 
 
-@pytest.mark.parametrize("variant", ["auto", "regloop"])
+@pytest.mark.parametrize("variant", ["auto", "regloop", "laneshfl", "bulkpipe"])
 def test_c2_full_size_sampled(variant):
     cfg = synth.CONFIGS["C2"]
     _run_sampled(cfg.n_pipelines, cfg.stage_sizes, 3, variant)

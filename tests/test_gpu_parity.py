@@ -21,7 +21,7 @@ from tests._parity import TOL, OracleStage, hyper, rel_err, to_np
 
 pytestmark = pytest.mark.gpu
 
-VARIANTS = ("regloop", "laneshfl")
+VARIANTS = ("regloop", "laneshfl", "bulkpipe")
 
 
 def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nesterov=False, wd=0.0, lr=synth.LR,
