@@ -349,18 +349,18 @@ struct LanePow2 {
   static constexpr int value = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : 16;
 };
 
-template <int N>
+template <int N, int PASSES = kLanePasses>
 struct LaneGeom {
   static constexpr int NP = LanePow2<N>::value;
   static constexpr int CH = 32 / NP;                              // chunks per warp pass
-  static constexpr int kVecPerWarp = kLanePasses * CH;            // float4 of a tile per warp
+  static constexpr int kVecPerWarp = PASSES * CH;                 // float4 of a tile per warp
   static constexpr int kTileVec = (kThreads / 32) * kVecPerWarp;  // float4 of center per tile
 };
 
-template <int N, int HINT>
-__global__ void __launch_bounds__(kThreads) colocated_laneshfl(const StageBatch b, const Hyper hp) {
-  using G = LaneGeom<N>;
-  constexpr int CH = G::CH, kPasses = kLanePasses, kVecPerWarp = G::kVecPerWarp, kTileVec = G::kTileVec;
+template <int N, int HINT, int PASSES = kLanePasses, int MINB = 1>
+__global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const StageBatch b, const Hyper hp) {
+  using G = LaneGeom<N, PASSES>;
+  constexpr int CH = G::CH, kPasses = PASSES, kVecPerWarp = G::kVecPerWarp, kTileVec = G::kTileVec;
   __shared__ __align__(128) float4 s_center[2][kTileVec];
   __shared__ __align__(8) uint64_t s_bar[2];
   const Mem<HINT> mem;
@@ -667,8 +667,36 @@ cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_regloop_u<N, HINT, U>(b, hp, num_sms, s);
 }
 
+// Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4 only).
+int lane_tune() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_LANE_TUNE");
+    return e ? std::atoi(e) : 0;
+  }();
+  return v;
+}
+
+template <int N, int HINT, int PASSES, int MINB>
+cudaError_t launch_laneshfl_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  constexpr int kTileVec = LaneGeom<N, PASSES>::kTileVec;
+  int64_t units = 0;
+  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kTileVec - 1) / kTileVec;
+  if (units < 1) units = 1;
+  auto k = colocated_laneshfl<N, HINT, PASSES, MINB>;
+  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
+  return cudaGetLastError();
+}
+
 template <int N, int HINT>
 cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  if constexpr (N == 4 && HINT == 0) {
+    switch (lane_tune()) {
+      case 23: return launch_laneshfl_t<N, HINT, 2, 3>(b, hp, num_sms, s);
+      case 24: return launch_laneshfl_t<N, HINT, 2, 4>(b, hp, num_sms, s);
+      case 81: return launch_laneshfl_t<N, HINT, 8, 1>(b, hp, num_sms, s);
+      default: break;
+    }
+  }
   constexpr int kTileVec = LaneGeom<N>::kTileVec;
   int64_t units = 0;
   for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kTileVec - 1) / kTileVec;
