@@ -509,6 +509,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
       for (int k = 0; wave_item(b, T, cur, s, v0, nv); ++k) {
         const int slot = k % S;
         mbar_wait(&empty[slot], ((k / S) & 1) ^ 1);
+        fence_proxy_async();  // the consumers' generic-proxy reads of this slot precede the bulk writes
         float4* base = smem + slot * G::kSlotVec;
         const uint32_t bytes = static_cast<uint32_t>(nv * 16);
         const StageRefs& st = b.st[s];
@@ -623,13 +624,29 @@ __global__ void __launch_bounds__(kThreads) spread_apply(float* __restrict__ sha
 }
 
 // ---------------------------------------------------------------- launch helpers
+// Grid-size knob for co-scheduling with compute (row a8):
+// AVGPIPE_EA_GRID unset/0 = persistent (#SMs x occupancy); -1 = one work
+// chunk per CTA (short CTAs the block scheduler can interleave with other
+// streams' kernels); k > 0 = at most k CTAs.
+int grid_knob() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_GRID");
+    return e ? std::atoi(e) : 0;
+  }();
+  return v;
+}
+
 template <typename K>
 int persistent_grid(K kernel, int64_t work_units, int num_sms) {
   int per_sm = 0;
   if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kThreads, 0) != cudaSuccess || per_sm < 1)
     per_sm = 1;
   int64_t grid = (int64_t)num_sms * per_sm;
+  const int knob = grid_knob();
+  if (knob < 0) grid = work_units;
+  else if (knob > 0 && knob < grid) grid = knob;
   if (grid > work_units) grid = work_units;
+  if (grid > 0x7fffffff) grid = 0x7fffffff;
   return grid < 1 ? 1 : static_cast<int>(grid);
 }
 

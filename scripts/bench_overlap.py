@@ -61,8 +61,9 @@ def main():
         reps, c, g = synth.device_state(a.n, p, dev, seed=s)
         state.append((reps, g, c))
     order = list(reversed(range(a.stages)))
-    comp = torch.cuda.current_stream()
-    side = torch.cuda.Stream()
+    comp = torch.cuda.Stream(priority=-1)     # backward: high priority
+    side = torch.cuda.Stream(priority=0)      # EA: low priority (fills SM slots the GEMMs leave)
+    torch.cuda.set_stream(comp)
 
     def ea(stream):
         h.step_many(order, [state[s][0] for s in order], [state[s][1] for s in order], [state[s][2] for s in order],
@@ -104,6 +105,7 @@ def main():
     t_bwd, t_ea, t_ser, t_ovl = timed(bwd_only), timed(ea_only), timed(serial), timed(overlap)
     ea_bytes = sum((20 * a.n + 8) * p for p in sizes)
     out = {"what": "a8 stream overlap (1 GPU, co-located EA step on a side stream vs bf16 GEMM backward)",
+           "grid_knob": os.environ.get("AVGPIPE_EA_GRID", "0"),
            "n": a.n, "stages": a.stages, "params_per_stage": a.params, "tokens": a.tokens, "layers": a.layers,
            "micro_batches": a.micro, "t_bwd_ms": t_bwd, "t_ea_ms": t_ea, "t_serial_ms": t_ser, "t_overlap_ms": t_ovl,
            "exposed_ea_ms": t_ovl - t_bwd, "hidden_fraction": 1 - (t_ovl - t_bwd) / t_ea,
