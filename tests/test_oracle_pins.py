@@ -268,3 +268,66 @@ def test_inputs_not_modified_and_fixed_point():
         np.testing.assert_array_equal(nx[i], x)
         np.testing.assert_array_equal(xs[i], x)
     np.testing.assert_array_equal(nc, x)
+
+
+# ---------------------------------------------------------------- Adam / AdamW (row f1, reading c21)
+from oracle.ea_oracle import ea_step_adam  # noqa: E402
+
+
+@pytest.mark.parametrize("decoupled,wd", [(False, 0.0), (False, 1e-2), (True, 1e-2), (True, 0.0)])
+@pytest.mark.parametrize("beta,rho", [(0.0, 1.0), (2.0, 0.0)])
+def test_p1_adam_alpha0_is_independent_torch_adam(decoupled, wd, beta, rho):
+    """alpha = 0 => N independent torch.optim.Adam / AdamW trajectories (library routine)."""
+    rng = np.random.default_rng(21)
+    n, p, steps, lr = 2, 300, 15, 1e-3
+    xs, _, c = _rand_state(rng, n, p)
+    gs = _grads(rng, n, p, steps)
+    hp = Hyper(alpha=0.0, beta=beta, rho=rho, lr=lr, weight_decay=wd, beta1=0.9, beta2=0.999, eps=1e-8)
+    ox = [x.copy() for x in xs]
+    om = [np.zeros(p) for _ in range(n)]
+    ov = [np.zeros(p) for _ in range(n)]
+    oc = c.copy()
+    for t in range(steps):
+        ox, om, ov, oc = ea_step_adam(ox, om, ov, oc, gs[t], hp, t + 1, decoupled)
+    for i in range(n):
+        w = torch.nn.Parameter(torch.tensor(xs[i], dtype=torch.float64))
+        cls = torch.optim.AdamW if decoupled else torch.optim.Adam
+        opt = cls([w], lr=lr, betas=(0.9, 0.999), eps=1e-8, weight_decay=wd)
+        for t in range(steps):
+            w.grad = torch.tensor(gs[t][i], dtype=torch.float64)
+            opt.step()
+        np.testing.assert_allclose(ox[i], w.detach().numpy(), rtol=1e-12, atol=1e-16)
+        np.testing.assert_allclose(om[i], opt.state[w]["exp_avg"].numpy(), rtol=1e-12, atol=1e-18)
+        np.testing.assert_allclose(ov[i], opt.state[w]["exp_avg_sq"].numpy(), rtol=1e-12, atol=1e-20)
+
+
+@pytest.mark.parametrize("decoupled", [False, True])
+def test_p3_adam_center_stays_the_average(decoupled):
+    """'stays the average' holds whatever the optimizer (rho = 1)."""
+    rng = np.random.default_rng(22)
+    n, p = 3, 200
+    xs, _, _ = _rand_state(rng, n, p)
+    c = np.mean(xs, axis=0)
+    hp = Hyper(alpha=1 / n, beta=0.5, rho=1.0, lr=1e-3, weight_decay=1e-2)
+    ms = [np.zeros(p)] * n
+    vs = [np.zeros(p)] * n
+    for t, g in enumerate(_grads(rng, n, p, 30)):
+        xs, ms, vs, c = ea_step_adam(xs, ms, vs, c, g, hp, t + 1, decoupled)
+        np.testing.assert_allclose(c, np.mean(xs, axis=0), rtol=0, atol=1e-15)
+
+
+def test_p2_adam_zero_gradients_decay():
+    """Zero gradients and zero moments: Delta = 0, so the P2 closed forms hold for Adam too."""
+    rng = np.random.default_rng(23)
+    n, p, alpha = 4, 50, 0.1
+    xs, _, c = _rand_state(rng, n, p)
+    c = c + 1e-3
+    hp = Hyper(alpha=alpha, beta=n * alpha, rho=1.0, lr=1e-3)
+    d0 = np.mean(xs, axis=0) - c
+    total0 = sum(xs) + c
+    ms = [np.zeros(p)] * n
+    vs = [np.zeros(p)] * n
+    for t in range(10):
+        xs, ms, vs, c = ea_step_adam(xs, ms, vs, c, [np.zeros(p)] * n, hp, t + 1)
+    np.testing.assert_allclose(np.mean(xs, axis=0) - c, (1 - alpha - n * alpha) ** 10 * d0, rtol=1e-9, atol=1e-16)
+    np.testing.assert_allclose(sum(xs) + c, total0, rtol=0, atol=1e-13)
