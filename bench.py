@@ -41,6 +41,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
     ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
+    ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw"), default="sgd",
+                    help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
     ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
@@ -129,15 +131,17 @@ def workload_key(gpus: int, override):
 
 
 # ----------------------------------------------------------------------------- our arm
-def bytes_colocated(n, p):
-    """Algorithmic HBM bytes of one co-located launch: read x~ and x_i, g_i,
-    m_i of every replica, write x_i, m_i and x~ (fp32): (20 N + 8) P."""
-    return (20 * n + 8) * p
+def bytes_colocated(n, p, optimizer="sgd"):
+    """Algorithmic HBM bytes of one co-located launch (fp32): read x~ and, per
+    replica, x_i, g_i and the optimizer state; write x_i, the state and x~.
+    SGD-momentum (one state vector): (20 N + 8) P; Adam(W) (two): (28 N + 8) P."""
+    return ((20 if optimizer == "sgd" else 28) * n + 8) * p
 
 
-def bytes_spread_local(p):
-    """HBM bytes of the spread local kernel: read x, g, m, x~; write x, m, r: 28 P."""
-    return 28 * p
+def bytes_spread_local(p, optimizer="sgd"):
+    """HBM bytes of the spread local kernel: read x, g, state, x~; write x, state, r:
+    28 P (SGD) / 36 P (Adam)."""
+    return (28 if optimizer == "sgd" else 36) * p
 
 
 def run_ours(args, rank, world, local):
@@ -154,13 +158,15 @@ def run_ours(args, rank, world, local):
     n = cfg.n_pipelines if world == 1 else world
     sizes = cfg.stage_sizes
     a, b, r = synth.mode_coeffs(MODE, n)
+    lr = synth.LR if args.optimizer == "sgd" else 1e-3
     stream = torch.cuda.current_stream(dev)
     spread = world > 1
     if spread:
         dist.init_process_group("nccl", device_id=dev)
         uid = parallel.broadcast_unique_id()
-        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
-                             layout="spread", rank=rank, world=world, device=local, nccl_id=uid)
+        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
+                             layout="spread", rank=rank, world=world, device=local, nccl_id=uid,
+                             optimizer=args.optimizer)
         state = []
         for s, p in enumerate(sizes):
             reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s)   # same center on every rank
@@ -168,8 +174,8 @@ def run_ours(args, rank, world, local):
             cc[:p] = c0
             state.append((reps, grads, cc))
     else:
-        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
-                             device=local, kernel_variant=args.variant)
+        h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
+                             device=local, kernel_variant=args.variant, optimizer=args.optimizer)
         state = [synth.device_state(n, p, dev, seed=s) for s, p in enumerate(sizes)]
         state = [(reps, grads, c) for (reps, c, grads) in state]
     order = parallel.stage_order(len(sizes))
@@ -228,10 +234,11 @@ def run_ours(args, rank, world, local):
     ws_bytes = (n * 3 + 1) * 4 * total_params if not spread else 5 * 4 * total_params
     out["config"] = {"workload": cfg.name, "n_pipelines": n, "n_stages": len(sizes), "params": total_params,
                      "stage_params": sizes, "layout": "spread" if spread else "colocated", "mode": MODE,
-                     "optimizer": "sgd-momentum(0.9)", "kernel": args.variant,
+                     "optimizer": "sgd-momentum(0.9)" if args.optimizer == "sgd" else args.optimizer,
+                     "kernel": args.variant,
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
     if not spread:
-        step_bytes = sum(bytes_colocated(n, p) for p in sizes)
+        step_bytes = sum(bytes_colocated(n, p, args.optimizer) for p in sizes)
         launches_per_step = 1 if batched else len(sizes)
         kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(launches_per_step)]
         # per launch (batched: all stages; per-stage: averaged over the equal-sized stages)
@@ -241,13 +248,15 @@ def run_ours(args, rank, world, local):
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
-                           "kernel": "colocated_" + ("laneshfl" if args.variant == "auto" else args.variant),
+                           "kernel": "colocated_" + ("laneshfl" if args.variant == "auto" or args.optimizer != "sgd"
+                                                     else args.variant) + ("" if args.optimizer == "sgd"
+                                                                           else "<" + args.optimizer + ">"),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * launches_per_step
         out["config"]["launch"] = "ea_step_many (1 launch/step)" if batched else "ea_step per stage"
     else:
-        step_bytes = sum(bytes_spread_local(p) for p in sizes)
+        step_bytes = sum(bytes_spread_local(p, args.optimizer) for p in sizes)
         nv_bytes = sum(2 * (n - 1) / n * 4 * h.center_capacity(s) for s in range(len(sizes)))
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         nv_gbs = nv_bytes / (ms * 1e-3) / 1e9
@@ -301,20 +310,17 @@ def traffic_from_profiles(workload):
 
 
 def e2e_colocated(h, state, sizes, n, args, stream, dev, order):
-    """Same step through the same API, gradients copied from pinned host memory
-    before each stage's update and the new center copied back after it."""
+    """Same step through the public API with HOST buffers: ea_step_many_host
+    takes the gradients from pinned host memory and writes the new centers
+    back to pinned host memory every step (the library pipelines H2D, kernel
+    and D2H in 4 Mi-element chunks on its own copy streams)."""
     import torch
     host_g = [[g.cpu().pin_memory() for g in grads] for (_, grads, _) in state]
     host_c = [torch.empty(p, dtype=torch.float32).pin_memory() for p in sizes]
-    dev_g = [[torch.empty_like(g) for g in grads] for (_, grads, _) in state]
 
     def step():
-        for s in order:
-            reps, _, c = state[s]
-            for i in range(n):
-                dev_g[s][i].copy_(host_g[s][i], non_blocking=True)
-            h.step(s, reps, dev_g[s], c, stream=stream)
-            host_c[s].copy_(c, non_blocking=True)
+        h.step_many_host(order, [state[s][0] for s in order], [host_g[s] for s in order],
+                         [state[s][2] for s in order], [host_c[s] for s in order], stream=stream)
 
     for _ in range(3):
         step()
@@ -328,7 +334,8 @@ def e2e_colocated(h, state, sizes, n, args, stream, dev, order):
     ms = t0.elapsed_time(t1) / args.e2e_steps
     return {"value": n * sum(sizes) / (ms * 1e-3), "unit": UNIT, "ms_per_step": ms,
             "h2d_bytes_per_step": 4 * n * sum(sizes), "d2h_bytes_per_step": 4 * sum(sizes),
-            "path": "binding ElasticAveraging.step; pinned host grads -> device, center -> pinned host"}
+            "path": "ea_step_many_host: pinned host grads -> device (chunked, copy stream), fused kernel per chunk, "
+                    "center chunks -> pinned host (second copy stream)"}
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs

@@ -9,11 +9,15 @@
  *   reference ("center") model x~ is co-partitioned with them.  For
  *   every element j, with x~ = x~_t and all right-hand sides at step t:
  *
- *     Step 1  local update of a user-specified optimizer -- here SGD
- *                     with momentum, PyTorch convention (buffer starts at 0,
- *                     dampening 0):
+ *     Step 1  local update of a user-specified optimizer (ea_optimizer),
+ *                     PyTorch conventions:
+ *                     SGD+momentum (buffer starts at 0, dampening 0):
  *                       g' = g_i + lambda*x_i;  m_i <- mu*m_i + g';
  *                       Delta_i = -lr * (nesterov ? g' + mu*m_i : m_i)
+ *                     Adam / AdamW (t = the stage's step count; DESIGN.md c21):
+ *                       m <- b1 m + (1-b1) g';  v <- b2 v + (1-b2) g'^2;
+ *                       Delta_i = -(lr/(1-b1^t)) m / (sqrt(v)/sqrt(1-b2^t) + eps)
+ *                       (Adam: g' = g + lambda x;  AdamW: g' = g, Delta -= lr lambda x)
  *     Step 2  dilution in the ratio (1-alpha):alpha plus the local update:
  *                       x_i <- (1-alpha)*x_i + alpha*x~ + Delta_i
  *     Step 3/4  send and accumulate the contribution
@@ -60,7 +64,7 @@ extern "C" {
 #define EA_API
 #endif
 
-#define EA_ABI_VERSION 1
+#define EA_ABI_VERSION 2
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 
@@ -75,6 +79,10 @@ typedef enum {
 
 typedef enum { EA_COLOCATED = 0, EA_SPREAD = 1 } ea_layout;
 
+/* Local optimizer of Step 1 ("a user-specified optimizer"; the paper
+ * trains with Adam and SGD). */
+typedef enum { EA_OPT_SGD = 0, EA_OPT_ADAM = 1, EA_OPT_ADAMW = 2 } ea_optimizer;
+
 typedef struct {
   int32_t n_pipelines;          /* N >= 1 parallel pipelines */
   int32_t n_stages;             /* stages hosted by this process, >= 1 */
@@ -82,10 +90,10 @@ typedef struct {
   float alpha;                  /* dilution rate in [0,1], P:112 (default 1/N) */
   float beta;                   /* center pull (EASGD); 0 in the paper's mode */
   float rho;                    /* weight of Delta_i in the contribution; 1 in the paper's mode */
-  float lr;                     /* SGD learning rate eta */
-  float momentum;               /* mu in [0,1) */
-  float weight_decay;           /* lambda >= 0 (L2, added to the gradient) */
-  int32_t nesterov;             /* 0/1 */
+  float lr;                     /* learning rate eta */
+  float momentum;               /* SGD: mu in [0,1) */
+  float weight_decay;           /* lambda >= 0 (SGD/Adam: L2 added to the gradient; AdamW: decoupled) */
+  int32_t nesterov;             /* SGD: 0/1 */
   int32_t layout;               /* ea_layout */
   int32_t rank;                 /* EA_SPREAD: 0 <= rank < world; ignored otherwise */
   int32_t world;                /* EA_SPREAD: must equal n_pipelines; ignored otherwise */
@@ -95,7 +103,11 @@ typedef struct {
                                    2 = lane-per-replica, center tile staged by cp.async.bulk,
                                    warp-shuffle reduction, 3 = bulk-copy pipeline (every input
                                    tile by cp.async.bulk into an mbarrier ring).  Same results
-                                   up to fp32 summation order (DESIGN.md c14). */
+                                   up to fp32 summation order (DESIGN.md c14).  Adam(W) always
+                                   uses 2 (or the N > 8 kernel). */
+  int32_t optimizer;            /* ea_optimizer */
+  float beta1, beta2;           /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999) */
+  float eps;                    /* Adam(W): denominator epsilon > 0 (torch default 1e-8) */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;
@@ -164,6 +176,20 @@ EA_API ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
 EA_API ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
                               const float* const* grad_ptrs, float* const* center_ptrs, void* stream);
 
+/* End-to-end variant of ea_step_many for callers whose gradients live in HOST
+ * memory (EA_COLOCATED): host_grad_ptrs are count*N host pointers (pinned
+ * memory gives asynchronous, full-duplex copies), replica_ptrs / center_ptrs
+ * device pointers as in ea_step_many, host_center_out `count` host buffers of
+ * P_s floats that receive the updated centers.  The library streams the
+ * gradients through double-buffered device staging in chunks of 4 Mi
+ * elements on its own copy streams, runs the fused kernel on each chunk as it
+ * lands (on `stream`) and copies each finished center chunk back on a second
+ * copy stream, so H2D, kernel and D2H overlap.  When `stream` reaches the end
+ * of this work, host_center_out is complete.  EA_ESTATE for EA_SPREAD. */
+EA_API ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                                   const float* const* host_grad_ptrs, float* const* center_ptrs,
+                                   float* const* host_center_out, void* stream);
+
 /* Make `stream` wait until every center update enqueued so far is complete,
  * then report any asynchronous CUDA/NCCL error seen so far.  Does not block
  * the host. */
@@ -186,20 +212,28 @@ EA_API ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard
 
 /* ---- Optimizer state (checkpoint / resume) ---- */
 
-/* *momentum_dev = device pointer to the momentum of (stage, replica): P_s
- * floats, owned by the library, valid until ea_destroy.  EA_SPREAD: replica
- * must be 0. */
-EA_API ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, float** momentum_dev);
+/* *state_dev = device pointer to optimizer-state slot `slot` of (stage,
+ * replica): P_s floats, owned by the library, valid until ea_destroy.
+ * slot 0 = SGD momentum / Adam first moment, slot 1 = Adam second moment
+ * (EA_EINVAL for SGD).  EA_SPREAD: replica must be 0. */
+EA_API ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, float** state_dev);
 
-/* Copy P_s floats from device pointer momentum_src into the momentum of
- * (stage, replica), ordered on `stream`. */
-EA_API ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, const float* momentum_src,
-                       void* stream);
+/* Copy P_s floats from device pointer src into state slot `slot` of (stage,
+ * replica), ordered on `stream` (after pending EA_SPREAD side-stream work). */
+EA_API ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, const float* src,
+                              void* stream);
 
-/* Replace the hyper-parameters (e.g. a learning-rate schedule); same
- * validation as ea_init.  Takes effect for steps enqueued afterwards. */
-EA_API ea_status ea_set_hyper(ea_handle h, float alpha, float beta, float rho, float lr, float momentum,
-                       float weight_decay, int32_t nesterov);
+/* Step count t of `stage` (number of ea_step / ea_spread_local calls so far;
+ * Adam's bias correction uses t+1 for the next step). */
+EA_API ea_status ea_get_step(ea_handle h, int32_t stage, int64_t* step);
+EA_API ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step);
+
+/* Replace the hyper-parameters (alpha, beta, rho, lr, momentum, weight_decay,
+ * nesterov, beta1, beta2, eps) from cfg, e.g. for a learning-rate schedule;
+ * same validation as ea_init; optimizer, n_pipelines and layout must equal
+ * the handle's (other fields are ignored).  Takes effect for steps enqueued
+ * afterwards. */
+EA_API ea_status ea_set_hyper(ea_handle h, const ea_config* cfg);
 
 /* Wait for outstanding work, free everything the library owns, destroy the
  * communicator.  NULL is a no-op. */

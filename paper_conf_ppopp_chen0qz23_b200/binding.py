@@ -21,8 +21,9 @@ EA_COLOCATED, EA_SPREAD = 0, 1
 STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA_ESTATE", 5: "EA_ENOMEM"}
 LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
 VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3}
+OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2}
 UNIQUE_ID_BYTES = 128
-ABI_VERSION = 1
+ABI_VERSION = 2
 
 
 class LibraryNotBuilt(RuntimeError):
@@ -52,6 +53,10 @@ class EAConfig(ctypes.Structure):
         ("world", ctypes.c_int32),
         ("device", ctypes.c_int32),
         ("kernel_variant", ctypes.c_int32),
+        ("optimizer", ctypes.c_int32),
+        ("beta1", ctypes.c_float),
+        ("beta2", ctypes.c_float),
+        ("eps", ctypes.c_float),
     ]
 
 
@@ -70,13 +75,16 @@ SIGNATURES = {
     "ea_shard_elems": (ctypes.c_int64, [_VP, ctypes.c_int32]),
     "ea_step": (ctypes.c_int, [_VP, ctypes.c_int32, _FPP, _FPP, _VP, _VP]),
     "ea_step_many": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP, _VP]),
+    "ea_step_many_host": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP,
+                                         _FPP, _VP]),
     "ea_sync": (ctypes.c_int, [_VP, _VP]),
     "ea_spread_local": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP, _VP, _VP]),
     "ea_spread_apply": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP]),
-    "ea_get_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, ctypes.POINTER(_VP)]),
-    "ea_set_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, _VP, _VP]),
-    "ea_set_hyper": (ctypes.c_int, [_VP, ctypes.c_float, ctypes.c_float, ctypes.c_float, ctypes.c_float,
-                                    ctypes.c_float, ctypes.c_float, ctypes.c_int32]),
+    "ea_get_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.POINTER(_VP)]),
+    "ea_set_state": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, _VP, _VP]),
+    "ea_get_step": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int64)]),
+    "ea_set_step": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.c_int64]),
+    "ea_set_hyper": (ctypes.c_int, [_VP, ctypes.POINTER(EAConfig)]),
     "ea_destroy": (ctypes.c_int, [_VP]),
     "ea_last_error": (ctypes.c_char_p, [_VP]),
     "ea_schedule": (ctypes.c_int32, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
@@ -149,6 +157,13 @@ def _ptr(t, what: str) -> int:
     return t.data_ptr()
 
 
+def _host_ptr(t, what: str) -> int:
+    import torch
+    if not isinstance(t, torch.Tensor) or t.dtype != torch.float32 or t.is_cuda or not t.is_contiguous():
+        raise TypeError(f"{what} must be a contiguous float32 CPU tensor (pinned for asynchronous copies)")
+    return t.data_ptr()
+
+
 class ElasticAveraging:
     """Handle over ``ea_init`` for the stages this process hosts.
 
@@ -160,7 +175,7 @@ class ElasticAveraging:
                  beta: float = 0.0, rho: float = 1.0, lr: float = 0.05, momentum: float = 0.0,
                  weight_decay: float = 0.0, nesterov: bool = False, layout: str = "colocated", rank: int = 0,
                  world: int = 1, device: Optional[int] = None, kernel_variant: str = "auto",
-                 nccl_id: Optional[bytes] = None):
+                 nccl_id: Optional[bytes] = None, optimizer: str = "sgd", betas=(0.9, 0.999), eps: float = 1e-8):
         import torch
         self._lib = load_library()
         self.n = int(n_pipelines)
@@ -170,10 +185,13 @@ class ElasticAveraging:
             device = torch.cuda.current_device()
         self.device = int(device)
         self._sp = (ctypes.c_int64 * len(self.stage_params))(*self.stage_params)
+        self.optimizer = optimizer
         cfg = EAConfig(self.n, len(self.stage_params), self._sp,
                        1.0 / self.n if alpha is None else float(alpha), float(beta), float(rho), float(lr),
                        float(momentum), float(weight_decay), int(bool(nesterov)), LAYOUTS[layout], int(rank),
-                       int(world), self.device, VARIANTS[kernel_variant])
+                       int(world), self.device, VARIANTS[kernel_variant], OPTIMIZERS[optimizer],
+                       float(betas[0]), float(betas[1]), float(eps))
+        self._cfg = cfg
         self.rank, self.world = int(rank), int(world)
         idbuf = None
         if nccl_id is not None:
@@ -228,6 +246,24 @@ class ElasticAveraging:
         ca = (ctypes.c_void_p * k)(*[_ptr(c, "center") for c in centers])
         _check(self._lib.ea_step_many(self._h, len(stages), st, ra, ga, ca, _stream_ptr(stream)), self._h)
 
+    def step_many_host(self, stages, replicas, host_grads, centers, host_centers_out, stream=None):
+        """ea_step_many with gradients in (pinned) host tensors and the new
+        centers copied back into host tensors; copies and kernels overlap."""
+        stages = [int(s) for s in stages]
+        rp, gp = [], []
+        for j in range(len(stages)):
+            if len(replicas[j]) != self.n or len(host_grads[j]) != self.n:
+                raise ValueError(f"stage {stages[j]}: need {self.n} replica and gradient tensors")
+            rp += [_ptr(t, "replica") for t in replicas[j]]
+            gp += [_host_ptr(t, "host grad") for t in host_grads[j]]
+        k = max(len(stages), 1)
+        st = (ctypes.c_int32 * k)(*stages)
+        ra = (ctypes.c_void_p * max(len(rp), 1))(*rp)
+        ga = (ctypes.c_void_p * max(len(gp), 1))(*gp)
+        ca = (ctypes.c_void_p * k)(*[_ptr(c, "center") for c in centers])
+        oa = (ctypes.c_void_p * k)(*[_host_ptr(c, "host center out") for c in host_centers_out])
+        _check(self._lib.ea_step_many_host(self._h, len(stages), st, ra, ga, ca, oa, _stream_ptr(stream)), self._h)
+
     def sync(self, stream=None):
         _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)
 
@@ -241,20 +277,42 @@ class ElasticAveraging:
                                          _ptr(reduced, "reduced"), _stream_ptr(stream)), self._h)
 
     # -- optimizer state
-    def momentum(self, stage: int, replica: int):
-        """A torch view of the library-owned momentum of (stage, replica)."""
-        import torch
+    def state(self, stage: int, replica: int, slot: int = 0):
+        """Zero-copy torch view of library-owned optimizer state: slot 0 = SGD
+        momentum / Adam first moment, slot 1 = Adam second moment."""
         ptr = ctypes.c_void_p()
-        _check(self._lib.ea_get_state(self._h, stage, replica, ctypes.byref(ptr)), self._h)
+        _check(self._lib.ea_get_state(self._h, stage, replica, slot, ctypes.byref(ptr)), self._h)
         return _device_view(ptr.value, self.stage_params[stage], self.device)
 
-    def set_momentum(self, stage: int, replica: int, src, stream=None):
-        _check(self._lib.ea_set_state(self._h, stage, replica, _ptr(src, "momentum"), _stream_ptr(stream)),
+    def momentum(self, stage: int, replica: int):
+        return self.state(stage, replica, 0)
+
+    def set_state(self, stage: int, replica: int, src, slot: int = 0, stream=None):
+        _check(self._lib.ea_set_state(self._h, stage, replica, slot, _ptr(src, "state"), _stream_ptr(stream)),
                self._h)
 
-    def set_hyper(self, *, alpha, beta, rho, lr, momentum, weight_decay=0.0, nesterov=False):
-        _check(self._lib.ea_set_hyper(self._h, alpha, beta, rho, lr, momentum, weight_decay, int(bool(nesterov))),
-               self._h)
+    def set_momentum(self, stage: int, replica: int, src, stream=None):
+        self.set_state(stage, replica, src, 0, stream)
+
+    def get_step(self, stage: int) -> int:
+        t = ctypes.c_int64()
+        _check(self._lib.ea_get_step(self._h, stage, ctypes.byref(t)), self._h)
+        return t.value
+
+    def set_step(self, stage: int, step: int):
+        _check(self._lib.ea_set_step(self._h, stage, int(step)), self._h)
+
+    def set_hyper(self, **kw):
+        """Change hyper-parameters (alpha, beta, rho, lr, momentum, weight_decay,
+        nesterov, beta1, beta2, eps) for the steps enqueued afterwards."""
+        cfg = EAConfig.from_buffer_copy(self._cfg)
+        for k, v in kw.items():
+            if k not in ("alpha", "beta", "rho", "lr", "momentum", "weight_decay", "nesterov", "beta1", "beta2",
+                         "eps"):
+                raise KeyError(k)
+            setattr(cfg, k, int(bool(v)) if k == "nesterov" else float(v))
+        _check(self._lib.ea_set_hyper(self._h, ctypes.byref(cfg)), self._h)
+        self._cfg = cfg
 
     def close(self):
         if getattr(self, "_h", None) is not None and self._h.value:

@@ -1,14 +1,16 @@
 // C-ABI layer of the elastic-averaging library (declared in include/ea.h).
 //
-// Owns: the handle, per-stage momentum (zero-initialised, P:112 Step 1
-// optimizer state), and for EA_SPREAD the side stream, events, contribution
-// scratch and the NCCL communicator that replace the paper's reference
-// process and message queues.  Validates every argument before
-// enqueuing anything; never throws or aborts.
+// Owns: the handle, per-stage optimizer state (zero-initialised, P:112 Step 1:
+// SGD momentum, or Adam's two moments plus the per-stage step count), and for
+// EA_SPREAD the side stream, events, contribution scratch and the NCCL
+// communicator that replace the paper's reference process and message queues
+// (P:112-116).  Validates every argument before enqueuing anything; never
+// throws or aborts.
 #include <cuda_runtime.h>
 #include <nccl.h>
 #include <stdint.h>
 
+#include <cmath>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -26,16 +28,24 @@ struct ea_ctx {
   int num_sms = 148;
   std::vector<int64_t> p;       // P_s
   std::vector<int64_t> p_pad;   // center capacity
-  std::vector<int64_t> stride;  // momentum row stride (floats)
-  std::vector<float*> mom;      // per stage: [replicas][stride]
+  std::vector<int64_t> stride;  // optimizer-state row stride (floats)
+  std::vector<float*> state[2]; // per stage: [replicas][stride]; slot 0 = momentum / Adam m, slot 1 = Adam v
+  std::vector<int64_t> steps;   // per-stage step count t (Adam bias correction)
   // EA_SPREAD
   cudaStream_t side = nullptr;
   cudaEvent_t ev_in = nullptr, ev_local = nullptr, ev_done = nullptr;
   float* contrib = nullptr;  // max P_pad floats
   float* reduced = nullptr;  // max P_pad/N floats
   ncclComm_t comm = nullptr;
+  // host-buffer path (ea_step_many_host), allocated on first use
+  cudaStream_t h2d = nullptr, d2h = nullptr;
+  float* staging[2] = {nullptr, nullptr};  // N * kHostChunk floats each
+  cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_d2h = nullptr;
   std::string err;
 };
+
+// Elements per pipelined chunk of the host-buffer path (a multiple of 64).
+constexpr int64_t kHostChunk = 4 << 20;
 
 namespace {
 
@@ -65,14 +75,26 @@ bool is_device_ptr(const void* p, int device) {
   return a.type == cudaMemoryTypeDevice && a.device == device;
 }
 
-ea_status check_hyper(ea_ctx* h, float alpha, float beta, float rho, float lr, float momentum, float wd, int nesterov) {
-  auto finite = [](float v) { return v == v && v - v == 0.f; };
-  if (!(alpha >= 0.f && alpha <= 1.f)) { set_err(h, "alpha must be in [0,1] (P:112), got %g", alpha); return EA_EINVAL; }
-  if (!finite(beta) || !finite(rho) || !finite(lr)) { set_err(h, "beta, rho, lr must be finite"); return EA_EINVAL; }
-  if (!(momentum >= 0.f && momentum < 1.f)) { set_err(h, "momentum must be in [0,1), got %g", momentum); return EA_EINVAL; }
-  if (!(wd >= 0.f) || !finite(wd)) { set_err(h, "weight_decay must be finite and >= 0"); return EA_EINVAL; }
-  if (nesterov != 0 && nesterov != 1) { set_err(h, "nesterov must be 0 or 1"); return EA_EINVAL; }
-  if (nesterov && momentum <= 0.f) { set_err(h, "nesterov needs momentum > 0 (torch.optim.SGD rule)"); return EA_EINVAL; }
+bool finite(float v) { return v == v && v - v == 0.f; }
+
+ea_status check_hyper(ea_ctx* h, const ea_config& c) {
+  if (!(c.alpha >= 0.f && c.alpha <= 1.f)) { set_err(h, "alpha must be in [0,1] (P:112), got %g", c.alpha); return EA_EINVAL; }
+  if (!finite(c.beta) || !finite(c.rho) || !finite(c.lr)) { set_err(h, "beta, rho, lr must be finite"); return EA_EINVAL; }
+  if (!(c.weight_decay >= 0.f) || !finite(c.weight_decay)) { set_err(h, "weight_decay must be finite and >= 0"); return EA_EINVAL; }
+  if (c.optimizer == EA_OPT_SGD) {
+    if (!(c.momentum >= 0.f && c.momentum < 1.f)) { set_err(h, "momentum must be in [0,1), got %g", c.momentum); return EA_EINVAL; }
+    if (c.nesterov != 0 && c.nesterov != 1) { set_err(h, "nesterov must be 0 or 1"); return EA_EINVAL; }
+    if (c.nesterov && c.momentum <= 0.f) { set_err(h, "nesterov needs momentum > 0 (torch.optim.SGD rule)"); return EA_EINVAL; }
+  } else if (c.optimizer == EA_OPT_ADAM || c.optimizer == EA_OPT_ADAMW) {
+    if (!(c.beta1 >= 0.f && c.beta1 < 1.f) || !(c.beta2 >= 0.f && c.beta2 < 1.f)) {
+      set_err(h, "Adam betas must be in [0,1), got %g, %g", c.beta1, c.beta2);
+      return EA_EINVAL;
+    }
+    if (!(c.eps > 0.f) || !finite(c.eps)) { set_err(h, "Adam eps must be finite and > 0"); return EA_EINVAL; }
+  } else {
+    set_err(h, "unknown optimizer %d", c.optimizer);
+    return EA_EINVAL;
+  }
   return EA_OK;
 }
 
@@ -81,7 +103,29 @@ ea::Hyper make_hyper(const ea_config& c) {
   hp.alpha = c.alpha; hp.beta = c.beta; hp.rho = c.rho; hp.lr = c.lr;
   hp.momentum = c.momentum; hp.wd = c.weight_decay; hp.nesterov = c.nesterov;
   hp.inv_n = 1.0f / static_cast<float>(c.n_pipelines);
+  hp.beta1 = c.beta1; hp.one_minus_beta1 = static_cast<float>(1.0 - (double)c.beta1);
+  hp.beta2 = c.beta2; hp.one_minus_beta2 = static_cast<float>(1.0 - (double)c.beta2);
+  hp.eps = c.eps;
+  hp.lr_wd = static_cast<float>((double)c.lr * (double)c.weight_decay);
   return hp;
+}
+
+int state_slots(const ea_ctx* h) { return h->cfg.optimizer == EA_OPT_SGD ? 1 : 2; }
+
+// Advance the stage's step count and return the Adam bias corrections for it.
+ea::StepCoef next_coef(ea_ctx* h, int stage) {
+  const int64_t t = ++h->steps[stage];
+  ea::StepCoef sc;
+  if (h->cfg.optimizer == EA_OPT_SGD) {
+    sc.step_size = 0.f;
+    sc.inv_sqrt_bc2 = 0.f;
+    return sc;
+  }
+  const double bc1 = 1.0 - std::pow((double)h->cfg.beta1, (double)t);
+  const double bc2 = 1.0 - std::pow((double)h->cfg.beta2, (double)t);
+  sc.step_size = static_cast<float>((double)h->cfg.lr / bc1);
+  sc.inv_sqrt_bc2 = static_cast<float>(1.0 / std::sqrt(bc2));
+  return sc;
 }
 
 ea_status cuda_fail(ea_ctx* h, cudaError_t e, const char* what) {
@@ -99,17 +143,164 @@ void free_ctx(ea_ctx* h) {
   cudaSetDevice(h->cfg.device);
   if (h->side) cudaStreamSynchronize(h->side);
   if (h->comm) ncclCommDestroy(h->comm);
-  for (float* m : h->mom) if (m) cudaFree(m);
+  for (auto& slot : h->state)
+    for (float* m : slot) if (m) cudaFree(m);
   if (h->contrib) cudaFree(h->contrib);
   if (h->reduced) cudaFree(h->reduced);
   if (h->ev_in) cudaEventDestroy(h->ev_in);
   if (h->ev_local) cudaEventDestroy(h->ev_local);
   if (h->ev_done) cudaEventDestroy(h->ev_done);
   if (h->side) cudaStreamDestroy(h->side);
+  if (h->h2d) cudaStreamSynchronize(h->h2d);
+  if (h->d2h) cudaStreamSynchronize(h->d2h);
+  for (int i = 0; i < 2; ++i) {
+    if (h->staging[i]) cudaFree(h->staging[i]);
+    if (h->ev_h2d[i]) cudaEventDestroy(h->ev_h2d[i]);
+    if (h->ev_kern[i]) cudaEventDestroy(h->ev_kern[i]);
+  }
+  if (h->ev_d2h) cudaEventDestroy(h->ev_d2h);
+  if (h->h2d) cudaStreamDestroy(h->h2d);
+  if (h->d2h) cudaStreamDestroy(h->d2h);
   delete h;
 }
 
 int replicas_here(const ea_ctx* h) { return h->cfg.layout == EA_SPREAD ? 1 : h->cfg.n_pipelines; }
+
+float* state_ptr(const ea_ctx* h, int slot, int stage, int replica) {
+  if (slot >= state_slots(h)) return nullptr;
+  return h->state[slot][stage] + h->stride[stage] * replica;
+}
+
+// Validates one stage's pointers (nothing enqueued on failure).
+ea_status check_stage_ptrs(ea_ctx* h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
+                           const float* center_ptr) {
+  if (stage < 0 || stage >= h->cfg.n_stages) { set_err(h, "stage %d out of range", stage); return EA_EINVAL; }
+  if (!replica_ptrs || !grad_ptrs) { set_err(h, "replica_ptrs / grad_ptrs is NULL"); return EA_EINVAL; }
+  const int reps = replicas_here(h);
+  const int dev = h->cfg.device;
+  if (!center_ptr || !aligned16(center_ptr) || !is_device_ptr(center_ptr, dev)) {
+    set_err(h, "center_ptr must be a 16-byte aligned device pointer on device %d", dev);
+    return EA_EINVAL;
+  }
+  for (int i = 0; i < reps; ++i) {
+    if (!replica_ptrs[i] || !grad_ptrs[i] || !aligned16(replica_ptrs[i]) || !aligned16(grad_ptrs[i]) ||
+        !is_device_ptr(replica_ptrs[i], dev) || !is_device_ptr(grad_ptrs[i], dev)) {
+      set_err(h, "stage %d: replica/grad pointer %d must be a 16-byte aligned device pointer on device %d", stage, i,
+              dev);
+      return EA_EINVAL;
+    }
+  }
+  return EA_OK;
+}
+
+// Co-located: `count` validated stages in as few launches as possible.
+ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                           const float* const* grad_ptrs, float* const* center_ptrs, cudaStream_t s) {
+  const int n = h->cfg.n_pipelines;
+  const int opt = h->cfg.optimizer;
+  const bool two = state_slots(h) == 2;
+  cudaError_t e = cudaSuccess;
+  if (n > ea::kMaxFusedN) {  // wide N: one launch per stage
+    for (int j = 0; j < count; ++j) {
+      const int st = stages[j];
+      ea::ReplicaTable t;
+      for (int i = 0; i < n; ++i) {
+        t.x[i] = replica_ptrs[j * n + i];
+        t.g[i] = grad_ptrs[j * n + i];
+        t.m[i] = state_ptr(h, 0, st, i);
+        t.v[i] = two ? state_ptr(h, 1, st, i) : nullptr;
+      }
+      const ea::StepCoef sc = next_coef(h, st);
+      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, opt, sc, h->num_sms, s);
+      if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
+    }
+    return EA_OK;
+  }
+  for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
+    ea::StageBatch b;
+    b.nstages = 0;
+    for (int j = j0; j < count && j < j0 + ea::kMaxLaunchStages; ++j) {
+      const int st = stages[j];
+      ea::StageRefs& r = b.st[b.nstages++];
+      for (int i = 0; i < ea::kMaxFusedN; ++i) {
+        const bool on = i < n;
+        r.x[i] = on ? replica_ptrs[j * n + i] : nullptr;
+        r.g[i] = on ? grad_ptrs[j * n + i] : nullptr;
+        r.m[i] = on ? state_ptr(h, 0, st, i) : nullptr;
+        r.v[i] = (on && two) ? state_ptr(h, 1, st, i) : nullptr;
+      }
+      r.c = center_ptrs[j];
+      r.p = h->p[st];
+      r.sc = next_coef(h, st);
+    }
+    e = ea::launch_colocated_batch(b, n, h->hp, opt, h->variant, h->num_sms, s);
+    if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
+  }
+  return EA_OK;
+}
+
+// Spread: one stage's exchange on the side stream (rows a6-a8).
+ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s) {
+  if (!h->comm) {
+    set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
+    return EA_ESTATE;
+  }
+  cudaError_t e;
+  const int n = h->cfg.n_pipelines;
+  const int64_t pad = h->p_pad[stage], shard = pad / n;
+  float* own = center_ptr + shard * h->cfg.rank;
+  if ((e = cudaEventRecord(h->ev_in, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  if ((e = cudaStreamWaitEvent(h->side, h->ev_in, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  const ea::StepCoef sc = next_coef(h, stage);
+  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr,
+                              h->contrib, h->p[stage], pad, h->hp, h->cfg.optimizer, sc, h->num_sms, h->side);
+  if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
+  if ((e = cudaEventRecord(h->ev_local, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  ncclResult_t r = ncclReduceScatter(h->contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
+                                     h->side);
+  if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
+  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, h->side);
+  if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
+  r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
+  if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
+  // The caller's stream waits only for x_i (the next forward may start now).
+  if ((e = cudaStreamWaitEvent(s, h->ev_local, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  return EA_OK;
+}
+
+// Orders `stream` after everything enqueued on the side stream so far.
+ea_status join_side(ea_ctx* h, cudaStream_t s) {
+  if (h->cfg.layout != EA_SPREAD) return EA_OK;
+  cudaError_t e;
+  if ((e = cudaEventRecord(h->ev_done, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  if ((e = cudaStreamWaitEvent(s, h->ev_done, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  return EA_OK;
+}
+
+bool is_host_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return true;  // unregistered pageable memory
+  }
+  return a.type == cudaMemoryTypeHost || a.type == cudaMemoryTypeUnregistered;
+}
+
+ea_status host_path_resources(ea_ctx* h) {
+  if (h->h2d) return EA_OK;
+  cudaError_t e;
+  const size_t bytes = sizeof(float) * (size_t)h->cfg.n_pipelines * kHostChunk;
+  if ((e = cudaStreamCreateWithFlags(&h->h2d, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaStreamCreateWithFlags(&h->d2h, cudaStreamNonBlocking)) != cudaSuccess ||
+      (e = cudaMalloc(&h->staging[0], bytes)) != cudaSuccess || (e = cudaMalloc(&h->staging[1], bytes)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&h->ev_h2d[0], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&h->ev_h2d[1], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&h->ev_kern[0], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&h->ev_kern[1], cudaEventDisableTiming)) != cudaSuccess ||
+      (e = cudaEventCreateWithFlags(&h->ev_d2h, cudaEventDisableTiming)) != cudaSuccess)
+    return cuda_fail(h, e, "host-path resources");
+  return EA_OK;
+}
 
 }  // namespace
 
@@ -146,7 +337,7 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (c.rank < 0 || c.rank >= c.world) { set_err(nullptr, "rank %d out of [0,%d)", c.rank, c.world); return EA_EINVAL; }
   }
   if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
-  ea_status st = check_hyper(nullptr, c.alpha, c.beta, c.rho, c.lr, c.momentum, c.weight_decay, c.nesterov);
+  ea_status st = check_hyper(nullptr, c);
   if (st != EA_OK) return st;
   int ndev = 0;
   cudaError_t e = cudaGetDeviceCount(&ndev);
@@ -159,6 +350,7 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   h->hp = make_hyper(c);
   h->variant = c.kernel_variant;
   h->p.assign(c.stage_params, c.stage_params + c.n_stages);
+  h->steps.assign(c.n_stages, 0);
   h->cfg.stage_params = nullptr;  // not retained
   e = cudaSetDevice(c.device);
   if (e != cudaSuccess) { ea_status r = cuda_fail(nullptr, e, "cudaSetDevice"); free_ctx(h); return r; }
@@ -173,16 +365,18 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (pad > max_pad) max_pad = pad;
     const int64_t stride = round_up(ps, 64);
     h->stride.push_back(stride);
-    float* m = nullptr;
-    e = cudaMalloc(&m, sizeof(float) * stride * reps);
-    if (e == cudaSuccess) e = cudaMemset(m, 0, sizeof(float) * stride * reps);
-    if (e != cudaSuccess) {
-      ea_status r = cuda_fail(nullptr, e, "momentum allocation");
-      if (m) cudaFree(m);
-      free_ctx(h);
-      return r;
+    for (int slot = 0; slot < state_slots(h); ++slot) {
+      float* m = nullptr;
+      e = cudaMalloc(&m, sizeof(float) * stride * reps);
+      if (e == cudaSuccess) e = cudaMemset(m, 0, sizeof(float) * stride * reps);
+      if (e != cudaSuccess) {
+        ea_status r = cuda_fail(nullptr, e, "optimizer-state allocation");
+        if (m) cudaFree(m);
+        free_ctx(h);
+        return r;
+      }
+      h->state[slot].push_back(m);
     }
-    h->mom.push_back(m);
   }
   if (c.layout == EA_SPREAD) {
     if ((e = cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking)) != cudaSuccess ||
@@ -223,102 +417,15 @@ int64_t ea_shard_elems(ea_handle h, int32_t stage) {
   return h->cfg.layout == EA_SPREAD ? h->p_pad[stage] / h->cfg.n_pipelines : h->p[stage];
 }
 
-// Validates one stage's pointers (nothing enqueued on failure).
-static ea_status check_stage_ptrs(ea_ctx* h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
-                                  const float* center_ptr) {
-  if (stage < 0 || stage >= h->cfg.n_stages) { set_err(h, "stage %d out of range", stage); return EA_EINVAL; }
-  if (!replica_ptrs || !grad_ptrs) { set_err(h, "replica_ptrs / grad_ptrs is NULL"); return EA_EINVAL; }
-  const int reps = replicas_here(h);
-  const int dev = h->cfg.device;
-  if (!center_ptr || !aligned16(center_ptr) || !is_device_ptr(center_ptr, dev)) {
-    set_err(h, "center_ptr must be a 16-byte aligned device pointer on device %d", dev);
-    return EA_EINVAL;
-  }
-  for (int i = 0; i < reps; ++i) {
-    if (!replica_ptrs[i] || !grad_ptrs[i] || !aligned16(replica_ptrs[i]) || !aligned16(grad_ptrs[i]) ||
-        !is_device_ptr(replica_ptrs[i], dev) || !is_device_ptr(grad_ptrs[i], dev)) {
-      set_err(h, "stage %d: replica/grad pointer %d must be a 16-byte aligned device pointer on device %d", stage, i,
-              dev);
-      return EA_EINVAL;
-    }
-  }
-  return EA_OK;
-}
-
-// Co-located: `count` validated stages in as few launches as possible.
-static ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
-                                  const float* const* grad_ptrs, float* const* center_ptrs, cudaStream_t s) {
-  const int n = h->cfg.n_pipelines;
-  cudaError_t e = cudaSuccess;
-  if (n > ea::kMaxFusedN) {  // wide N: one launch per stage
-    for (int j = 0; j < count; ++j) {
-      const int st = stages[j];
-      ea::ReplicaTable t;
-      for (int i = 0; i < n; ++i) {
-        t.x[i] = replica_ptrs[j * n + i];
-        t.g[i] = grad_ptrs[j * n + i];
-        t.m[i] = h->mom[st] + h->stride[st] * i;
-      }
-      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, h->num_sms, s);
-      if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
-    }
-    return EA_OK;
-  }
-  for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
-    ea::StageBatch b;
-    b.nstages = 0;
-    for (int j = j0; j < count && j < j0 + ea::kMaxLaunchStages; ++j) {
-      const int st = stages[j];
-      ea::StageRefs& r = b.st[b.nstages++];
-      for (int i = 0; i < ea::kMaxFusedN; ++i) {
-        const bool on = i < n;
-        r.x[i] = on ? replica_ptrs[j * n + i] : nullptr;
-        r.g[i] = on ? grad_ptrs[j * n + i] : nullptr;
-        r.m[i] = on ? h->mom[st] + h->stride[st] * i : nullptr;
-      }
-      r.c = center_ptrs[j];
-      r.p = h->p[st];
-    }
-    e = ea::launch_colocated_batch(b, n, h->hp, h->variant, h->num_sms, s);
-    if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
-  }
-  return EA_OK;
-}
-
-// Spread: one stage's exchange on the side stream (rows a6-a8).
-static ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr,
-                             cudaStream_t s) {
-  if (!h->comm) {
-    set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
-    return EA_ESTATE;
-  }
-  cudaError_t e;
-  const int n = h->cfg.n_pipelines;
-  const int64_t pad = h->p_pad[stage], shard = pad / n;
-  float* own = center_ptr + shard * h->cfg.rank;
-  if ((e = cudaEventRecord(h->ev_in, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-  if ((e = cudaStreamWaitEvent(h->side, h->ev_in, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  e = ea::launch_spread_local(replica, grad, h->mom[stage], center_ptr, h->contrib, h->p[stage], pad, h->hp,
-                              h->num_sms, h->side);
-  if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
-  if ((e = cudaEventRecord(h->ev_local, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-  ncclResult_t r = ncclReduceScatter(h->contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
-                                     h->side);
-  if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
-  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, h->side);
-  if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
-  r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
-  if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
-  // The caller's stream waits only for x_i (the next forward may start now).
-  if ((e = cudaStreamWaitEvent(s, h->ev_local, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  return EA_OK;
-}
-
 ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
                   float* center_ptr, void* stream) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   ea_status st = check_stage_ptrs(h, stage, replica_ptrs, grad_ptrs, center_ptr);
   if (st != EA_OK) return st;
+  if (h->cfg.layout == EA_SPREAD && !h->comm) {
+    set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
+    return EA_ESTATE;
+  }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -342,6 +449,10 @@ ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float*
     if (st != EA_OK) return st;
   }
   if (count == 0) return EA_OK;
+  if (h->cfg.layout == EA_SPREAD && !h->comm) {
+    set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
+    return EA_ESTATE;
+  }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
@@ -353,15 +464,113 @@ ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float*
   return EA_OK;
 }
 
+ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
+                            const float* const* host_grad_ptrs, float* const* center_ptrs,
+                            float* const* host_center_out, void* stream) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  if (h->cfg.layout != EA_COLOCATED) { set_err(h, "ea_step_many_host needs EA_COLOCATED"); return EA_ESTATE; }
+  if (count < 0 || (count > 0 && (!stages || !replica_ptrs || !host_grad_ptrs || !center_ptrs || !host_center_out))) {
+    set_err(h, "ea_step_many_host: bad count or NULL array");
+    return EA_EINVAL;
+  }
+  const int n = h->cfg.n_pipelines;
+  const int dev = h->cfg.device;
+  for (int j = 0; j < count; ++j) {
+    const int st = stages[j];
+    if (st < 0 || st >= h->cfg.n_stages) { set_err(h, "stage %d out of range", st); return EA_EINVAL; }
+    for (int k = 0; k < j; ++k)
+      if (stages[k] == st) { set_err(h, "ea_step_many_host: stage %d listed twice", st); return EA_EINVAL; }
+    if (!center_ptrs[j] || !aligned16(center_ptrs[j]) || !is_device_ptr(center_ptrs[j], dev) ||
+        !host_center_out[j] || !is_host_ptr(host_center_out[j])) {
+      set_err(h, "stage %d: center must be an aligned device pointer and host_center_out a host pointer", st);
+      return EA_EINVAL;
+    }
+    for (int i = 0; i < n; ++i) {
+      const float* x = replica_ptrs[(size_t)j * n + i];
+      const float* g = host_grad_ptrs[(size_t)j * n + i];
+      if (!x || !aligned16(x) || !is_device_ptr(x, dev) || !g || !is_host_ptr(g)) {
+        set_err(h, "stage %d replica %d: replica must be an aligned device pointer, grad a host pointer", st, i);
+        return EA_EINVAL;
+      }
+    }
+  }
+  if (count == 0) return EA_OK;
+  cudaError_t e = cudaSetDevice(dev);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
+  ea_status rs = host_path_resources(h);
+  if (rs != EA_OK) return rs;
+  cudaStream_t s = static_cast<cudaStream_t>(stream);
+  const int opt = h->cfg.optimizer;
+  const bool two = state_slots(h) == 2;
+  // the copies must not overtake work already queued on the caller's stream
+  if ((e = cudaEventRecord(h->ev_d2h, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  if ((e = cudaStreamWaitEvent(h->h2d, h->ev_d2h, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  int64_t k = 0;  // chunk counter (staging buffer k % 2)
+  for (int j = 0; j < count; ++j) {
+    const int st = stages[j];
+    const ea::StepCoef sc = next_coef(h, st);
+    const int64_t ps = h->p[st];
+    for (int64_t off = 0; off < ps; off += kHostChunk, ++k) {
+      const int64_t len = ps - off < kHostChunk ? ps - off : kHostChunk;
+      const int b = static_cast<int>(k & 1);
+      float* stage_buf = h->staging[b];
+      // H2D of this chunk's gradients once the kernel that last read this buffer is done
+      if (k >= 2 && (e = cudaStreamWaitEvent(h->h2d, h->ev_kern[b], 0)) != cudaSuccess)
+        return cuda_fail(h, e, "cudaStreamWaitEvent");
+      for (int i = 0; i < n; ++i) {
+        e = cudaMemcpyAsync(stage_buf + (size_t)i * kHostChunk, host_grad_ptrs[(size_t)j * n + i] + off,
+                            sizeof(float) * len, cudaMemcpyHostToDevice, h->h2d);
+        if (e != cudaSuccess) return cuda_fail(h, e, "H2D gradients");
+      }
+      if ((e = cudaEventRecord(h->ev_h2d[b], h->h2d)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+      if ((e = cudaStreamWaitEvent(s, h->ev_h2d[b], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+      // the fused step on [off, off+len) of the stage (elementwise: any chunk is a valid sub-problem)
+      if (n > ea::kMaxFusedN) {
+        ea::ReplicaTable t;
+        for (int i = 0; i < n; ++i) {
+          t.x[i] = replica_ptrs[(size_t)j * n + i] + off;
+          t.g[i] = stage_buf + (size_t)i * kHostChunk;
+          t.m[i] = state_ptr(h, 0, st, i) + off;
+          t.v[i] = two ? state_ptr(h, 1, st, i) + off : nullptr;
+        }
+        e = ea::launch_colocated_wide(t, n, center_ptrs[j] + off, len, h->hp, opt, sc, h->num_sms, s);
+      } else {
+        ea::StageBatch bt;
+        bt.nstages = 1;
+        ea::StageRefs& r = bt.st[0];
+        for (int i = 0; i < ea::kMaxFusedN; ++i) {
+          const bool on = i < n;
+          r.x[i] = on ? replica_ptrs[(size_t)j * n + i] + off : nullptr;
+          r.g[i] = on ? stage_buf + (size_t)i * kHostChunk : nullptr;
+          r.m[i] = on ? state_ptr(h, 0, st, i) + off : nullptr;
+          r.v[i] = (on && two) ? state_ptr(h, 1, st, i) + off : nullptr;
+        }
+        r.c = center_ptrs[j] + off;
+        r.p = len;
+        r.sc = sc;
+        e = ea::launch_colocated_batch(bt, n, h->hp, opt, h->variant, h->num_sms, s);
+      }
+      if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
+      if ((e = cudaEventRecord(h->ev_kern[b], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+      // D2H of the updated center chunk
+      if ((e = cudaStreamWaitEvent(h->d2h, h->ev_kern[b], 0)) != cudaSuccess)
+        return cuda_fail(h, e, "cudaStreamWaitEvent");
+      e = cudaMemcpyAsync(host_center_out[j] + off, center_ptrs[j] + off, sizeof(float) * len, cudaMemcpyDeviceToHost,
+                          h->d2h);
+      if (e != cudaSuccess) return cuda_fail(h, e, "D2H center");
+    }
+  }
+  if ((e = cudaEventRecord(h->ev_d2h, h->d2h)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  if ((e = cudaStreamWaitEvent(s, h->ev_d2h, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  return EA_OK;
+}
+
 ea_status ea_sync(ea_handle h, void* stream) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
-  cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (h->cfg.layout == EA_SPREAD) {
-    if ((e = cudaEventRecord(h->ev_done, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-    if ((e = cudaStreamWaitEvent(s, h->ev_done, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  }
+  ea_status st = join_side(h, static_cast<cudaStream_t>(stream));
+  if (st != EA_OK) return st;
   if (h->comm) {
     ncclResult_t async_err = ncclSuccess;
     ncclResult_t r = ncclCommGetAsyncError(h->comm, &async_err);
@@ -387,8 +596,10 @@ ea_status ea_spread_local(ea_handle h, int32_t stage, float* replica_ptr, const 
     }
   cudaError_t e = cudaSetDevice(dev);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
-  e = ea::launch_spread_local(replica_ptr, grad_ptr, h->mom[stage], center_ptr, contrib, h->p[stage], h->p_pad[stage],
-                              h->hp, h->num_sms, static_cast<cudaStream_t>(stream));
+  const ea::StepCoef sc = next_coef(h, stage);
+  e = ea::launch_spread_local(replica_ptr, grad_ptr, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr,
+                              contrib, h->p[stage], h->p_pad[stage], h->hp, h->cfg.optimizer, sc, h->num_sms,
+                              static_cast<cudaStream_t>(stream));
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
   return EA_OK;
 }
@@ -411,44 +622,64 @@ ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const
   return EA_OK;
 }
 
-ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, float** momentum_dev) {
+ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, float** state_dev) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
-  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || !momentum_dev) {
-    set_err(h, "bad stage/replica/out pointer");
+  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || !state_dev ||
+      slot < 0 || slot >= state_slots(h)) {
+    set_err(h, "bad stage/replica/slot or NULL out pointer (this optimizer has %d state slot(s))", state_slots(h));
     return EA_EINVAL;
   }
-  *momentum_dev = h->mom[stage] + h->stride[stage] * replica;
+  *state_dev = state_ptr(h, slot, stage, replica);
   return EA_OK;
 }
 
-ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, const float* momentum_src, void* stream) {
+ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, const float* src, void* stream) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
-  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || !momentum_src ||
-      !is_device_ptr(momentum_src, h->cfg.device)) {
-    set_err(h, "bad stage/replica or momentum_src is not a device pointer");
+  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || slot < 0 ||
+      slot >= state_slots(h) || !src || !is_device_ptr(src, h->cfg.device)) {
+    set_err(h, "bad stage/replica/slot or src is not a device pointer");
     return EA_EINVAL;
   }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
   cudaStream_t s = static_cast<cudaStream_t>(stream);
-  if (h->cfg.layout == EA_SPREAD) {  // order after pending side-stream work on this momentum
-    if ((e = cudaEventRecord(h->ev_done, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-    if ((e = cudaStreamWaitEvent(s, h->ev_done, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  }
-  e = cudaMemcpyAsync(h->mom[stage] + h->stride[stage] * replica, momentum_src, sizeof(float) * h->p[stage],
-                      cudaMemcpyDeviceToDevice, s);
+  ea_status st = join_side(h, s);  // order after pending side-stream work on this state
+  if (st != EA_OK) return st;
+  e = cudaMemcpyAsync(state_ptr(h, slot, stage, replica), src, sizeof(float) * h->p[stage], cudaMemcpyDeviceToDevice,
+                      s);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaMemcpyAsync");
   return EA_OK;
 }
 
-ea_status ea_set_hyper(ea_handle h, float alpha, float beta, float rho, float lr, float momentum, float weight_decay,
-                       int32_t nesterov) {
+ea_status ea_get_step(ea_handle h, int32_t stage, int64_t* step) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
-  ea_status st = check_hyper(h, alpha, beta, rho, lr, momentum, weight_decay, nesterov);
+  if (stage < 0 || stage >= h->cfg.n_stages || !step) { set_err(h, "bad stage or NULL out pointer"); return EA_EINVAL; }
+  *step = h->steps[stage];
+  return EA_OK;
+}
+
+ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  if (stage < 0 || stage >= h->cfg.n_stages || step < 0) { set_err(h, "bad stage or negative step"); return EA_EINVAL; }
+  h->steps[stage] = step;
+  return EA_OK;
+}
+
+ea_status ea_set_hyper(ea_handle h, const ea_config* cfg) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  if (!cfg) { set_err(h, "cfg is NULL"); return EA_EINVAL; }
+  if (cfg->optimizer != h->cfg.optimizer || cfg->n_pipelines != h->cfg.n_pipelines || cfg->layout != h->cfg.layout) {
+    set_err(h, "ea_set_hyper cannot change optimizer, n_pipelines or layout");
+    return EA_EINVAL;
+  }
+  ea_status st = check_hyper(h, *cfg);
   if (st != EA_OK) return st;
-  h->cfg.alpha = alpha; h->cfg.beta = beta; h->cfg.rho = rho; h->cfg.lr = lr;
-  h->cfg.momentum = momentum; h->cfg.weight_decay = weight_decay; h->cfg.nesterov = nesterov;
-  h->hp = make_hyper(h->cfg);
+  ea_config c = h->cfg;
+  c.alpha = cfg->alpha; c.beta = cfg->beta; c.rho = cfg->rho; c.lr = cfg->lr;
+  c.momentum = cfg->momentum; c.weight_decay = cfg->weight_decay; c.nesterov = cfg->nesterov;
+  c.beta1 = cfg->beta1; c.beta2 = cfg->beta2; c.eps = cfg->eps;
+  h->cfg = c;
+  h->hp = make_hyper(c);
   return EA_OK;
 }
 

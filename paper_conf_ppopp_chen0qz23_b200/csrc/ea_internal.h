@@ -7,16 +7,29 @@
 
 namespace ea {
 
-// Hyper-parameters in the form the kernels consume (fp32, P:112 / DESIGN.md c7).
+// Local optimizer of Step 1 (DESIGN.md c7 SGD-momentum, c21 Adam/AdamW).
+enum Opt : int { kOptSGD = 0, kOptAdam = 1, kOptAdamW = 2 };
+
+// Hyper-parameters in the form the kernels consume (fp32).
 struct Hyper {
   float alpha;     // dilution rate
   float beta;      // center pull (EASGD)
   float rho;       // weight of Delta_i in the contribution
-  float lr;        // SGD learning rate
-  float momentum;  // mu
-  float wd;        // L2 weight decay lambda
-  int nesterov;    // 0/1
+  float lr;        // learning rate
+  float momentum;  // mu (SGD)
+  float wd;        // weight decay lambda (SGD/Adam: L2 on the gradient; AdamW: decoupled)
+  int nesterov;    // 0/1 (SGD)
   float inv_n;     // 1/N (step 5 normalisation)
+  float beta1, one_minus_beta1;  // Adam
+  float beta2, one_minus_beta2;
+  float eps;
+  float lr_wd;     // lr * wd (AdamW decoupled decay)
+};
+
+// Per-stage, per-call Adam bias corrections (t = this stage's step count).
+struct StepCoef {
+  float step_size;     // lr / (1 - beta1^t)
+  float inv_sqrt_bc2;  // 1 / sqrt(1 - beta2^t)
 };
 
 constexpr int kMaxReplicas = 64;      // EA_MAX_REPLICAS
@@ -27,13 +40,14 @@ constexpr int kMaxLaunchStages = 8;   // stages fused into one launch
 struct StageRefs {
   float* x[kMaxFusedN];
   const float* g[kMaxFusedN];
-  float* m[kMaxFusedN];
+  float* m[kMaxFusedN];  // SGD momentum / Adam first moment
+  float* v[kMaxFusedN];  // Adam second moment (unused by SGD)
   float* c;
-  int64_t p;  // elements
+  int64_t p;             // elements
+  StepCoef sc;
 };
 
-// Up to kMaxLaunchStages stages updated by ONE launch (same N): the work of
-// all stages is concatenated and split evenly over the persistent grid.
+// Up to kMaxLaunchStages stages updated by ONE launch (same N).
 struct StageBatch {
   StageRefs st[kMaxLaunchStages];
   int nstages;
@@ -44,31 +58,34 @@ struct ReplicaTable {
   float* x[kMaxReplicas];
   const float* g[kMaxReplicas];
   float* m[kMaxReplicas];
+  float* v[kMaxReplicas];
 };
 
 enum KernelVariant : int {
-  kVariantAuto = 0,      // library picks (see launch_colocated_batch)
-  kVariantRegLoop = 1,   // one thread per float4 of center, loops over N replicas in registers
+  kVariantAuto = 0,      // library picks (lane/shuffle, the measured best)
+  kVariantRegLoop = 1,   // one thread per float4 of center, loops over N replicas in registers (SGD)
   kVariantLaneShfl = 2,  // lanes = (replica, float4 chunk); center tile staged by cp.async.bulk
-                         // into shared memory; replica reduction by warp shuffles
+                         // into shared memory; replica reduction by warp shuffles (SGD, Adam)
   kVariantBulkPipe = 3,  // every input tile streamed by cp.async.bulk into a multi-stage smem
-                         // ring (producer warp + mbarriers); consumers store from registers
+                         // ring (producer warp + mbarriers); consumers store from registers (SGD)
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N
-// (N <= kMaxFusedN): updates x_i, m_i and x~ of every stage in place, one launch.
-cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int variant, int num_sms,
+// (N <= kMaxFusedN): updates x_i, optimizer state and x~ of every stage in
+// place, one launch.  Adam/AdamW always use the lane kernel.
+cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s);
 
 // Co-located step for one stage with any N <= kMaxReplicas (N > 8 path).
-cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
-                                  int num_sms, cudaStream_t s);
+cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
+                                  const StepCoef& sc, int num_sms, cudaStream_t s);
 
-// Spread local step (rows a1-a4 for one replica): updates x, m in place and
-// writes r = rho*Delta + beta*(x - x~) into contrib[0..p), zeros into
-// contrib[p..p_pad).
-cudaError_t launch_spread_local(float* x, const float* g, float* m, const float* center, float* contrib,
-                                int64_t p, int64_t p_pad, const Hyper& hp, int num_sms, cudaStream_t s);
+// Spread local step (rows a1-a4 for one replica): updates x and the optimizer
+// state in place and writes r = rho*Delta + beta*(x - x~) into contrib[0..p),
+// zeros into contrib[p..p_pad).
+cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef& sc, int num_sms,
+                                cudaStream_t s);
 
 // Spread shard epilogue (row a5): shard[k] += reduced[k] * inv_n for k < count.
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,

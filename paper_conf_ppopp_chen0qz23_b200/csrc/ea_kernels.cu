@@ -1,20 +1,20 @@
 // Fused elastic-averaging kernels for sm_100a (B200).
 //
-// Per element j of a stage and replica i (§3.2; DESIGN.md c1-c14):
-//   g'  = g_i + wd*x_i                          Step 1: SGD-momentum local update
-//   m_i = mu*m_i + g'
-//   D_i = -lr * (nesterov ? g' + mu*m_i : m_i)
-//   x_i = (1-alpha)*x_i + alpha*x~ + D_i         Step 2: (1-a):a dilution + local update
-//   R  += rho*D_i + beta*(x_i - x~)              Steps 3-4: send + accumulate
-//   x~  = x~ + R/N                               Step 5: normalise + apply
+// Per element j of a stage and replica i (§3.2; DESIGN.md c1-c14, c21):
+//   Step 1 (local update of the user-specified optimizer):
+//     SGD-momentum: g' = g + wd*x; m = mu*m + g'; D = -lr*(nesterov ? g' + mu*m : m)
+//     Adam(W):      g' = g (+ wd*x for Adam); m = b1*m + (1-b1)*g'; v = b2*v + (1-b2)*g'^2;
+//                   D = -(lr/bc1) * m / (sqrt(v)/sqrt(bc2) + eps)  (- lr*wd*x for AdamW)
+//   Step 2: x_i = (1-alpha)*x_i + alpha*x~ + D_i          ((1-a):a dilution + local update)
+//   Steps 3-4: R += rho*D_i + beta*(x_i - x~)               (send + accumulate)
+//   Step 5: x~ = x~ + R/N                                    (normalise + apply)
 //
 // The path is elementwise plus a reduction over the N replicas: ~0.5 flop per
 // byte, far below the fp32 ridge, so every kernel here is HBM-bound and is
-// written for bytes in flight: 128-bit coalesced accesses, no shared-memory
-// round trips for data that is used once, persistent grids (#SMs x resident
-// blocks) sweeping the stages of a launch in waves with the ragged remainder
-// split evenly (wave_item), so no SM idles in a partial last wave.  Tensor
-// cores are not used (no contraction).
+// written for bytes in flight: 128-bit coalesced accesses, persistent grids
+// (#SMs x resident blocks) sweeping the stages of a launch in waves with the
+// ragged remainder split evenly (wave_item), so no SM idles in a partial last
+// wave.  Tensor cores are not used (no contraction).
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -29,8 +29,7 @@ constexpr int kThreads = 256;
 
 // ---------------------------------------------------------------- memory ops
 // HINT = 0: plain streaming (L1 bypass); HINT = 1: additionally mark every
-// access L2 evict-first (the data is touched once per step and the working
-// set is far above the 126 MB L2).
+// access L2 evict-first (measured: no effect; kept as a knob).
 template <int HINT>
 struct Mem {
   uint64_t pol;
@@ -75,24 +74,41 @@ struct Mem {
 
 // ---------------------------------------------------------------- the math
 // One (replica, element) update; returns the replica's contribution r_i.
-__device__ __forceinline__ float ea_elem(float& x, float g, float& m, float c, const Hyper& hp) {
-  const float gg = fmaf(hp.wd, x, g);             // g + lambda*x
-  const float mn = fmaf(hp.momentum, m, gg);      // mu*m + g'
-  const float d = hp.nesterov ? fmaf(hp.momentum, mn, gg) : mn;
-  const float delta = -hp.lr * d;                 // local update Delta_i (Step 1)
-  const float gap = x - c;                        // x_i - x~ (pre-step values, c1/c2)
+// m: SGD momentum / Adam first moment; v: Adam second moment (SGD: untouched).
+template <int OPT>
+__device__ __forceinline__ float ea_elem(float& x, float g, float& m, float& v, float c, const Hyper& hp,
+                                         const StepCoef& sc) {
+  float delta;
+  if constexpr (OPT == kOptSGD) {
+    const float gg = fmaf(hp.wd, x, g);             // g + lambda*x
+    const float mn = fmaf(hp.momentum, m, gg);      // mu*m + g'
+    const float d = hp.nesterov ? fmaf(hp.momentum, mn, gg) : mn;
+    delta = -hp.lr * d;                             // local update Delta_i (Step 1)
+    m = mn;
+  } else {
+    const float gg = OPT == kOptAdam ? fmaf(hp.wd, x, g) : g;
+    const float mn = fmaf(hp.beta1, m, hp.one_minus_beta1 * gg);
+    const float vn = fmaf(hp.beta2, v, hp.one_minus_beta2 * (gg * gg));
+    const float denom = fmaf(sqrtf(vn), sc.inv_sqrt_bc2, hp.eps);
+    delta = -sc.step_size * (mn / denom);
+    if constexpr (OPT == kOptAdamW) delta = fmaf(-hp.lr_wd, x, delta);
+    m = mn;
+    v = vn;
+  }
+  const float gap = x - c;                          // x_i - x~ (pre-step values, c1/c2)
   const float r = fmaf(hp.beta, gap, hp.rho * delta);
-  x = fmaf(-hp.alpha, gap, x) + delta;            // (1-a)x + a*x~ + Delta (Step 2)
-  m = mn;
+  x = fmaf(-hp.alpha, gap, x) + delta;              // (1-a)x + a*x~ + Delta (Step 2)
   return r;
 }
 
-__device__ __forceinline__ float4 ea_vec(float4& x, float4 g, float4& m, float4 c, const Hyper& hp) {
+template <int OPT>
+__device__ __forceinline__ float4 ea_vec(float4& x, float4 g, float4& m, float4& v, float4 c, const Hyper& hp,
+                                         const StepCoef& sc) {
   float4 r;
-  r.x = ea_elem(x.x, g.x, m.x, c.x, hp);
-  r.y = ea_elem(x.y, g.y, m.y, c.y, hp);
-  r.z = ea_elem(x.z, g.z, m.z, c.z, hp);
-  r.w = ea_elem(x.w, g.w, m.w, c.w, hp);
+  r.x = ea_elem<OPT>(x.x, g.x, m.x, v.x, c.x, hp, sc);
+  r.y = ea_elem<OPT>(x.y, g.y, m.y, v.y, c.y, hp, sc);
+  r.z = ea_elem<OPT>(x.z, g.z, m.z, v.z, c.z, hp, sc);
+  r.w = ea_elem<OPT>(x.w, g.w, m.w, v.w, c.w, hp, sc);
   return r;
 }
 
@@ -105,34 +121,30 @@ __device__ __forceinline__ float4 center_apply(float4 c, float4 acc, float inv_n
 }
 
 // Scalar tail of one stage: elements [4*(p/4), p) (fewer than 4), one thread.
-template <int N>
+template <int N, int OPT>
 __device__ void stage_tail(const StageRefs& st, const Hyper& hp) {
   for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
     const float c = st.c[j];
     float acc = 0.f;
 #pragma unroll
     for (int i = 0; i < N; ++i) {
-      float x = st.x[i][j], m = st.m[i][j];
-      acc += ea_elem(x, st.g[i][j], m, c, hp);
+      float x = st.x[i][j], m = st.m[i][j], v = OPT == kOptSGD ? 0.f : st.v[i][j];
+      acc += ea_elem<OPT>(x, st.g[i][j], m, v, c, hp, st.sc);
       st.x[i][j] = x;
       st.m[i][j] = m;
+      if (OPT != kOptSGD) st.v[i][j] = v;
     }
     st.c[j] = fmaf(acc, hp.inv_n, c);
   }
 }
 
-// Even split of [0, total) units over the grid: this block's [lo, hi).
-__device__ __forceinline__ void block_range(int64_t total, int64_t& lo, int64_t& hi) {
-  lo = total * blockIdx.x / gridDim.x;
-  hi = total * (blockIdx.x + 1) / gridDim.x;
-}
-
-// Wave schedule over the stages of a launch.  Chunks of C float4: in stage s
-// the grid sweeps full waves (chunk w*G + b for block b, so the G blocks of
-// a wave touch one contiguous window of every stream -- DRAM-page friendly),
-// then the ragged remainder R < G*C is split evenly over all G blocks (no
-// block idles in a partial last wave).  Every block walks the same sequence
-// of (stage, wave) items, so the cursor is warp- and block-uniform.
+// ---------------------------------------------------------------- wave schedule
+// Chunks of C float4: in stage s the grid sweeps full waves (chunk w*G + b for
+// block b, so the G blocks of a wave touch one contiguous window of every
+// stream -- DRAM-page friendly), then the ragged remainder R < G*C is split
+// evenly over all G blocks (no block idles in a partial last wave).  Every
+// block walks the same sequence of (stage, wave) items, so the cursor is
+// warp- and block-uniform.
 struct WaveCursor {
   int s;
   int64_t w;
@@ -175,7 +187,7 @@ __device__ __forceinline__ bool wave_item(const StageBatch& b, int64_t C, WaveCu
 }
 
 // ============================================================================
-// Variant 1: register-resident replica loop.
+// Variant 1 (SGD): register-resident replica loop.
 // One thread owns U float4 of a center; it issues all (3N+1)*U 128-bit loads
 // before any arithmetic (maximal memory-level parallelism per thread: the
 // replica pointers may alias as far as the compiler knows, so the loads are
@@ -183,8 +195,6 @@ __device__ __forceinline__ bool wave_item(const StageBatch& b, int64_t C, WaveCu
 // registers, reduces the N contributions in registers and writes x_i, m_i
 // and x~ once.  Work unit: kThreads*U float4 per block, scheduled by wave_item.
 // ============================================================================
-constexpr int kUnitVec = 32;
-
 template <int N, int U, int HINT>
 __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, int64_t ve, const Hyper& hp,
                                               const Mem<HINT>& mem) {
@@ -216,7 +226,8 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
       float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
       for (int i = 0; i < N; ++i) {
-        add4(acc, ea_vec(x[i][u], g[i][u], m[i][u], c[u], hp));
+        float4 unused;
+        add4(acc, ea_vec<kOptSGD>(x[i][u], g[i][u], m[i][u], unused, c[u], hp, st.sc));
         mem.st(st.x[i] + 4 * v, x[i][u]);
         mem.st(st.m[i] + 4 * v, m[i][u]);
       }
@@ -233,51 +244,57 @@ __global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b
   int64_t v0, nv;
   while (wave_item(b, (int64_t)kThreads * U, cur, s, v0, nv)) regloop_range<N, U, HINT>(b.st[s], v0, v0 + nv, hp, mem);
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
 }
 
 // Runtime-N fallback (N > 8): one stage, replicas visited in a loop.
-template <int U>
+template <int U, int OPT>
 __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t, int n, float* __restrict__ center,
-                                                           int64_t nvec, int64_t p, const Hyper hp) {
+                                                           int64_t nvec, int64_t p, const Hyper hp,
+                                                           const StepCoef sc) {
   const Mem<0> mem;
-  int64_t lo, hi;
-  block_range((nvec + kUnitVec - 1) / kUnitVec, lo, hi);
-  const int64_t va = lo * kUnitVec, ve = hi * kUnitVec < nvec ? hi * kUnitVec : nvec;
-  for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
-    float4 c[U], acc[U];
-    bool ok[U];
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t v = base + (int64_t)u * kThreads;
-      ok[u] = v < ve;
-      acc[u] = make_float4(0.f, 0.f, 0.f, 0.f);
-      if (ok[u]) c[u] = mem.ld(center + 4 * v);
-    }
-    for (int i = 0; i < n; ++i) {
-      float4 x[U], g[U], m[U];
+  WaveCursor cur{0, 0};
+  int sidx;
+  int64_t va, nv;
+  while (wave_item_f(1, [&](int) { return nvec; }, (int64_t)kThreads * U, cur, sidx, va, nv)) {
+    const int64_t ve = va + nv;
+    for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
+      float4 c[U], acc[U];
+      bool ok[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int64_t v = base + (int64_t)u * kThreads;
-        if (ok[u]) {
-          x[u] = mem.ld(t.x[i] + 4 * v);
-          g[u] = mem.ld_ro(t.g[i] + 4 * v);
-          m[u] = mem.ld(t.m[i] + 4 * v);
+        ok[u] = v < ve;
+        acc[u] = make_float4(0.f, 0.f, 0.f, 0.f);
+        if (ok[u]) c[u] = mem.ld(center + 4 * v);
+      }
+      for (int i = 0; i < n; ++i) {
+        float4 x[U], g[U], m[U], w[U];
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int64_t v = base + (int64_t)u * kThreads;
+          if (ok[u]) {
+            x[u] = mem.ld(t.x[i] + 4 * v);
+            g[u] = mem.ld_ro(t.g[i] + 4 * v);
+            m[u] = mem.ld(t.m[i] + 4 * v);
+            if (OPT != kOptSGD) w[u] = mem.ld(t.v[i] + 4 * v);
+          }
+        }
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          if (!ok[u]) continue;
+          const int64_t v = base + (int64_t)u * kThreads;
+          add4(acc[u], ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc));
+          mem.st(t.x[i] + 4 * v, x[u]);
+          mem.st(t.m[i] + 4 * v, m[u]);
+          if (OPT != kOptSGD) mem.st(t.v[i] + 4 * v, w[u]);
         }
       }
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        if (!ok[u]) continue;
         const int64_t v = base + (int64_t)u * kThreads;
-        add4(acc[u], ea_vec(x[u], g[u], m[u], c[u], hp));
-        mem.st(t.x[i] + 4 * v, x[u]);
-        mem.st(t.m[i] + 4 * v, m[u]);
+        if (ok[u]) mem.st(center + 4 * v, center_apply(c[u], acc[u], hp.inv_n));
       }
-    }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t v = base + (int64_t)u * kThreads;
-      if (ok[u]) mem.st(center + 4 * v, center_apply(c[u], acc[u], hp.inv_n));
     }
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
@@ -285,10 +302,11 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
       const float c = center[j];
       float acc = 0.f;
       for (int i = 0; i < n; ++i) {
-        float x = t.x[i][j], m = t.m[i][j];
-        acc += ea_elem(x, t.g[i][j], m, c, hp);
+        float x = t.x[i][j], m = t.m[i][j], v = OPT == kOptSGD ? 0.f : t.v[i][j];
+        acc += ea_elem<OPT>(x, t.g[i][j], m, v, c, hp, sc);
         t.x[i][j] = x;
         t.m[i][j] = m;
+        if (OPT != kOptSGD) t.v[i][j] = v;
       }
       center[j] = fmaf(acc, hp.inv_n, c);
     }
@@ -296,21 +314,20 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
 }
 
 // ============================================================================
-// Variant 2: lanes = (replica, float4 chunk), center tile staged in shared
-// memory by the bulk-copy engine (cp.async.bulk + mbarrier, double-buffered),
-// replica reduction by warp shuffles.
+// Variant 2 (default; SGD and Adam): lanes = (replica, float4 chunk), center
+// tile staged in shared memory by the bulk-copy engine (cp.async.bulk +
+// mbarrier, double-buffered), replica reduction by warp shuffles.
 //
-// The tiles (kTileVec float4 of a center) of all stages of the launch are
-// concatenated and split evenly over the persistent grid; a block walks its
-// contiguous tiles and thread 0 prefetches tile k+1 (possibly of the next
-// stage) with one cp.async.bulk while the block computes tile k.  Inside a
-// warp, lane l works on replica l / CH and chunk l % CH (CH = 32/NP, NP = N
-// rounded up to a power of two), so each replica's CH lanes read CH*16
-// contiguous bytes of x_i, g_i, m_i, and the NP lanes of one chunk read the
-// same center word from shared memory (a broadcast).  The N contributions of a
-// chunk are reduced with log2(NP) __shfl_xor steps; replica-0 lanes write x~.
+// A block walks its wave-scheduled tiles (kTileVec float4 of a center) and
+// thread 0 prefetches tile k+1 (possibly of the next stage) with one
+// cp.async.bulk while the block computes tile k.  Inside a warp, lane l works
+// on replica l / CH and chunk l % CH (CH = 32/NP, NP = N rounded up to a power
+// of two), so each replica's CH lanes read CH*16 contiguous bytes of x_i, g_i
+// and the optimizer state, and the NP lanes of one chunk read the same center
+// word from shared memory (a broadcast).  The N contributions of a chunk are
+// reduced with log2(NP) __shfl_xor steps; replica-0 lanes write x~.
 // ============================================================================
-constexpr int kLanePasses = 4;  // float4 chunks per lane per tile (3 loads each in flight)
+constexpr int kLanePasses = 4;  // float4 chunks per lane per tile
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
@@ -321,6 +338,9 @@ __device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
 __device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
   asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
                : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   asm volatile(
@@ -357,10 +377,11 @@ struct LaneGeom {
   static constexpr int kTileVec = (kThreads / 32) * kVecPerWarp;  // float4 of center per tile
 };
 
-template <int N, int HINT, int PASSES = kLanePasses, int MINB = 1>
+template <int N, int HINT, int OPT, int PASSES = kLanePasses, int MINB = 1>
 __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const StageBatch b, const Hyper hp) {
   using G = LaneGeom<N, PASSES>;
   constexpr int CH = G::CH, kPasses = PASSES, kVecPerWarp = G::kVecPerWarp, kTileVec = G::kTileVec;
+  constexpr bool kTwoState = OPT != kOptSGD;
   __shared__ __align__(128) float4 s_center[2][kTileVec];
   __shared__ __align__(8) uint64_t s_bar[2];
   const Mem<HINT> mem;
@@ -400,12 +421,18 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
     float* xi = nullptr;
     const float* gi = nullptr;
     float* mi = nullptr;
+    float* vi = nullptr;
 #pragma unroll
     for (int i = 0; i < N; ++i)
-      if (rep == i) { xi = st.x[i]; gi = st.g[i]; mi = st.m[i]; }
+      if (rep == i) {
+        xi = st.x[i];
+        gi = st.g[i];
+        mi = st.m[i];
+        if (kTwoState) vi = st.v[i];
+      }
 
     // replica streams first (they do not depend on the center tile)
-    float4 x[kPasses], g[kPasses], m[kPasses];
+    float4 x[kPasses], g[kPasses], m[kPasses], w[kPasses];
 #pragma unroll
     for (int k = 0; k < kPasses; ++k) {
       const int lv = warp * kVecPerWarp + k * CH + chunk;
@@ -414,6 +441,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
         x[k] = mem.ld(xi + 4 * v);
         g[k] = mem.ld_ro(gi + 4 * v);
         m[k] = mem.ld(mi + 4 * v);
+        if (kTwoState) w[k] = mem.ld(vi + 4 * v);
       }
     }
     mbar_wait(&s_bar[buf], phase[buf]);
@@ -425,10 +453,11 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       const float4 c = in ? s_center[buf][lv] : make_float4(0.f, 0.f, 0.f, 0.f);
       float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
       if (active && in) {
-        r = ea_vec(x[k], g[k], m[k], c, hp);
+        r = ea_vec<OPT>(x[k], g[k], m[k], w[k], c, hp, st.sc);
         const int64_t v = v0 + lv;
         mem.st(xi + 4 * v, x[k]);
         mem.st(mi + 4 * v, m[k]);
+        if (kTwoState) mem.st(vi + 4 * v, w[k]);
       }
 #pragma unroll
       for (int off = CH; off < 32; off <<= 1) {
@@ -447,39 +476,32 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
     nv = nv_next;
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
 
 // ============================================================================
-// Variant 3: bulk-copy load pipeline (TMA engine feeds shared memory).
+// Variant 3 (SGD): bulk-copy load pipeline (TMA engine feeds shared memory).
 //
 // One producer warp (one elected thread) streams every input of a tile --
 // x~ and x_i, g_i, m_i of all N replicas, (3N+1) 1-D cp.async.bulk copies of
-// kBulkTile float4 each -- into a kBulkStages-deep ring of shared-memory
-// slots, completing on a per-slot "full" mbarrier with the byte count.  Eight
+// kTile float4 each -- into a kStages-deep ring of shared-memory slots,
+// completing on a per-slot "full" mbarrier with the byte count.  Eight
 // consumer warps read a slot (one float4 column per thread: the x~ value is
 // shared by the N replica rows in registers), update in registers, write x_i,
 // m_i and x~ straight to HBM with 128-bit stores, and release the slot on its
-// "empty" mbarrier (one arrive per consumer warp).  Requests reach the memory
-// system as (3N+1) x 4 KB bulk reads per tile instead of 16-byte loads, and the
-// loads of up to kBulkStages tiles are in flight per SM with no registers
-// held for them.  Tiles follow the same wave schedule as the other variants.
+// "empty" mbarrier (one arrive per consumer warp).  Tiles follow the same
+// wave schedule as the other variants.
 // ============================================================================
 constexpr int kBulkConsumerWarps = 8;
 constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 
 template <int N>
 struct BulkGeom {
-  // float4 per array per tile: keep one slot <= ~56 KB
-  static constexpr int kTile = (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128;
-  static constexpr int kSlotVec = (3 * N + 1) * kTile;  // float4 per slot
+  static constexpr int kTile = (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128;  // keep a slot <= ~56 KB
+  static constexpr int kSlotVec = (3 * N + 1) * kTile;                        // float4 per slot
   static constexpr int kStages = (kSlotVec * 16 * 4 <= 200 * 1024) ? 4 : 3;
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
-
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
 
 template <int N, int HINT>
 __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
@@ -542,7 +564,8 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
           float4 x = base[(1 + 3 * i) * T + lv];
           const float4 g = base[(2 + 3 * i) * T + lv];
           float4 m = base[(3 + 3 * i) * T + lv];
-          add4(acc, ea_vec(x, g, m, c, hp));
+          float4 unused;
+          add4(acc, ea_vec<kOptSGD>(x, g, m, unused, c, hp, st.sc));
           mem.st(st.x[i] + 4 * v, x);
           mem.st(st.m[i] + 4 * v, m);
         }
@@ -552,7 +575,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
       if (lane == 0) mbar_arrive(&empty[slot]);  // release: this warp's smem reads are done
     }
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-      for (int t = 0; t < b.nstages; ++t) stage_tail<N>(b.st[t], hp);
+      for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
   }
 }
 
@@ -560,50 +583,54 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
 // Spread layout (one replica on this GPU): local step + contribution, and the
 // owner-shard epilogue after the reduce-scatter.
 // ============================================================================
-template <int U>
+template <int U, int OPT>
 __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, const float* __restrict__ g,
-                                                         float* __restrict__ m, const float* __restrict__ center,
+                                                         float* __restrict__ m, float* __restrict__ vs,
+                                                         const float* __restrict__ center,
                                                          float* __restrict__ contrib, int64_t nvec, int64_t p,
-                                                         int64_t p_pad, const Hyper hp) {
+                                                         int64_t p_pad, const Hyper hp, const StepCoef sc) {
   const Mem<0> mem;
   WaveCursor cur{0, 0};
   int sidx;
-  int64_t va0, nv0;
-  while (wave_item_f(1, [&](int) { return nvec; }, (int64_t)kThreads * U, cur, sidx, va0, nv0)) {
-    const int64_t va = va0, ve = va0 + nv0;
+  int64_t va, nv;
+  while (wave_item_f(1, [&](int) { return nvec; }, (int64_t)kThreads * U, cur, sidx, va, nv)) {
+    const int64_t ve = va + nv;
     for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
-    float4 xv[U], gv[U], mv[U], cv[U];
+      float4 xv[U], gv[U], mv[U], wv[U], cv[U];
 #pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t v = base + (int64_t)u * kThreads;
-      if (v < ve) {
-        xv[u] = mem.ld(x + 4 * v);
-        gv[u] = mem.ld_ro(g + 4 * v);
-        mv[u] = mem.ld(m + 4 * v);
-        cv[u] = mem.ld_ro(center + 4 * v);
+      for (int u = 0; u < U; ++u) {
+        const int64_t v = base + (int64_t)u * kThreads;
+        if (v < ve) {
+          xv[u] = mem.ld(x + 4 * v);
+          gv[u] = mem.ld_ro(g + 4 * v);
+          mv[u] = mem.ld(m + 4 * v);
+          if (OPT != kOptSGD) wv[u] = mem.ld(vs + 4 * v);
+          cv[u] = mem.ld_ro(center + 4 * v);
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int64_t v = base + (int64_t)u * kThreads;
+        if (v < ve) {
+          const float4 r = ea_vec<OPT>(xv[u], gv[u], mv[u], wv[u], cv[u], hp, sc);
+          mem.st(x + 4 * v, xv[u]);
+          mem.st(m + 4 * v, mv[u]);
+          if (OPT != kOptSGD) mem.st(vs + 4 * v, wv[u]);
+          mem.st(contrib + 4 * v, r);
+        }
       }
     }
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int64_t v = base + (int64_t)u * kThreads;
-      if (v < ve) {
-        const float4 r = ea_vec(xv[u], gv[u], mv[u], cv[u], hp);
-        mem.st(x + 4 * v, xv[u]);
-        mem.st(m + 4 * v, mv[u]);
-        mem.st(contrib + 4 * v, r);
-      }
-    }
-  }
   }
   // scalar tail of the vector part and the zero padding of the contribution
   const int64_t gtid = (int64_t)blockIdx.x * kThreads + threadIdx.x;
   const int64_t gsz = (int64_t)gridDim.x * kThreads;
   for (int64_t j = 4 * nvec + gtid; j < p_pad; j += gsz) {
     if (j < p) {
-      float xs = x[j], ms = m[j];
-      contrib[j] = ea_elem(xs, g[j], ms, center[j], hp);
+      float xs = x[j], ms = m[j], ws = OPT == kOptSGD ? 0.f : vs[j];
+      contrib[j] = ea_elem<OPT>(xs, g[j], ms, ws, center[j], hp, sc);
       x[j] = xs;
       m[j] = ms;
+      if (OPT != kOptSGD) vs[j] = ws;
     } else {
       contrib[j] = 0.f;
     }
@@ -626,8 +653,7 @@ __global__ void __launch_bounds__(kThreads) spread_apply(float* __restrict__ sha
 // ---------------------------------------------------------------- launch helpers
 // Grid-size knob for co-scheduling with compute (row a8):
 // AVGPIPE_EA_GRID unset/0 = persistent (#SMs x occupancy); -1 = one work
-// chunk per CTA (short CTAs the block scheduler can interleave with other
-// streams' kernels); k > 0 = at most k CTAs.
+// chunk per CTA; k > 0 = at most k CTAs.
 int grid_knob() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_GRID");
@@ -637,9 +663,9 @@ int grid_knob() {
 }
 
 template <typename K>
-int persistent_grid(K kernel, int64_t work_units, int num_sms) {
+int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads) {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, kThreads, 0) != cudaSuccess || per_sm < 1)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0) != cudaSuccess || per_sm < 1)
     per_sm = 1;
   int64_t grid = (int64_t)num_sms * per_sm;
   const int knob = grid_knob();
@@ -650,7 +676,7 @@ int persistent_grid(K kernel, int64_t work_units, int num_sms) {
   return grid < 1 ? 1 : static_cast<int>(grid);
 }
 
-// L2 eviction-hint knob: AVGPIPE_EA_L2HINT=0|1, default 0.
+// L2 eviction-hint knob: AVGPIPE_EA_L2HINT=0|1, default 0 (SGD only).
 int l2_hint() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_L2HINT");
@@ -659,12 +685,16 @@ int l2_hint() {
   return v;
 }
 
+int64_t units_of(const StageBatch& b, int64_t chunk) {
+  int64_t units = 0;
+  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + chunk - 1) / chunk;
+  return units < 1 ? 1 : units;
+}
+
 template <int N, int HINT, int U>
 cudaError_t launch_regloop_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  int64_t units = 0;
-  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kThreads * U - 1) / (kThreads * U);
   auto k = colocated_regloop<N, U, HINT>;
-  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
+  k<<<persistent_grid(k, units_of(b, kThreads * U), num_sms), kThreads, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
 
@@ -684,7 +714,7 @@ cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_regloop_u<N, HINT, U>(b, hp, num_sms, s);
 }
 
-// Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4 only).
+// Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4, SGD).
 int lane_tune() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_LANE_TUNE");
@@ -693,34 +723,24 @@ int lane_tune() {
   return v;
 }
 
-template <int N, int HINT, int PASSES, int MINB>
+template <int N, int HINT, int OPT, int PASSES, int MINB>
 cudaError_t launch_laneshfl_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  constexpr int kTileVec = LaneGeom<N, PASSES>::kTileVec;
-  int64_t units = 0;
-  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kTileVec - 1) / kTileVec;
-  if (units < 1) units = 1;
-  auto k = colocated_laneshfl<N, HINT, PASSES, MINB>;
-  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
+  auto k = colocated_laneshfl<N, HINT, OPT, PASSES, MINB>;
+  k<<<persistent_grid(k, units_of(b, LaneGeom<N, PASSES>::kTileVec), num_sms), kThreads, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
 
-template <int N, int HINT>
+template <int N, int HINT, int OPT>
 cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  if constexpr (N == 4 && HINT == 0) {
+  if constexpr (N == 4 && HINT == 0 && OPT == kOptSGD) {
     switch (lane_tune()) {
-      case 23: return launch_laneshfl_t<N, HINT, 2, 3>(b, hp, num_sms, s);
-      case 24: return launch_laneshfl_t<N, HINT, 2, 4>(b, hp, num_sms, s);
-      case 81: return launch_laneshfl_t<N, HINT, 8, 1>(b, hp, num_sms, s);
+      case 23: return launch_laneshfl_t<N, HINT, OPT, 2, 3>(b, hp, num_sms, s);
+      case 24: return launch_laneshfl_t<N, HINT, OPT, 2, 4>(b, hp, num_sms, s);
+      case 81: return launch_laneshfl_t<N, HINT, OPT, 8, 1>(b, hp, num_sms, s);
       default: break;
     }
   }
-  constexpr int kTileVec = LaneGeom<N>::kTileVec;
-  int64_t units = 0;
-  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + kTileVec - 1) / kTileVec;
-  if (units < 1) units = 1;
-  auto k = colocated_laneshfl<N, HINT>;
-  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(b, hp);
-  return cudaGetLastError();
+  return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 1>(b, hp, num_sms, s);
 }
 
 template <int N, int HINT>
@@ -729,73 +749,92 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
   auto k = colocated_bulkpipe<N, HINT>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
   if (e != cudaSuccess) return e;
-  int64_t units = 0;
-  for (int i = 0; i < b.nstages; ++i) units += (b.st[i].p / 4 + G::kTile - 1) / G::kTile;
   int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
+  const int64_t units = units_of(b, G::kTile);
   if (grid > units) grid = units;
-  if (grid < 1) grid = 1;
   k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp);
   return cudaGetLastError();
 }
 
 template <int N>
-cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int variant, int num_sms, cudaStream_t s) {
+cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (opt == kOptAdam) return launch_laneshfl<N, 0, kOptAdam>(b, hp, num_sms, s);
+  if (opt == kOptAdamW) return launch_laneshfl<N, 0, kOptAdamW>(b, hp, num_sms, s);
   const bool hint = l2_hint() != 0;
   if (variant == kVariantBulkPipe)
     return hint ? launch_bulkpipe<N, 1>(b, hp, num_sms, s) : launch_bulkpipe<N, 0>(b, hp, num_sms, s);
   if (variant == kVariantRegLoop)
     return hint ? launch_regloop<N, 1>(b, hp, num_sms, s) : launch_regloop<N, 0>(b, hp, num_sms, s);
-  return hint ? launch_laneshfl<N, 1>(b, hp, num_sms, s) : launch_laneshfl<N, 0>(b, hp, num_sms, s);
+  return hint ? launch_laneshfl<N, 1, kOptSGD>(b, hp, num_sms, s) : launch_laneshfl<N, 0, kOptSGD>(b, hp, num_sms, s);
+}
+
+template <int OPT>
+cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
+                            const StepCoef& sc, int num_sms, cudaStream_t s) {
+  constexpr int U = 2;
+  const int64_t nvec = p / 4;
+  auto k = colocated_wide<U, OPT>;
+  const int64_t units = (nvec + kThreads * U - 1) / (kThreads * U);
+  k<<<persistent_grid(k, units < 1 ? 1 : units, num_sms), kThreads, 0, s>>>(t, n, center, nvec, p, hp, sc);
+  return cudaGetLastError();
+}
+
+template <int OPT>
+cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
+                                    float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef& sc,
+                                    int num_sms, cudaStream_t s) {
+  constexpr int U = OPT == kOptSGD ? 4 : 2;
+  const int64_t nvec = p / 4;
+  auto k = spread_local<U, OPT>;
+  int64_t units = (nvec + kThreads * U - 1) / (kThreads * U);
+  if (units < 1) units = 1;
+  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(x, g, m, v, center, contrib, nvec, p, p_pad, hp, sc);
+  return cudaGetLastError();
 }
 
 }  // namespace
 
-cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int variant, int num_sms,
+cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
-  // default: the lane/shuffle kernel with the bulk-staged center (measured faster, profiles/r01_*)
-  const int v = variant == kVariantAuto ? kVariantLaneShfl : variant;
   switch (n) {
-    case 1: return launch_n<1>(b, hp, v, num_sms, s);
-    case 2: return launch_n<2>(b, hp, v, num_sms, s);
-    case 3: return launch_n<3>(b, hp, v, num_sms, s);
-    case 4: return launch_n<4>(b, hp, v, num_sms, s);
-    case 5: return launch_n<5>(b, hp, v, num_sms, s);
-    case 6: return launch_n<6>(b, hp, v, num_sms, s);
-    case 7: return launch_n<7>(b, hp, v, num_sms, s);
-    case 8: return launch_n<8>(b, hp, v, num_sms, s);
+    case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
+    case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
+    case 3: return launch_n<3>(b, hp, opt, variant, num_sms, s);
+    case 4: return launch_n<4>(b, hp, opt, variant, num_sms, s);
+    case 5: return launch_n<5>(b, hp, opt, variant, num_sms, s);
+    case 6: return launch_n<6>(b, hp, opt, variant, num_sms, s);
+    case 7: return launch_n<7>(b, hp, opt, variant, num_sms, s);
+    case 8: return launch_n<8>(b, hp, opt, variant, num_sms, s);
     default: return cudaErrorInvalidValue;
   }
 }
 
-cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
-                                  int num_sms, cudaStream_t s) {
+cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
+                                  const StepCoef& sc, int num_sms, cudaStream_t s) {
   if (p <= 0) return cudaSuccess;
-  constexpr int U = 2;
-  const int64_t nvec = p / 4;
-  auto k = colocated_wide<U>;
-  k<<<persistent_grid(k, (nvec + kUnitVec - 1) / kUnitVec, num_sms), kThreads, 0, s>>>(t, n, center, nvec, p, hp);
-  return cudaGetLastError();
+  if (opt == kOptAdam) return launch_wide_opt<kOptAdam>(t, n, center, p, hp, sc, num_sms, s);
+  if (opt == kOptAdamW) return launch_wide_opt<kOptAdamW>(t, n, center, p, hp, sc, num_sms, s);
+  return launch_wide_opt<kOptSGD>(t, n, center, p, hp, sc, num_sms, s);
 }
 
-cudaError_t launch_spread_local(float* x, const float* g, float* m, const float* center, float* contrib, int64_t p,
-                                int64_t p_pad, const Hyper& hp, int num_sms, cudaStream_t s) {
+cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef& sc, int num_sms,
+                                cudaStream_t s) {
   if (p_pad <= 0) return cudaSuccess;
-  constexpr int U = 4;
-  const int64_t nvec = p / 4;
-  auto k = spread_local<U>;
-  int64_t units = (nvec + kUnitVec - 1) / kUnitVec;
-  if (units < 1) units = 1;
-  k<<<persistent_grid(k, units, num_sms), kThreads, 0, s>>>(x, g, m, center, contrib, nvec, p, p_pad, hp);
-  return cudaGetLastError();
+  if (opt == kOptAdam)
+    return launch_spread_local_opt<kOptAdam>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+  if (opt == kOptAdamW)
+    return launch_spread_local_opt<kOptAdamW>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+  return launch_spread_local_opt<kOptSGD>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
 }
 
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,
                                 cudaStream_t s) {
   if (count <= 0) return cudaSuccess;
   const int64_t nvec = count / 4;
-  const int grid = persistent_grid(spread_apply, (nvec + kThreads - 1) / kThreads > 0 ? (nvec + kThreads - 1) / kThreads : 1,
-                                   num_sms);
+  const int64_t units = (nvec + kThreads - 1) / kThreads;
+  const int grid = persistent_grid(spread_apply, units < 1 ? 1 : units, num_sms);
   spread_apply<<<grid, kThreads, 0, s>>>(shard, reduced, nvec, count, inv_n);
   return cudaGetLastError();
 }

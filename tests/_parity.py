@@ -12,7 +12,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from oracle.ea_oracle import Hyper, ea_step
+from oracle.ea_oracle import Hyper, ea_step, ea_step_adam
 from paper_conf_ppopp_chen0qz23_b200 import synth
 
 TOL = 1e-5
@@ -32,18 +32,28 @@ def to_np(t) -> np.ndarray:
     return t.detach().cpu().numpy()
 
 
-def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nesterov=False):
+def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nesterov=False, betas=(0.9, 0.999),
+          eps=1e-8):
     a, b, r = synth.mode_coeffs(mode, n, alpha)
-    return Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=momentum, weight_decay=wd, nesterov=nesterov)
+    return Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=momentum, weight_decay=wd, nesterov=nesterov,
+                 beta1=betas[0], beta2=betas[1], eps=eps)
 
 
 class OracleStage:
-    """float64 oracle state of one stage."""
+    """float64 oracle state of one stage (optimizer 'sgd' | 'adam' | 'adamw')."""
 
-    def __init__(self, reps, center):
+    def __init__(self, reps, center, optimizer="sgd"):
         self.xs = [np.asarray(x, dtype=np.float64) for x in reps]
         self.ms = [np.zeros_like(self.xs[0]) for _ in reps]
+        self.vs = [np.zeros_like(self.xs[0]) for _ in reps]
         self.c = np.asarray(center, dtype=np.float64)
+        self.opt = optimizer
+        self.t = 0
 
     def step(self, grads, hp):
-        self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)
+        self.t += 1
+        if self.opt == "sgd":
+            self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)
+        else:
+            self.xs, self.ms, self.vs, self.c = ea_step_adam(self.xs, self.ms, self.vs, self.c, grads, hp, self.t,
+                                                             decoupled=self.opt == "adamw")

@@ -52,8 +52,8 @@ def test_abi_version(lib):
 
 
 def test_config_struct_layout_matches_header():
-    # ea_config: 2 x int32, pointer, 6 floats, 6 int32  (x86-64 alignment)
-    assert ctypes.sizeof(binding.EAConfig) == 8 + 8 + 6 * 4 + 6 * 4
+    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, 3 floats  (x86-64 alignment)
+    assert ctypes.sizeof(binding.EAConfig) == 8 + 8 + 6 * 4 + 7 * 4 + 3 * 4
     assert binding.EAConfig.stage_params.offset == 8
     assert ctypes.sizeof(binding.EAOp) == 8
 
@@ -61,7 +61,8 @@ def test_config_struct_layout_matches_header():
 def _cfg(**kw):
     sp = (ctypes.c_int64 * 2)(1000, 1001)
     base = dict(n_pipelines=2, n_stages=2, stage_params=sp, alpha=0.5, beta=0.0, rho=1.0, lr=0.05, momentum=0.9,
-                weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0)
+                weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0, optimizer=0,
+                beta1=0.9, beta2=0.999, eps=1e-8)
     base.update(kw)
     c = binding.EAConfig(**base)
     c._keep = sp
@@ -83,6 +84,10 @@ def _cfg(**kw):
     (dict(kernel_variant=9), "kernel_variant"),
     (dict(n_pipelines=65), "N must be"),
     (dict(lr=float("nan")), "finite"),
+    (dict(optimizer=3), "optimizer"),
+    (dict(optimizer=1, beta1=1.0), "betas"),
+    (dict(optimizer=2, beta2=-0.5), "betas"),
+    (dict(optimizer=1, eps=0.0), "eps"),
 ])
 def test_init_rejects_bad_config(lib, kw, needle):
     h = ctypes.c_void_p(123)
@@ -107,7 +112,10 @@ def test_null_handle_paths(lib):
     assert lib.ea_step(None, 0, None, None, None, None) == binding.EA_EINVAL
     assert lib.ea_sync(None, None) == binding.EA_EINVAL
     assert lib.ea_destroy(None) == binding.EA_OK
-    assert lib.ea_set_hyper(None, 0.5, 0, 1, 0.1, 0.9, 0, 0) == binding.EA_EINVAL
+    assert lib.ea_set_hyper(None, None) == binding.EA_EINVAL
+    assert lib.ea_get_step(None, 0, None) == binding.EA_EINVAL
+    assert lib.ea_set_step(None, 0, 1) == binding.EA_EINVAL
+    assert lib.ea_get_state(None, 0, 0, 0, None) == binding.EA_EINVAL
     assert isinstance(lib.ea_last_error(None), bytes)
 
 

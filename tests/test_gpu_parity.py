@@ -21,11 +21,11 @@ from tests._parity import TOL, OracleStage, hyper, rel_err, to_np
 
 pytestmark = pytest.mark.gpu
 
-VARIANTS = ("regloop", "laneshfl", "bulkpipe")
+VARIANTS = ("regloop", "laneshfl", "bulkpipe")  # Adam(W): lane kernel whatever the variant
 
 
 def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nesterov=False, wd=0.0, lr=synth.LR,
-                   momentum=synth.MOMENTUM, seed=0, many=False):
+                   momentum=synth.MOMENTUM, seed=0, many=False, optimizer="sgd"):
     hp = hyper(n, mode, alpha=alpha, lr=lr, momentum=momentum, wd=wd, nesterov=nesterov)
     dev = torch.device("cuda:0")
     oracle, gstreams = [], []
@@ -33,14 +33,14 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
     handles = {}
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + 97 * seed + s)
-        oracle.append(OracleStage(reps, c))
+        oracle.append(OracleStage(reps, c, optimizer))
         gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + 97 * seed + s))
         for v in variants:
             gpu[v].append(([torch.from_numpy(x).to(dev) for x in reps], torch.from_numpy(c).to(dev)))
     for v in variants:
         handles[v] = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr,
                                       momentum=hp.momentum, weight_decay=hp.weight_decay, nesterov=hp.nesterov,
-                                      kernel_variant=v)
+                                      kernel_variant=v, optimizer=optimizer, betas=(hp.beta1, hp.beta2), eps=hp.eps)
     gbuf = [[torch.empty(p, device=dev) for _ in range(n)] for p in sizes]
     order = list(reversed(range(len(sizes))))
     for t in range(steps):
@@ -67,6 +67,10 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
             for i in range(n):
                 errs.append(rel_err(to_np(reps[i]), o.xs[i]))
                 errs.append(rel_err(to_np(handles[v].momentum(s, i)), o.ms[i]))
+                if optimizer != "sgd":
+                    errs.append(rel_err(to_np(handles[v].state(s, i, 1)), o.vs[i]))
+            if optimizer != "sgd":
+                assert handles[v].get_step(s) == steps
             e = max(errs)
             worst = max(worst, e)
             assert e <= TOL, f"variant={v} stage={s} (P={sizes[s]}) rel err {e:.3e} > {TOL}"
@@ -106,6 +110,23 @@ def test_step_many_rejects_duplicates_and_bad_stage():
     h.close()
 
 
+# ------------------------------------------------------------------ Adam / AdamW (row f1)
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_adam_c1_100_steps(optimizer, mode):
+    """C1 + tail stage, 100 steps, Adam(W) as the local optimizer (all stages in one launch)."""
+    _run_colocated(2, [1_000_000, 1_000_003], 100, mode, optimizer=optimizer, lr=1e-3, wd=1e-2, many=True,
+                   variants=("auto",))
+
+
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+@pytest.mark.parametrize("n", [1, 3, 4, 8, 12])
+def test_adam_replica_counts_and_sizes(optimizer, n):
+    sizes = [100_003, 7, 4096, 33]
+    _run_colocated(n, sizes, 20, "combined", optimizer=optimizer, lr=1e-3, wd=1e-2, many=True, variants=("auto",))
+    _run_colocated(n, sizes[:1], 10, "paper", optimizer=optimizer, lr=1e-3, variants=("auto",))
+
+
 @pytest.mark.parametrize("n", [1, 3, 5, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_replica_counts(n, mode):
@@ -139,21 +160,22 @@ def _placement(rank, stage, n):
     return replica_of(rank, stage, n)
 
 
-@pytest.mark.parametrize("n", [2, 3, 4, 8])
+@pytest.mark.parametrize("n,optimizer", [(2, "sgd"), (3, "sgd"), (4, "sgd"), (8, "sgd"), (2, "adam"), (4, "adamw")])
 @pytest.mark.parametrize("mode", synth.MODES)
-def test_spread_decomposition_virtual_ranks(n, mode):
+def test_spread_decomposition_virtual_ranks(n, mode, optimizer):
     """N ranks on one GPU, external-collective mode: the real local and shard
     kernels, with the reduce-scatter / all-gather done by the test."""
     sizes = [200_003, 64]
     steps = 20
-    hp = hyper(n, mode)
+    hp = hyper(n, mode, lr=synth.LR if optimizer == "sgd" else 1e-3, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     hs = [ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
-                           layout="spread", rank=r, world=n) for r in range(n)]
+                           weight_decay=hp.weight_decay, layout="spread", rank=r, world=n, optimizer=optimizer)
+          for r in range(n)]
     oracle, gstreams, xs, centers = [], [], [], []
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
-        oracle.append(OracleStage(reps, c))
+        oracle.append(OracleStage(reps, c, optimizer))
         gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
         cap = hs[0].center_capacity(s)
         assert cap % (32 * n) == 0 and cap >= p
@@ -192,6 +214,8 @@ def test_spread_decomposition_virtual_ranks(n, mode):
             i = _placement(r, s, n)
             assert rel_err(to_np(xs[s][r]), o.xs[i]) <= TOL
             assert rel_err(to_np(hs[r].momentum(s, 0)), o.ms[i]) <= TOL
+            if optimizer != "sgd":
+                assert rel_err(to_np(hs[r].state(s, 0, 1)), o.vs[i]) <= TOL
             assert rel_err(to_np(centers[s][r][:p]), o.c) <= TOL
             assert torch.all(centers[s][r][p:] == 0), "center padding must stay zero"
     for h in hs:
@@ -281,6 +305,46 @@ def test_state_roundtrip_and_set_hyper():
     h2.close()
 
 
+def test_adam_checkpoint_resume():
+    """Both Adam moments and the step count (bias correction) survive a
+    checkpoint into a fresh handle; the resumed run equals an uninterrupted one."""
+    n, p = 3, 70_001
+    dev = torch.device("cuda:0")
+    hp = hyper(n, "combined", lr=1e-3, wd=1e-2)
+    reps, c = synth.host_state(n, p)
+    o = OracleStage(reps, c, "adamw")
+    gs = synth.GradStream(n, p)
+    xs = [torch.from_numpy(x).to(dev) for x in reps]
+    cc = torch.from_numpy(c).to(dev)
+    kw = dict(alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, weight_decay=hp.weight_decay, optimizer="adamw")
+    h = ElasticAveraging([p], n, **kw)
+    for t in range(4):
+        g = gs.next()
+        h.step(0, xs, [torch.from_numpy(a).to(dev) for a in g], cc)
+        o.step(g, hp)
+    saved = [(h.state(0, i, 0).clone(), h.state(0, i, 1).clone()) for i in range(n)]
+    t_saved = h.get_step(0)
+    assert t_saved == 4
+    h.close()
+    h2 = ElasticAveraging([p], n, **kw)
+    for i in range(n):
+        h2.set_state(0, i, saved[i][0], slot=0)
+        h2.set_state(0, i, saved[i][1], slot=1)
+    h2.set_step(0, t_saved)
+    for t in range(4):
+        g = gs.next()
+        h2.step(0, xs, [torch.from_numpy(a).to(dev) for a in g], cc)
+        o.step(g, hp)
+    torch.cuda.synchronize()
+    assert rel_err(to_np(cc), o.c) <= TOL
+    for i in range(n):
+        assert rel_err(to_np(xs[i]), o.xs[i]) <= TOL
+        assert rel_err(to_np(h2.state(0, i, 1)), o.vs[i]) <= TOL
+    with pytest.raises(EAError):
+        ElasticAveraging([p], n).state(0, 0, 1)       # SGD has one state slot
+    h2.close()
+
+
 def test_bad_pointers_rejected_before_enqueue():
     n, p = 2, 1000
     h = ElasticAveraging([p], n)
@@ -298,4 +362,50 @@ def test_bad_pointers_rejected_before_enqueue():
     st = lib.ea_step(h._h, 0, arr, arr, c.data_ptr(), None)
     assert st == binding.EA_EINVAL                                     # host memory is not device memory
     h.sync()
+    h.close()
+
+
+# ------------------------------------------------------------------ host-buffer path
+@pytest.mark.parametrize("optimizer,n", [("sgd", 2), ("sgd", 4), ("adamw", 3), ("sgd", 12)])
+def test_step_many_host_pipelined(optimizer, n):
+    """ea_step_many_host: gradients from pinned host memory in 4 Mi-element
+    chunks (a 9,000,003-element stage spans 3 ragged chunks), centers copied
+    back to host; must equal the oracle and the device-resident center."""
+    sizes = [9_000_003, 1_000, 5] if n <= 4 else [4_500_001, 77]
+    steps = 3
+    lr = synth.LR if optimizer == "sgd" else 1e-3
+    hp = hyper(n, "combined", lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+    dev = torch.device("cuda:0")
+    h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                         weight_decay=hp.weight_decay, optimizer=optimizer)
+    oracle, gstreams, xs, cs, host_out = [], [], [], [], []
+    for s, p in enumerate(sizes):
+        reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
+        oracle.append(OracleStage(reps, c, optimizer))
+        gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
+        xs.append([torch.from_numpy(x).to(dev) for x in reps])
+        cs.append(torch.from_numpy(c).to(dev))
+        host_out.append(torch.empty(p, dtype=torch.float32).pin_memory())
+    order = list(reversed(range(len(sizes))))
+    stream = torch.cuda.Stream()
+    for t in range(steps):
+        hg = {}
+        for s in range(len(sizes)):
+            g = gstreams[s].next()
+            hg[s] = [torch.from_numpy(a).pin_memory() for a in g]
+            oracle[s].step(g, hp)
+        h.step_many_host(order, [xs[s] for s in order], [hg[s] for s in order], [cs[s] for s in order],
+                         [host_out[s] for s in order], stream=stream)
+        stream.synchronize()
+        for s in range(len(sizes)):
+            assert torch.equal(host_out[s], cs[s].cpu()), "host copy of the center differs from the device center"
+    for s, p in enumerate(sizes):
+        o = oracle[s]
+        assert rel_err(host_out[s].numpy(), o.c) <= TOL
+        for i in range(n):
+            assert rel_err(to_np(xs[s][i]), o.xs[i]) <= TOL
+            assert rel_err(to_np(h.momentum(s, i)), o.ms[i]) <= TOL
+        assert h.get_step(s) == steps
+    with pytest.raises(TypeError):
+        h.step_many_host([0], [xs[0]], [[a.to(dev) for a in hg[0]]], [cs[0]], [host_out[0]])
     h.close()
