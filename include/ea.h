@@ -106,7 +106,8 @@ typedef struct {
                                    up to fp32 summation order (DESIGN.md c14).  Adam(W) always
                                    uses 2 (or the N > 8 kernel). */
   int32_t optimizer;            /* ea_optimizer */
-  float beta1, beta2;           /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999) */
+  double beta1, beta2;          /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999); double so
+                                   that 1-beta2 keeps full precision (0.999f would be off by 1.3e-5) */
   float eps;                    /* Adam(W): denominator epsilon > 0 (torch default 1e-8) */
 } ea_config;
 

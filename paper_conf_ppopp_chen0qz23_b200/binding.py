@@ -54,8 +54,8 @@ class EAConfig(ctypes.Structure):
         ("device", ctypes.c_int32),
         ("kernel_variant", ctypes.c_int32),
         ("optimizer", ctypes.c_int32),
-        ("beta1", ctypes.c_float),
-        ("beta2", ctypes.c_float),
+        ("beta1", ctypes.c_double),
+        ("beta2", ctypes.c_double),
         ("eps", ctypes.c_float),
     ]
 

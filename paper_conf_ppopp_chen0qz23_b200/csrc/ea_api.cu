@@ -86,7 +86,7 @@ ea_status check_hyper(ea_ctx* h, const ea_config& c) {
     if (c.nesterov != 0 && c.nesterov != 1) { set_err(h, "nesterov must be 0 or 1"); return EA_EINVAL; }
     if (c.nesterov && c.momentum <= 0.f) { set_err(h, "nesterov needs momentum > 0 (torch.optim.SGD rule)"); return EA_EINVAL; }
   } else if (c.optimizer == EA_OPT_ADAM || c.optimizer == EA_OPT_ADAMW) {
-    if (!(c.beta1 >= 0.f && c.beta1 < 1.f) || !(c.beta2 >= 0.f && c.beta2 < 1.f)) {
+    if (!(c.beta1 >= 0.0 && c.beta1 < 1.0) || !(c.beta2 >= 0.0 && c.beta2 < 1.0)) {
       set_err(h, "Adam betas must be in [0,1), got %g, %g", c.beta1, c.beta2);
       return EA_EINVAL;
     }
@@ -103,8 +103,8 @@ ea::Hyper make_hyper(const ea_config& c) {
   hp.alpha = c.alpha; hp.beta = c.beta; hp.rho = c.rho; hp.lr = c.lr;
   hp.momentum = c.momentum; hp.wd = c.weight_decay; hp.nesterov = c.nesterov;
   hp.inv_n = 1.0f / static_cast<float>(c.n_pipelines);
-  hp.beta1 = c.beta1; hp.one_minus_beta1 = static_cast<float>(1.0 - (double)c.beta1);
-  hp.beta2 = c.beta2; hp.one_minus_beta2 = static_cast<float>(1.0 - (double)c.beta2);
+  hp.beta1 = static_cast<float>(c.beta1); hp.one_minus_beta1 = static_cast<float>(1.0 - c.beta1);
+  hp.beta2 = static_cast<float>(c.beta2); hp.one_minus_beta2 = static_cast<float>(1.0 - c.beta2);
   hp.eps = c.eps;
   hp.lr_wd = static_cast<float>((double)c.lr * (double)c.weight_decay);
   return hp;
@@ -121,8 +121,8 @@ ea::StepCoef next_coef(ea_ctx* h, int stage) {
     sc.inv_sqrt_bc2 = 0.f;
     return sc;
   }
-  const double bc1 = 1.0 - std::pow((double)h->cfg.beta1, (double)t);
-  const double bc2 = 1.0 - std::pow((double)h->cfg.beta2, (double)t);
+  const double bc1 = 1.0 - std::pow(h->cfg.beta1, (double)t);
+  const double bc2 = 1.0 - std::pow(h->cfg.beta2, (double)t);
   sc.step_size = static_cast<float>((double)h->cfg.lr / bc1);
   sc.inv_sqrt_bc2 = static_cast<float>(1.0 / std::sqrt(bc2));
   return sc;

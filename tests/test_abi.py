@@ -52,8 +52,9 @@ def test_abi_version(lib):
 
 
 def test_config_struct_layout_matches_header():
-    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, 3 floats  (x86-64 alignment)
-    assert ctypes.sizeof(binding.EAConfig) == 8 + 8 + 6 * 4 + 7 * 4 + 3 * 4
+    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, [pad], 2 doubles, 1 float, [pad]  (x86-64 alignment)
+    assert ctypes.sizeof(binding.EAConfig) == 96
+    assert binding.EAConfig.beta1.offset == 72 and binding.EAConfig.eps.offset == 88
     assert binding.EAConfig.stage_params.offset == 8
     assert ctypes.sizeof(binding.EAOp) == 8
 
@@ -159,3 +160,26 @@ def test_schedule_rejects_bad_args(lib):
     assert lib.ea_schedule(2, 9, 0, 1, out, 16) == -binding.EA_EINVAL      # cap < 2M
     assert lib.ea_schedule(2, 4, 0, 1, None, 8) == -binding.EA_EINVAL
     assert lib.ea_schedule(2, 0, 0, 1, None, 0) == 0
+
+
+def test_config_layout_matches_c_compiler(tmp_path):
+    """sizeof/offsetof of every ea_config / ea_op field as gcc lays out
+    include/ea.h must equal the ctypes mirror in the binding."""
+    import shutil
+    if not shutil.which("gcc"):
+        pytest.skip("gcc not available")
+    fields = [f for f, _ in binding.EAConfig._fields_]
+    src = ['#include <stdio.h>', '#include <stddef.h>', '#include "ea.h"', 'int main(void) {',
+           '  printf("%zu %zu\\n", sizeof(ea_config), sizeof(ea_op));']
+    for f in fields:
+        src.append(f'  printf("%zu\\n", offsetof(ea_config, {f}));')
+    src.append("  return 0; }")
+    c = tmp_path / "layout.c"
+    c.write_text("\n".join(src))
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-I", os.path.join(ROOT, "include"), str(c), "-o", str(exe)], check=True)
+    out = subprocess.run([str(exe)], capture_output=True, text=True, check=True).stdout.split()
+    assert int(out[0]) == ctypes.sizeof(binding.EAConfig)
+    assert int(out[1]) == ctypes.sizeof(binding.EAOp)
+    for f, off in zip(fields, out[2:]):
+        assert int(off) == getattr(binding.EAConfig, f).offset, f
