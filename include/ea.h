@@ -252,6 +252,49 @@ EA_API const char* ea_last_error(ea_handle h);
  * of range, cap < 2M or out == NULL (with M > 0).  Host only; no GPU needed. */
 EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
 
+/* ---- Profiling-based tuning predictor (§5.2, Eqs. (1)-(8); host only) ---- */
+
+/* One profiled setting: M = m micro-batches, N = n parallel pipelines, K GPUs. */
+typedef struct {
+  int32_t n_gpus;         /* K >= 1 */
+  int32_t m, n;           /* profiled micro-batches per batch and pipelines, >= 1 */
+  int32_t n_samples;      /* samples per utilisation curve (>= 0) */
+  double dt;              /* seconds between samples */
+  const double* phi;      /* K x n_samples, row-major: GPU k's utilisation phi^k(t) in [0, 1] */
+  const double* t_gpu;    /* K: computation time per batch T_gpu^k (s) */
+  const double* t_comm;   /* K: total communication time per batch TT^k (s) */
+  const double* f_mod;    /* K: parallel + reference model footprint F_mod^k (bytes) */
+  const double* f_dat;    /* K: data / intermediate-result footprint F_dat^k (bytes) */
+} ea_profile;
+
+/* Prediction for one GPU at a candidate (m*, n*). */
+typedef struct {
+  double t_gpu;    /* Eq. (2) */
+  double t_com;    /* Eq. (4) */
+  double t_up;     /* Eq. (6) */
+  double t_down;   /* Eq. (7) */
+  double t_bub;    /* Eq. (5) */
+  double t_total;  /* Eq. (1) */
+  double mem;      /* Eq. (8) */
+} ea_gpu_prediction;
+
+typedef enum { EA_TUNE_THROUGHPUT = 0, EA_TUNE_TIME = 1 } ea_tune_objective;
+
+/* Predict every GPU's time decomposition and memory at (m_star, n_star).
+ * out: K entries (may be NULL); *iter_time = max_k t_total; *peak_mem =
+ * max_k mem (either may be NULL).  EA_EINVAL on a malformed profile (NULL
+ * arrays, negative or non-finite values, phi outside [0, 1]) or m*, n* < 1. */
+EA_API ea_status ea_predict(const ea_profile* prof, int32_t m_star, int32_t n_star, ea_gpu_prediction* out,
+                            double* iter_time, double* peak_mem);
+
+/* Choose (m*, n*) from the candidate lists: the highest throughput
+ * n* / T* (EA_TUNE_THROUGHPUT) or the lowest T* (EA_TUNE_TIME) among settings
+ * whose peak memory <= mem_limit; ties go to lower memory, then smaller n*,
+ * then smaller m*.  EA_ESTATE (best = -1) if nothing fits the limit. */
+EA_API ea_status ea_tune(const ea_profile* prof, const int32_t* m_cands, int32_t n_m, const int32_t* n_cands,
+                         int32_t n_n, double mem_limit, int32_t objective, int32_t* best_m, int32_t* best_n,
+                         double* best_iter_time);
+
 #ifdef __cplusplus
 }
 #endif

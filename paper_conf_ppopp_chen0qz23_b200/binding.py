@@ -64,6 +64,18 @@ class EAOp(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("micro_batch", ctypes.c_int32)]
 
 
+class EAProfile(ctypes.Structure):
+    _fields_ = [("n_gpus", ctypes.c_int32), ("m", ctypes.c_int32), ("n", ctypes.c_int32),
+                ("n_samples", ctypes.c_int32), ("dt", ctypes.c_double),
+                ("phi", ctypes.POINTER(ctypes.c_double)), ("t_gpu", ctypes.POINTER(ctypes.c_double)),
+                ("t_comm", ctypes.POINTER(ctypes.c_double)), ("f_mod", ctypes.POINTER(ctypes.c_double)),
+                ("f_dat", ctypes.POINTER(ctypes.c_double))]
+
+
+class EAGpuPrediction(ctypes.Structure):
+    _fields_ = [(f, ctypes.c_double) for f in ("t_gpu", "t_com", "t_up", "t_down", "t_bub", "t_total", "mem")]
+
+
 # name -> (restype, argtypes); mirrors include/ea.h one to one.
 _VP = ctypes.c_void_p
 _FPP = ctypes.POINTER(ctypes.c_void_p)
@@ -87,6 +99,13 @@ SIGNATURES = {
     "ea_set_hyper": (ctypes.c_int, [_VP, ctypes.POINTER(EAConfig)]),
     "ea_destroy": (ctypes.c_int, [_VP]),
     "ea_last_error": (ctypes.c_char_p, [_VP]),
+    "ea_predict": (ctypes.c_int, [ctypes.POINTER(EAProfile), ctypes.c_int32, ctypes.c_int32,
+                                  ctypes.POINTER(EAGpuPrediction), ctypes.POINTER(ctypes.c_double),
+                                  ctypes.POINTER(ctypes.c_double)]),
+    "ea_tune": (ctypes.c_int, [ctypes.POINTER(EAProfile), ctypes.POINTER(ctypes.c_int32), ctypes.c_int32,
+                               ctypes.POINTER(ctypes.c_int32), ctypes.c_int32, ctypes.c_double, ctypes.c_int32,
+                               ctypes.POINTER(ctypes.c_int32), ctypes.POINTER(ctypes.c_int32),
+                               ctypes.POINTER(ctypes.c_double)]),
     "ea_schedule": (ctypes.c_int32, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
                                      ctypes.POINTER(EAOp), ctypes.c_int32]),
 }
@@ -141,6 +160,50 @@ def schedule(K: int, M: int, stage: int, advance: int) -> List[Tuple[str, int]]:
     if n < 0:
         raise EAError(-n, f"ea_schedule(K={K}, M={M}, stage={stage}, advance={advance}) rejected")
     return [("F" if out[i].kind == 0 else "B", out[i].micro_batch) for i in range(n)]
+
+
+def _make_profile(m, n, dt, phi, t_gpu, t_comm, f_mod, f_dat):
+    """Marshal a profile (sequences / numpy arrays) into an EAProfile; the
+    returned tuple keeps the ctypes buffers alive."""
+    K = len(t_gpu)
+    rows = [list(map(float, r)) for r in phi] if len(phi) else [[] for _ in range(K)]
+    S = len(rows[0]) if rows else 0
+    if len(rows) != K or any(len(r) != S for r in rows):
+        raise ValueError("phi must be K rows of equal length")
+    arr = lambda v: (ctypes.c_double * max(len(v), 1))(*map(float, v))
+    flat = arr([x for r in rows for x in r])
+    bufs = [flat, arr(t_gpu), arr(t_comm), arr(f_mod), arr(f_dat)]
+    prof = EAProfile(K, int(m), int(n), S, float(dt), *[ctypes.cast(b, ctypes.POINTER(ctypes.c_double)) for b in bufs])
+    return prof, bufs
+
+
+def predict(m, n, dt, phi, t_gpu, t_comm, f_mod, f_dat, m_star, n_star):
+    """ea_predict: per-GPU predictions (list of dicts), iteration time, peak memory."""
+    prof, _keep = _make_profile(m, n, dt, phi, t_gpu, t_comm, f_mod, f_dat)
+    out = (EAGpuPrediction * prof.n_gpus)()
+    it, pk = ctypes.c_double(), ctypes.c_double()
+    st = load_library().ea_predict(ctypes.byref(prof), int(m_star), int(n_star), out, ctypes.byref(it),
+                                   ctypes.byref(pk))
+    if st != EA_OK:
+        raise EAError(st, "ea_predict rejected the profile or (m*, n*)")
+    per = [{f: getattr(o, f) for f, _ in EAGpuPrediction._fields_} for o in out]
+    return per, it.value, pk.value
+
+
+def tune(m, n, dt, phi, t_gpu, t_comm, f_mod, f_dat, m_cands, n_cands, mem_limit, objective="throughput"):
+    """ea_tune: (m*, n*, iteration time) or None if no candidate fits mem_limit."""
+    prof, _keep = _make_profile(m, n, dt, phi, t_gpu, t_comm, f_mod, f_dat)
+    mc = (ctypes.c_int32 * len(m_cands))(*m_cands)
+    nc = (ctypes.c_int32 * len(n_cands))(*n_cands)
+    bm, bn, bt = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_double()
+    st = load_library().ea_tune(ctypes.byref(prof), mc, len(m_cands), nc, len(n_cands), float(mem_limit),
+                                {"throughput": 0, "time": 1}[objective], ctypes.byref(bm), ctypes.byref(bn),
+                                ctypes.byref(bt))
+    if st == EA_ESTATE:
+        return None
+    if st != EA_OK:
+        raise EAError(st, "ea_tune rejected its arguments")
+    return bm.value, bn.value, bt.value
 
 
 def _stream_ptr(stream) -> Optional[int]:
