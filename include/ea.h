@@ -252,6 +252,29 @@ EA_API const char* ea_last_error(ea_handle h);
  * of range, cap < 2M or out == NULL (with M > 0).  Host only; no GPU needed. */
 EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
 
+/* ---- Run-time advance adjustment (Algorithm 1 lines 1, 9-10) ---- */
+
+/* Controller state (plain data, caller-owned; DESIGN.md c27). */
+typedef struct {
+  int32_t K, M;          /* pipeline depth and micro-batches per batch */
+  int32_t advance_num;   /* forwards in advance on the first stage (starts at K-1: 1F1B) */
+  int32_t has_last;      /* a previous batch time is recorded */
+  double last_time;      /* previous batch time */
+} ea_advance_ctl;
+
+/* Line 1: advance_num = min(K-1, M).  EA_EINVAL for K < 1, M < 0 or ctl == NULL. */
+EA_API ea_status ea_advance_init(ea_advance_ctl* ctl, int32_t K, int32_t M);
+
+/* Lines 9-10 after one batch: if the batch was faster than the previous one
+ * (the first batch counts as faster) and peak_mem + mem_per_microbatch <=
+ * mem_limit, advance_num++ (capped at M).  Returns the new advance_num, or
+ * -EA_EINVAL on NULL / NaN arguments. */
+EA_API int32_t ea_advance_update(ea_advance_ctl* ctl, double batch_time, double peak_mem, double mem_per_microbatch,
+                                 double mem_limit);
+
+/* Advance of `stage` (0-based): min(M, K-1-stage + advance_num - min(K-1, M)) (c15); -EA_EINVAL if out of range. */
+EA_API int32_t ea_advance_for_stage(const ea_advance_ctl* ctl, int32_t stage);
+
 /* ---- Profiling-based tuning predictor (§5.2, Eqs. (1)-(8); host only) ---- */
 
 /* One profiled setting: M = m micro-batches, N = n parallel pipelines, K GPUs. */

@@ -99,3 +99,48 @@ def simulate_pipeline(K: int, M: int, advances: Sequence[int]) -> Dict[str, obje
                 progressed = True
     ok = all(pos[k] == len(lists[k]) for k in range(K))
     return {"ok": ok, "order": order}
+
+
+class AdvanceController:
+    """Algorithm 1's run-time adjustment of ``advance_num``.
+
+    Line 1: advance_num <- K - 1 (1F1B on GPU 1).  After every batch (lines
+    9-10): if is_faster() and is_mem_available() then advance_num++.
+
+    Readings (DESIGN.md c27):
+      is_faster()        the batch just finished took strictly less time than
+                         the batch before it; the first batch has nothing to
+                         compare with and counts as faster (exploration starts).
+      is_mem_available() peak memory of the batch + the activation stash of one
+                         more micro-batch <= the user's limit (one more forward
+                         in advance holds one more micro-batch).
+      advance_num never exceeds M (AFAB) and never decreases.
+      GPU k (1-based) runs min(M, K - k + extra) with extra = advance_num - (K-1) (c15).
+    """
+
+    def __init__(self, K: int, M: int):
+        if K < 1 or M < 0:
+            raise ValueError("need K >= 1 and M >= 0")
+        self.K, self.M = K, M
+        self.advance_num = min(K - 1, M)      # Alg. 1 line 1
+        self.last_time = None
+
+    def is_faster(self, batch_time: float) -> bool:
+        return self.last_time is None or batch_time < self.last_time
+
+    @staticmethod
+    def is_mem_available(peak_mem: float, mem_per_microbatch: float, mem_limit: float) -> bool:
+        return peak_mem + mem_per_microbatch <= mem_limit
+
+    def update(self, batch_time: float, peak_mem: float, mem_per_microbatch: float, mem_limit: float) -> int:
+        """Lines 9-10 after one batch; returns the advance_num for the next batch."""
+        if self.is_faster(batch_time) and self.is_mem_available(peak_mem, mem_per_microbatch, mem_limit):
+            if self.advance_num < self.M:
+                self.advance_num += 1
+        self.last_time = batch_time
+        return self.advance_num
+
+    def advance_for(self, k: int) -> int:
+        """advance of GPU k (1-based)."""
+        extra = self.advance_num - min(self.K - 1, self.M)
+        return default_advance(self.K, self.M, k, extra)

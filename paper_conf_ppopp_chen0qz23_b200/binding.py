@@ -64,6 +64,36 @@ class EAOp(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("micro_batch", ctypes.c_int32)]
 
 
+class EAAdvanceCtl(ctypes.Structure):
+    _fields_ = [("K", ctypes.c_int32), ("M", ctypes.c_int32), ("advance_num", ctypes.c_int32),
+                ("has_last", ctypes.c_int32), ("last_time", ctypes.c_double)]
+
+
+class AdvanceController:
+    """Algorithm 1's run-time advance_num adjustment (ea_advance_*)."""
+
+    def __init__(self, K: int, M: int):
+        self.ctl = EAAdvanceCtl()
+        _check(load_library().ea_advance_init(ctypes.byref(self.ctl), K, M))
+
+    @property
+    def advance_num(self) -> int:
+        return self.ctl.advance_num
+
+    def update(self, batch_time: float, peak_mem: float, mem_per_microbatch: float, mem_limit: float) -> int:
+        r = load_library().ea_advance_update(ctypes.byref(self.ctl), batch_time, peak_mem, mem_per_microbatch,
+                                             mem_limit)
+        if r < 0:
+            raise EAError(-r, "ea_advance_update rejected its arguments")
+        return r
+
+    def advance_for_stage(self, stage: int) -> int:
+        r = load_library().ea_advance_for_stage(ctypes.byref(self.ctl), stage)
+        if r < 0:
+            raise EAError(-r, f"bad stage {stage}")
+        return r
+
+
 class EAProfile(ctypes.Structure):
     _fields_ = [("n_gpus", ctypes.c_int32), ("m", ctypes.c_int32), ("n", ctypes.c_int32),
                 ("n_samples", ctypes.c_int32), ("dt", ctypes.c_double),
@@ -99,6 +129,10 @@ SIGNATURES = {
     "ea_set_hyper": (ctypes.c_int, [_VP, ctypes.POINTER(EAConfig)]),
     "ea_destroy": (ctypes.c_int, [_VP]),
     "ea_last_error": (ctypes.c_char_p, [_VP]),
+    "ea_advance_init": (ctypes.c_int, [ctypes.POINTER(EAAdvanceCtl), ctypes.c_int32, ctypes.c_int32]),
+    "ea_advance_update": (ctypes.c_int32, [ctypes.POINTER(EAAdvanceCtl), ctypes.c_double, ctypes.c_double,
+                                           ctypes.c_double, ctypes.c_double]),
+    "ea_advance_for_stage": (ctypes.c_int32, [ctypes.POINTER(EAAdvanceCtl), ctypes.c_int32]),
     "ea_predict": (ctypes.c_int, [ctypes.POINTER(EAProfile), ctypes.c_int32, ctypes.c_int32,
                                   ctypes.POINTER(EAGpuPrediction), ctypes.POINTER(ctypes.c_double),
                                   ctypes.POINTER(ctypes.c_double)]),

@@ -714,7 +714,8 @@ cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_regloop_u<N, HINT, U>(b, hp, num_sms, s);
 }
 
-// Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4, SGD).
+// Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4,
+// SGD), "22", "23", "31" (N=4, Adam).
 int lane_tune() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_LANE_TUNE");
@@ -737,6 +738,14 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
       case 23: return launch_laneshfl_t<N, HINT, OPT, 2, 3>(b, hp, num_sms, s);
       case 24: return launch_laneshfl_t<N, HINT, OPT, 2, 4>(b, hp, num_sms, s);
       case 81: return launch_laneshfl_t<N, HINT, OPT, 8, 1>(b, hp, num_sms, s);
+      default: break;
+    }
+  }
+  if constexpr (N == 4 && HINT == 0 && OPT == kOptAdam) {
+    switch (lane_tune()) {
+      case 22: return launch_laneshfl_t<N, HINT, OPT, 2, 2>(b, hp, num_sms, s);
+      case 23: return launch_laneshfl_t<N, HINT, OPT, 2, 3>(b, hp, num_sms, s);
+      case 31: return launch_laneshfl_t<N, HINT, OPT, 3, 1>(b, hp, num_sms, s);
       default: break;
     }
   }

@@ -183,3 +183,19 @@ def test_config_layout_matches_c_compiler(tmp_path):
     assert int(out[1]) == ctypes.sizeof(binding.EAOp)
     for f, off in zip(fields, out[2:]):
         assert int(off) == getattr(binding.EAConfig, f).offset, f
+
+
+def test_advance_controller_native_equals_oracle(lib):
+    """ea_advance_* (Alg. 1 lines 1, 9-10) bit-exact against oracle.schedule.AdvanceController."""
+    from oracle.schedule import AdvanceController as OracleCtl
+    rnd = random.Random(5)
+    for _ in range(300):
+        K, M = rnd.randint(1, 12), rnd.randint(0, 64)
+        a, b = OracleCtl(K, M), binding.AdvanceController(K, M)
+        assert a.advance_num == b.advance_num
+        limit = rnd.uniform(5, 50)
+        for _ in range(rnd.randint(1, 40)):
+            t = rnd.choice([rnd.uniform(1, 10), a.last_time if a.last_time is not None else 3.0])
+            peak, per = rnd.uniform(0, 50), rnd.uniform(0, 5)
+            assert a.update(t, peak, per, limit) == b.update(t, peak, per, limit)
+            assert [a.advance_for(k) for k in range(1, K + 1)] == [b.advance_for_stage(s) for s in range(K)]

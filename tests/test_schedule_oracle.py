@@ -101,3 +101,39 @@ def test_default_advance_is_feasible():
             for e in range(0, 4):
                 adv = [default_advance(K, M, k, e) for k in range(1, K + 1)]
                 assert simulate_pipeline(K, M, adv)["ok"]
+
+
+# ---------------------------------------------------------------- Alg. 1 lines 9-10 (row f2)
+from oracle.schedule import AdvanceController  # noqa: E402
+
+
+def test_controller_starts_at_1f1b_and_grows_to_afab():
+    ctl = AdvanceController(K=4, M=8)
+    assert ctl.advance_num == 3                                      # line 1: K-1 (1F1B)
+    assert [ctl.advance_for(k) for k in range(1, 5)] == [3, 2, 1, 0]
+    t = 10.0
+    for expect in [4, 5, 6, 7, 8, 8, 8]:                             # always faster, plenty of memory
+        t -= 1.0
+        assert ctl.update(t, peak_mem=1.0, mem_per_microbatch=0.1, mem_limit=100.0) == expect
+    assert peak_in_flight(advance_forward_schedule(4, 8, 1, ctl.advance_for(1))) == 8   # AFAB
+
+
+def test_controller_stops_at_the_memory_limit():
+    ctl = AdvanceController(K=2, M=8)
+    per_mb, limit = 1.0, 5.0
+    t = 100.0
+    for _ in range(10):
+        peak = per_mb * peak_in_flight(advance_forward_schedule(2, 8, 1, ctl.advance_num))
+        t -= 1.0
+        ctl.update(t, peak, per_mb, limit)
+    # stash = advance + 1 micro-batches; growth stops once one more would exceed the limit
+    assert ctl.advance_num == 4
+    assert peak_in_flight(advance_forward_schedule(2, 8, 1, ctl.advance_num)) * per_mb == limit
+
+
+def test_controller_holds_when_not_faster():
+    ctl = AdvanceController(K=3, M=16)
+    assert ctl.advance_num == 2
+    # first batch counts as faster -> 3; 9 < 10 -> 4; 9.5 not faster; 9.5 not < 9.5; 8 < 9.5 -> 5; 8 not < 8
+    for t, expect in [(10.0, 3), (9.0, 4), (9.5, 4), (9.5, 4), (8.0, 5), (8.0, 5)]:
+        assert ctl.update(t, 0.0, 1.0, 1e9) == expect
