@@ -14,6 +14,9 @@ timeout 600 python bench.py >> gpurun_out/bench.json 2> gpurun_out/bench.err
 for v in "--optimizer adam" "--optimizer adamw" "--variant regloop" "--variant bulkpipe" ${EXTRA_BENCH}; do
   timeout 300 python bench.py $v --no-e2e --no-cpu-baseline >> gpurun_out/bench.json 2>> gpurun_out/bench.err
 done
+for t in 22 23 31; do
+  AVGPIPE_EA_LANE_TUNE=$t timeout 300 python bench.py --optimizer adam --no-e2e --no-cpu-baseline | sed "s/^{/{\"tune\": \"$t\", /" >> gpurun_out/bench_tune_adam.json 2>> gpurun_out/bench.err
+done
 timeout 300 python bench.py --impl reference --steps 200 --warmup 3 > gpurun_out/bench_reference.json 2>> gpurun_out/bench.err
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -k regex:"colocated|spread" -c 60 --csv --log-file gpurun_out/launches.csv \
     python bench.py --steps 50 --warmup 5 --no-e2e --no-cpu-baseline > gpurun_out/ncu_launch_bench.log 2>&1
