@@ -83,6 +83,14 @@ typedef enum { EA_COLOCATED = 0, EA_SPREAD = 1 } ea_layout;
  * trains with Adam and SGD). */
 typedef enum { EA_OPT_SGD = 0, EA_OPT_ADAM = 1, EA_OPT_ADAMW = 2 } ea_optimizer;
 
+/* How EA_SPREAD exchanges contributions and the center (rows a6/a7). */
+typedef enum {
+  EA_XCHG_NCCL = 0,  /* ncclReduceScatter -> shard update kernel -> in-place ncclAllGather on a side stream */
+  EA_XCHG_P2P = 1    /* ONE fused kernel per stage: local update, contributions pushed into the owners'
+                        inboxes over NVLink peer memory (CUDA IPC), owner reduction + center update,
+                        center chunks pulled back -- overlapped chunk by chunk (see ea_p2p.cu) */
+} ea_exchange;
+
 typedef struct {
   int32_t n_pipelines;          /* N >= 1 parallel pipelines */
   int32_t n_stages;             /* stages hosted by this process, >= 1 */
@@ -109,6 +117,7 @@ typedef struct {
   double beta1, beta2;          /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999); double so
                                    that 1-beta2 keeps full precision (0.999f would be off by 1.3e-5) */
   float eps;                    /* Adam(W): denominator epsilon > 0 (torch default 1e-8) */
+  int32_t exchange;             /* EA_SPREAD: ea_exchange (ignored for EA_COLOCATED) */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;
@@ -190,6 +199,15 @@ EA_API ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages,
 EA_API ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
                                    const float* const* host_grad_ptrs, float* const* center_ptrs,
                                    float* const* host_center_out, void* stream);
+
+/* EA_XCHG_P2P between handles of ONE process (e.g. N ranks on one device, or
+ * N devices driven by one process): peers[q] is rank q's handle (peers[rank]
+ * == h); every handle must call this with the same list.  Ranks created with
+ * an NCCL id are connected by ea_init itself (CUDA IPC handles all-gathered
+ * over NCCL) and need no call.  All ranks' ea_step kernels wait for one
+ * another, so each rank must drive its own stream; ranks that share a device
+ * split its SMs.  EA_ESTATE for other layouts/exchanges. */
+EA_API ea_status ea_p2p_connect(ea_handle h, const ea_handle* peers, int32_t world);
 
 /* Make `stream` wait until every center update enqueued so far is complete,
  * then report any asynchronous CUDA/NCCL error seen so far.  Does not block

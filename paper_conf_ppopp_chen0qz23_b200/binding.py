@@ -22,6 +22,7 @@ STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA
 LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
 VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3}
 OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2}
+EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
 ABI_VERSION = 2
 
@@ -57,6 +58,7 @@ class EAConfig(ctypes.Structure):
         ("beta1", ctypes.c_double),
         ("beta2", ctypes.c_double),
         ("eps", ctypes.c_float),
+        ("exchange", ctypes.c_int32),
     ]
 
 
@@ -119,6 +121,7 @@ SIGNATURES = {
     "ea_step_many": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP, _VP]),
     "ea_step_many_host": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP,
                                          _FPP, _VP]),
+    "ea_p2p_connect": (ctypes.c_int, [_VP, ctypes.POINTER(_VP), ctypes.c_int32]),
     "ea_sync": (ctypes.c_int, [_VP, _VP]),
     "ea_spread_local": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP, _VP, _VP]),
     "ea_spread_apply": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP]),
@@ -272,7 +275,8 @@ class ElasticAveraging:
                  beta: float = 0.0, rho: float = 1.0, lr: float = 0.05, momentum: float = 0.0,
                  weight_decay: float = 0.0, nesterov: bool = False, layout: str = "colocated", rank: int = 0,
                  world: int = 1, device: Optional[int] = None, kernel_variant: str = "auto",
-                 nccl_id: Optional[bytes] = None, optimizer: str = "sgd", betas=(0.9, 0.999), eps: float = 1e-8):
+                 nccl_id: Optional[bytes] = None, optimizer: str = "sgd", betas=(0.9, 0.999), eps: float = 1e-8,
+                 exchange: str = "nccl"):
         import torch
         self._lib = load_library()
         self.n = int(n_pipelines)
@@ -287,7 +291,7 @@ class ElasticAveraging:
                        1.0 / self.n if alpha is None else float(alpha), float(beta), float(rho), float(lr),
                        float(momentum), float(weight_decay), int(bool(nesterov)), LAYOUTS[layout], int(rank),
                        int(world), self.device, VARIANTS[kernel_variant], OPTIMIZERS[optimizer],
-                       float(betas[0]), float(betas[1]), float(eps))
+                       float(betas[0]), float(betas[1]), float(eps), EXCHANGES[exchange])
         self._cfg = cfg
         self.rank, self.world = int(rank), int(world)
         idbuf = None
@@ -360,6 +364,14 @@ class ElasticAveraging:
         ca = (ctypes.c_void_p * k)(*[_ptr(c, "center") for c in centers])
         oa = (ctypes.c_void_p * k)(*[_host_ptr(c, "host center out") for c in host_centers_out])
         _check(self._lib.ea_step_many_host(self._h, len(stages), st, ra, ga, ca, oa, _stream_ptr(stream)), self._h)
+
+    @staticmethod
+    def p2p_connect(handles):
+        """Connect in-process EA_XCHG_P2P ranks (handles[q] = rank q)."""
+        lib = load_library()
+        arr = (ctypes.c_void_p * len(handles))(*[h._h.value for h in handles])
+        for h in handles:
+            _check(lib.ea_p2p_connect(h._h, arr, len(handles)), h._h)
 
     def sync(self, stream=None):
         _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)

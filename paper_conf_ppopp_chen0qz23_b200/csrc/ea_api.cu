@@ -11,6 +11,7 @@
 #include <stdint.h>
 
 #include <cmath>
+#include <cstdlib>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -37,6 +38,17 @@ struct ea_ctx {
   float* contrib = nullptr;  // max P_pad floats
   float* reduced = nullptr;  // max P_pad/N floats
   ncclComm_t comm = nullptr;
+  // EA_SPREAD with exchange == EA_XCHG_P2P (fused peer-memory kernel)
+  char* xbuf = nullptr;  // this rank's exchange buffer (exported by CUDA IPC)
+  size_t xbuf_bytes = 0;
+  std::vector<size_t> x_inbox, x_outbox, x_arrive, x_ready;  // per-stage byte offsets into xbuf
+  std::vector<int64_t> x_nchunks, x_slots;
+  std::vector<char*> peer_base;   // world entries, as mapped on this device (self = xbuf)
+  std::vector<char> peer_ipc;     // 1 = opened with cudaIpcOpenMemHandle (closed at destroy)
+  bool p2p_ready = false;
+  int same_device_ranks = 1;
+  uint32_t* err_host = nullptr;   // host-mapped exchange error flag
+  uint32_t* err_dev = nullptr;
   // host-buffer path (ea_step_many_host), allocated on first use
   cudaStream_t h2d = nullptr, d2h = nullptr;
   float* staging[2] = {nullptr, nullptr};  // N * kHostChunk floats each
@@ -46,6 +58,8 @@ struct ea_ctx {
 
 // Elements per pipelined chunk of the host-buffer path (a multiple of 64).
 constexpr int64_t kHostChunk = 4 << 20;
+// Floats per exchange chunk of the fused peer-memory spread kernel (32 KB).
+constexpr int64_t kP2PChunk = 8192;
 
 namespace {
 
@@ -159,6 +173,10 @@ void free_ctx(ea_ctx* h) {
     if (h->ev_kern[i]) cudaEventDestroy(h->ev_kern[i]);
   }
   if (h->ev_d2h) cudaEventDestroy(h->ev_d2h);
+  for (size_t i = 0; i < h->peer_base.size(); ++i)
+    if (i < h->peer_ipc.size() && h->peer_ipc[i] && h->peer_base[i]) cudaIpcCloseMemHandle(h->peer_base[i]);
+  if (h->xbuf) cudaFree(h->xbuf);
+  if (h->err_host) cudaFreeHost(h->err_host);
   if (h->h2d) cudaStreamDestroy(h->h2d);
   if (h->d2h) cudaStreamDestroy(h->d2h);
   delete h;
@@ -240,7 +258,10 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
 }
 
 // Spread: one stage's exchange on the side stream (rows a6-a8).
+ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s);
+
 ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s) {
+  if (h->cfg.exchange == EA_XCHG_P2P) return p2p_step(h, stage, replica, grad, center_ptr, s);
   if (!h->comm) {
     set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
     return EA_ESTATE;
@@ -274,6 +295,128 @@ ea_status join_side(ea_ctx* h, cudaStream_t s) {
   cudaError_t e;
   if ((e = cudaEventRecord(h->ev_done, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   if ((e = cudaStreamWaitEvent(s, h->ev_done, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  return EA_OK;
+}
+
+uint64_t p2p_timeout_ns() {
+  const char* e = std::getenv("AVGPIPE_EA_P2P_TIMEOUT_MS");
+  const long long ms = e ? std::atoll(e) : 30000;
+  return static_cast<uint64_t>(ms > 0 ? ms : 30000) * 1000000ull;
+}
+
+// Lay out and allocate this rank's exchange buffer (per stage: inbox, outbox, counters).
+ea_status p2p_alloc(ea_ctx* h) {
+  const int n = h->cfg.n_pipelines;
+  size_t off = 0;
+  auto take = [&](size_t bytes) {
+    const size_t at = off;
+    off += (bytes + 255) / 256 * 256;
+    return at;
+  };
+  for (int s = 0; s < h->cfg.n_stages; ++s) {
+    const int64_t nch = (h->p_pad[s] + kP2PChunk - 1) / kP2PChunk;
+    const int64_t slots = (nch + n - 1) / n;
+    h->x_nchunks.push_back(nch);
+    h->x_slots.push_back(slots);
+    h->x_inbox.push_back(take(sizeof(float) * (size_t)n * slots * kP2PChunk));
+    h->x_outbox.push_back(take(sizeof(float) * (size_t)slots * kP2PChunk));
+    h->x_arrive.push_back(take(sizeof(uint32_t) * (size_t)slots));
+    h->x_ready.push_back(take(sizeof(uint32_t) * (size_t)slots));
+  }
+  h->xbuf_bytes = off;
+  cudaError_t e;
+  if ((e = cudaMalloc(&h->xbuf, off)) != cudaSuccess) return cuda_fail(h, e, "exchange buffer");
+  if ((e = cudaMemset(h->xbuf, 0, off)) != cudaSuccess) return cuda_fail(h, e, "exchange buffer init");
+  if ((e = cudaHostAlloc(&h->err_host, sizeof(uint32_t), cudaHostAllocMapped)) != cudaSuccess)
+    return cuda_fail(h, e, "error flag");
+  *h->err_host = 0;
+  if ((e = cudaHostGetDevicePointer(&h->err_dev, h->err_host, 0)) != cudaSuccess) return cuda_fail(h, e, "error flag");
+  h->peer_base.assign(n, nullptr);
+  h->peer_ipc.assign(n, 0);
+  h->peer_base[h->cfg.rank] = h->xbuf;
+  return EA_OK;
+}
+
+// Map every peer's exchange buffer through CUDA IPC (handles all-gathered over NCCL).
+ea_status p2p_ipc_connect(ea_ctx* h) {
+  const int n = h->cfg.n_pipelines, r = h->cfg.rank;
+  cudaIpcMemHandle_t mine;
+  cudaError_t e = cudaIpcGetMemHandle(&mine, h->xbuf);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaIpcGetMemHandle");
+  const size_t hb = sizeof(cudaIpcMemHandle_t);
+  char* dev = nullptr;
+  if ((e = cudaMalloc(&dev, hb * (n + 1))) != cudaSuccess) return cuda_fail(h, e, "handle exchange buffer");
+  std::vector<char> all(hb * n);
+  ea_status st = EA_OK;
+  cudaStream_t s = h->side;
+  if ((e = cudaMemcpyAsync(dev + hb * n, &mine, hb, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
+    st = cuda_fail(h, e, "handle upload");
+  } else {
+    ncclResult_t nr = ncclAllGather(dev + hb * n, dev, hb, ncclChar, h->comm, s);
+    if (nr != ncclSuccess) st = nccl_fail(h, nr, "IPC handle all-gather");
+    else if ((e = cudaMemcpyAsync(all.data(), dev, hb * n, cudaMemcpyDeviceToHost, s)) != cudaSuccess ||
+             (e = cudaStreamSynchronize(s)) != cudaSuccess)
+      st = cuda_fail(h, e, "handle download");
+  }
+  cudaFree(dev);
+  if (st != EA_OK) return st;
+  for (int q = 0; q < n; ++q) {
+    if (q == r) continue;
+    cudaIpcMemHandle_t hq;
+    std::memcpy(&hq, all.data() + hb * q, hb);
+    void* p = nullptr;
+    if ((e = cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess)) != cudaSuccess)
+      return cuda_fail(h, e, "cudaIpcOpenMemHandle (peer exchange buffer)");
+    h->peer_base[q] = static_cast<char*>(p);
+    h->peer_ipc[q] = 1;
+  }
+  h->same_device_ranks = 1;
+  h->p2p_ready = true;
+  return EA_OK;
+}
+
+// One stage of the fused peer-memory exchange, on the caller's stream.
+ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s) {
+  if (!h->p2p_ready) {
+    set_err(h, "peer-memory exchange not connected (needs an NCCL id at ea_init or ea_p2p_connect)");
+    return EA_ESTATE;
+  }
+  if (*h->err_host) {
+    set_err(h, "a previous peer-memory exchange timed out; the handle is unusable");
+    return EA_ECUDA;
+  }
+  const int n = h->cfg.n_pipelines;
+  ea::P2PView v;
+  for (int q = 0; q < ea::kMaxWorld; ++q) {
+    char* b = q < n ? h->peer_base[q] : nullptr;
+    v.inbox[q] = b ? reinterpret_cast<float*>(b + h->x_inbox[stage]) : nullptr;
+    v.outbox[q] = b ? reinterpret_cast<float*>(b + h->x_outbox[stage]) : nullptr;
+    v.arrive[q] = b ? reinterpret_cast<uint32_t*>(b + h->x_arrive[stage]) : nullptr;
+    v.ready[q] = b ? reinterpret_cast<uint32_t*>(b + h->x_ready[stage]) : nullptr;
+  }
+  ea::P2PArgs a;
+  a.x = replica;
+  a.g = grad;
+  a.m = state_ptr(h, 0, stage, 0);
+  a.v = state_ptr(h, 1, stage, 0);
+  a.center = center_ptr;
+  a.p = h->p[stage];
+  a.p_pad = h->p_pad[stage];
+  a.chunk = kP2PChunk;
+  a.nchunks = h->x_nchunks[stage];
+  a.slots = h->x_slots[stage];
+  a.rank = h->cfg.rank;
+  a.world = n;
+  a.sc = next_coef(h, stage);
+  a.epoch = static_cast<uint32_t>(h->steps[stage]);
+  a.hp = h->hp;
+  a.err = h->err_dev;
+  a.timeout_ns = p2p_timeout_ns();
+  // all ranks' kernels must be resident together: ranks sharing this device share its SMs
+  int max_ctas = h->num_sms * ea::p2p_blocks_per_sm() / h->same_device_ranks;
+  if (max_ctas < 1) max_ctas = 1;
+  cudaError_t e = ea::launch_spread_p2p(a, v, h->cfg.optimizer, max_ctas, s);
+  if (e != cudaSuccess) return cuda_fail(h, e, "peer-memory exchange kernel launch");
   return EA_OK;
 }
 
@@ -337,6 +480,11 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (c.rank < 0 || c.rank >= c.world) { set_err(nullptr, "rank %d out of [0,%d)", c.rank, c.world); return EA_EINVAL; }
   }
   if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
+  if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
+  if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {
+    set_err(nullptr, "peer-memory exchange supports world <= %d", ea::kMaxWorld);
+    return EA_EINVAL;
+  }
   ea_status st = check_hyper(nullptr, c);
   if (st != EA_OK) return st;
   int ndev = 0;
@@ -400,6 +548,16 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
         return r;
       }
     }
+    if (c.exchange == EA_XCHG_P2P) {
+      ea_status r = p2p_alloc(h);
+      if (r == EA_OK && c.world == 1) h->p2p_ready = true;
+      else if (r == EA_OK && h->comm) r = p2p_ipc_connect(h);
+      if (r != EA_OK) {
+        g_init_err = h->err;
+        free_ctx(h);
+        return r;
+      }
+    }
   }
   e = cudaDeviceSynchronize();
   if (e != cudaSuccess) { ea_status r = cuda_fail(nullptr, e, "init sync"); free_ctx(h); return r; }
@@ -422,7 +580,7 @@ ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const 
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   ea_status st = check_stage_ptrs(h, stage, replica_ptrs, grad_ptrs, center_ptr);
   if (st != EA_OK) return st;
-  if (h->cfg.layout == EA_SPREAD && !h->comm) {
+  if (h->cfg.layout == EA_SPREAD && h->cfg.exchange == EA_XCHG_NCCL && !h->comm) {
     set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
     return EA_ESTATE;
   }
@@ -449,7 +607,7 @@ ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float*
     if (st != EA_OK) return st;
   }
   if (count == 0) return EA_OK;
-  if (h->cfg.layout == EA_SPREAD && !h->comm) {
+  if (h->cfg.layout == EA_SPREAD && h->cfg.exchange == EA_XCHG_NCCL && !h->comm) {
     set_err(h, "EA_SPREAD handle created without an NCCL id: use ea_spread_local / ea_spread_apply");
     return EA_ESTATE;
   }
@@ -565,12 +723,50 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
   return EA_OK;
 }
 
+ea_status ea_p2p_connect(ea_handle h, const ea_handle* peers, int32_t world) {
+  if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
+  if (h->cfg.layout != EA_SPREAD || h->cfg.exchange != EA_XCHG_P2P) {
+    set_err(h, "ea_p2p_connect needs EA_SPREAD with exchange EA_XCHG_P2P");
+    return EA_ESTATE;
+  }
+  if (!peers || world != h->cfg.world) { set_err(h, "peers must list all %d ranks", h->cfg.world); return EA_EINVAL; }
+  int same = 0;
+  for (int q = 0; q < world; ++q) {
+    const ea_ctx* o = peers[q];
+    if (!o || o->cfg.rank != q || o->cfg.world != world || o->cfg.layout != EA_SPREAD ||
+        o->cfg.exchange != EA_XCHG_P2P || o->cfg.n_stages != h->cfg.n_stages || o->p != h->p || !o->xbuf) {
+      set_err(h, "peer %d is not a matching EA_SPREAD/EA_XCHG_P2P handle of rank %d", q, q);
+      return EA_EINVAL;
+    }
+    if (o->cfg.device == h->cfg.device) {
+      ++same;
+    } else {
+      int can = 0;
+      cudaDeviceCanAccessPeer(&can, h->cfg.device, o->cfg.device);
+      if (!can) { set_err(h, "device %d cannot access device %d", h->cfg.device, o->cfg.device); return EA_EINVAL; }
+      cudaSetDevice(h->cfg.device);
+      cudaError_t e = cudaDeviceEnablePeerAccess(o->cfg.device, 0);
+      if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_fail(h, e, "cudaDeviceEnablePeerAccess");
+      cudaGetLastError();
+    }
+  }
+  if (h != peers[h->cfg.rank]) { set_err(h, "peers[rank] must be this handle"); return EA_EINVAL; }
+  for (int q = 0; q < world; ++q) h->peer_base[q] = peers[q]->xbuf;
+  h->same_device_ranks = same;
+  h->p2p_ready = true;
+  return EA_OK;
+}
+
 ea_status ea_sync(ea_handle h, void* stream) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
   ea_status st = join_side(h, static_cast<cudaStream_t>(stream));
   if (st != EA_OK) return st;
+  if (h->err_host && *h->err_host) {
+    set_err(h, "peer-memory exchange timed out (a rank did not reach the same step)");
+    return EA_ECUDA;
+  }
   if (h->comm) {
     ncclResult_t async_err = ncclSuccess;
     ncclResult_t r = ncclCommGetAsyncError(h->comm, &async_err);

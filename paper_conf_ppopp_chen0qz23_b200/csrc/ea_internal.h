@@ -87,6 +87,37 @@ cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, co
                                 int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef& sc, int num_sms,
                                 cudaStream_t s);
 
+// ---- fused peer-memory spread step (ea_p2p.cu)
+constexpr int kMaxWorld = 16;
+
+// Addresses of every rank's exchange buffers for one stage, as seen from this GPU.
+struct P2PView {
+  float* inbox[kMaxWorld];     // rank o: [N][slots][chunk] contributions for the chunks o owns
+  float* outbox[kMaxWorld];    // rank o: [slots][chunk] updated center of the chunks o owns
+  uint32_t* arrive[kMaxWorld]; // rank o: [slots] cumulative arrival counters
+  uint32_t* ready[kMaxWorld];  // rank o: [slots] epoch at which the outbox chunk is final
+};
+
+struct P2PArgs {
+  float* x;            // this rank's replica (p floats)
+  const float* g;      // its gradient
+  float* m;            // optimizer state slot 0
+  float* v;            // optimizer state slot 1 (Adam) or null
+  float* center;       // this rank's copy of x~ (p_pad floats, zero padding)
+  int64_t p, p_pad;    // elements / padded elements
+  int64_t chunk;       // floats per chunk (multiple of 4)
+  int64_t nchunks, slots;
+  int rank, world;
+  uint32_t epoch;      // this stage's step count (>= 1)
+  Hyper hp;
+  StepCoef sc;
+  uint32_t* err;       // host-mapped error flag (timeouts)
+  uint64_t timeout_ns;
+};
+
+cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);
+int p2p_blocks_per_sm();
+
 // Spread shard epilogue (row a5): shard[k] += reduced[k] * inv_n for k < count.
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,
                                 cudaStream_t s);

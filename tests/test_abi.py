@@ -26,7 +26,7 @@ def lib():
 def header_functions():
     text = open(HEADER).read()
     text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
-    return sorted(set(re.findall(r"\b(ea_[a-z_]+)\s*\(", text)))
+    return sorted(set(re.findall(r"\b(ea_[a-z0-9_]+)\s*\(", text)))
 
 
 def test_header_lists_the_north_star_calls():
@@ -55,6 +55,7 @@ def test_config_struct_layout_matches_header():
     # ea_config: 2 x int32, pointer, 6 floats, 7 int32, [pad], 2 doubles, 1 float, [pad]  (x86-64 alignment)
     assert ctypes.sizeof(binding.EAConfig) == 96
     assert binding.EAConfig.beta1.offset == 72 and binding.EAConfig.eps.offset == 88
+    assert binding.EAConfig.exchange.offset == 92
     assert binding.EAConfig.stage_params.offset == 8
     assert ctypes.sizeof(binding.EAOp) == 8
 
@@ -63,7 +64,7 @@ def _cfg(**kw):
     sp = (ctypes.c_int64 * 2)(1000, 1001)
     base = dict(n_pipelines=2, n_stages=2, stage_params=sp, alpha=0.5, beta=0.0, rho=1.0, lr=0.05, momentum=0.9,
                 weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0, optimizer=0,
-                beta1=0.9, beta2=0.999, eps=1e-8)
+                beta1=0.9, beta2=0.999, eps=1e-8, exchange=0)
     base.update(kw)
     c = binding.EAConfig(**base)
     c._keep = sp
@@ -86,6 +87,8 @@ def _cfg(**kw):
     (dict(n_pipelines=65), "N must be"),
     (dict(lr=float("nan")), "finite"),
     (dict(optimizer=3), "optimizer"),
+    (dict(exchange=5), "exchange"),
+    (dict(layout=1, world=17, n_pipelines=17, rank=0, exchange=1), "world <="),
     (dict(optimizer=1, beta1=1.0), "betas"),
     (dict(optimizer=2, beta2=-0.5), "betas"),
     (dict(optimizer=1, eps=0.0), "eps"),
