@@ -381,7 +381,7 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
     set_err(h, "peer-memory exchange not connected (needs an NCCL id at ea_init or ea_p2p_connect)");
     return EA_ESTATE;
   }
-  if (*h->err_host) {
+  if (*reinterpret_cast<volatile uint32_t*>(h->err_host)) {
     set_err(h, "a previous peer-memory exchange timed out; the handle is unusable");
     return EA_ECUDA;
   }
@@ -763,7 +763,7 @@ ea_status ea_sync(ea_handle h, void* stream) {
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
   ea_status st = join_side(h, static_cast<cudaStream_t>(stream));
   if (st != EA_OK) return st;
-  if (h->err_host && *h->err_host) {
+  if (h->err_host && *reinterpret_cast<volatile uint32_t*>(h->err_host)) {
     set_err(h, "peer-memory exchange timed out (a rank did not reach the same step)");
     return EA_ECUDA;
   }
