@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
     ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw"), default="sgd",
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
+    ap.add_argument("--exchange", choices=("nccl", "p2p"), default="nccl",
+                    help="N>1 spread exchange: NCCL RS/AG or the fused peer-memory kernel")
     ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
@@ -166,7 +168,7 @@ def run_ours(args, rank, world, local):
         uid = parallel.broadcast_unique_id()
         h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
                              layout="spread", rank=rank, world=world, device=local, nccl_id=uid,
-                             optimizer=args.optimizer)
+                             optimizer=args.optimizer, exchange=args.exchange)
         state = []
         for s, p in enumerate(sizes):
             reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s)   # same center on every rank
@@ -234,6 +236,7 @@ def run_ours(args, rank, world, local):
     ws_bytes = (n * 3 + 1) * 4 * total_params if not spread else 5 * 4 * total_params
     out["config"] = {"workload": cfg.name, "n_pipelines": n, "n_stages": len(sizes), "params": total_params,
                      "stage_params": sizes, "layout": "spread" if spread else "colocated", "mode": MODE,
+                     "exchange": args.exchange if spread else None,
                      "optimizer": "sgd-momentum(0.9)" if args.optimizer == "sgd" else args.optimizer,
                      "kernel": args.variant,
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
