@@ -45,6 +45,7 @@ def parse():
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
     ap.add_argument("--exchange", choices=("nccl", "p2p"), default="nccl",
                     help="N>1 spread exchange: NCCL RS/AG or the fused peer-memory kernel")
+    ap.add_argument("--graph", action="store_true", help="capture one step in a CUDA graph and replay it")
     ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
@@ -206,6 +207,26 @@ def run_ours(args, rank, world, local):
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
+    if args.graph and not spread and args.optimizer == "sgd":
+        # the whole step as one CUDA graph (no per-step host work at all); SGD only:
+        # Adam's bias correction is a host-side per-step coefficient
+        graph = torch.cuda.CUDAGraph()
+        cap = torch.cuda.Stream()
+        cap.wait_stream(stream)
+        with torch.cuda.stream(cap):
+            with torch.cuda.graph(graph, stream=cap):
+                h.step_many(order, [state[s_][0] for s_ in order], [state[s_][1] for s_ in order],
+                            [state[s_][2] for s_ in order], stream=cap)
+        torch.cuda.synchronize()
+
+        def one_step(evs=None):  # noqa: F811
+            if evs is not None:
+                evs[0][0].record(stream)
+            graph.replay()
+            if evs is not None:
+                evs[0][1].record(stream)
+        one_step()
+        torch.cuda.synchronize()
     if spread:
         dist.barrier()
     # per-launch events for the dominant kernel (co-located: every ea_step is one kernel)
@@ -257,7 +278,8 @@ def run_ours(args, rank, world, local):
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * launches_per_step
-        out["config"]["launch"] = "ea_step_many (1 launch/step)" if batched else "ea_step per stage"
+        out["config"]["launch"] = ("CUDA graph replay of ea_step_many" if args.graph and args.optimizer == "sgd"
+                                   else "ea_step_many (1 launch/step)" if batched else "ea_step per stage")
     else:
         step_bytes = sum(bytes_spread_local(p, args.optimizer) for p in sizes)
         nv_bytes = sum(2 * (n - 1) / n * 4 * h.center_capacity(s) for s in range(len(sizes)))

@@ -409,3 +409,43 @@ def test_step_many_host_pipelined(optimizer, n):
     with pytest.raises(TypeError):
         h.step_many_host([0], [xs[0]], [[a.to(dev) for a in hg[0]]], [cs[0]], [host_out[0]])
     h.close()
+
+
+# ------------------------------------------------------------------ CUDA graphs
+def test_step_many_captured_in_a_cuda_graph():
+    """ea_step_many is stream-ordered work only, so a whole EA step can be
+    captured once and replayed (SGD: no per-step host state).  Replays must
+    equal the oracle run step by step."""
+    n, sizes, steps = 3, [100_003, 4096, 7], 6
+    hp = hyper(n, "combined")
+    dev = torch.device("cuda:0")
+    h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum)
+    oracle, gstreams, xs, cs, gb = [], [], [], [], []
+    for s, p in enumerate(sizes):
+        reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
+        oracle.append(OracleStage(reps, c))
+        gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
+        xs.append([torch.from_numpy(x).to(dev) for x in reps])
+        cs.append(torch.from_numpy(c).to(dev))
+        gb.append([torch.zeros(p, device=dev) for _ in range(n)])
+    order = list(reversed(range(len(sizes))))
+    graph = torch.cuda.CUDAGraph()
+    side = torch.cuda.Stream()
+    side.wait_stream(torch.cuda.current_stream())
+    with torch.cuda.stream(side):
+        with torch.cuda.graph(graph, stream=side):
+            h.step_many(order, [xs[s] for s in order], [gb[s] for s in order], [cs[s] for s in order], stream=side)
+    torch.cuda.synchronize()
+    for t in range(steps):
+        for s in range(len(sizes)):
+            g = gstreams[s].next()
+            for i in range(n):
+                gb[s][i].copy_(torch.from_numpy(g[i]))
+            oracle[s].step(g, hp)
+        graph.replay()
+    torch.cuda.synchronize()
+    for s in range(len(sizes)):
+        assert rel_err(to_np(cs[s]), oracle[s].c) <= TOL
+        for i in range(n):
+            assert rel_err(to_np(xs[s][i]), oracle[s].xs[i]) <= TOL
+    h.close()
