@@ -45,7 +45,8 @@ def parse():
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
     ap.add_argument("--exchange", choices=("nccl", "p2p"), default="nccl",
                     help="N>1 spread exchange: NCCL RS/AG or the fused peer-memory kernel")
-    ap.add_argument("--graph", action="store_true", help="capture one step in a CUDA graph and replay it")
+    ap.add_argument("--no-graph", action="store_true",
+                    help="launch ea_step_many every step instead of replaying one captured CUDA graph (SGD)")
     ap.add_argument("--per-stage", action="store_true", help="one ea_step launch per stage instead of ea_step_many")
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--no-e2e", action="store_true")
@@ -207,7 +208,8 @@ def run_ours(args, rank, world, local):
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
-    if args.graph and not spread and args.optimizer == "sgd":
+    use_graph = not args.no_graph and not spread and args.optimizer == "sgd" and batched
+    if use_graph:
         # the whole step as one CUDA graph (no per-step host work at all); SGD only:
         # Adam's bias correction is a host-side per-step coefficient
         graph = torch.cuda.CUDAGraph()
@@ -278,7 +280,7 @@ def run_ours(args, rank, world, local):
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * launches_per_step
-        out["config"]["launch"] = ("CUDA graph replay of ea_step_many" if args.graph and args.optimizer == "sgd"
+        out["config"]["launch"] = ("CUDA graph replay of ea_step_many (1 kernel/step)" if use_graph
                                    else "ea_step_many (1 launch/step)" if batched else "ea_step per stage")
     else:
         step_bytes = sum(bytes_spread_local(p, args.optimizer) for p in sizes)
