@@ -10,7 +10,7 @@ import numpy as np
 import pytest
 import torch
 
-from oracle.ea_oracle import Hyper, ea_step
+from oracle.ea_oracle import Hyper, ea_step, ea_step_adam
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
 from tests._parity import TOL, rel_err
@@ -24,12 +24,13 @@ def _sample_idx(p, k, rng):
     return torch.from_numpy(np.unique(np.r_[idx, edge]).astype(np.int64))
 
 
-def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000):
+def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000, optimizer="sgd"):
     dev = torch.device("cuda:0")
     a, b, r = synth.mode_coeffs(mode, n)
-    hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
-    h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM,
-                         kernel_variant=variant)
+    lr = synth.LR if optimizer == "sgd" else 1e-3
+    hp = Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM, weight_decay=0.0 if optimizer == "sgd" else 1e-2)
+    h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
+                         weight_decay=hp.weight_decay, kernel_variant=variant, optimizer=optimizer)
     gen = torch.Generator(device=dev)
     gen.manual_seed(7)
     rng = np.random.default_rng(0)
@@ -44,8 +45,9 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
         for s, (reps, c, grads, idx) in enumerate(state):
             for g in grads:
                 g.normal_(0.0, synth.GRAD_STD, generator=gen)
+            vs = [f64(h.state(s, i, 1), idx) for i in range(n)] if optimizer != "sgd" else None
             before.append(([f64(x, idx) for x in reps], [f64(h.momentum(s, i), idx) for i in range(n)],
-                           f64(c, idx), [f64(g, idx) for g in grads]))
+                           f64(c, idx), [f64(g, idx) for g in grads], vs))
         if many:
             h.step_many(order, [state[s][0] for s in order], [state[s][2] for s in order],
                         [state[s][1] for s in order])
@@ -54,8 +56,13 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
                 h.step(s, state[s][0], state[s][2], state[s][1])
         torch.cuda.synchronize()
         for s, (reps, c, grads, idx) in enumerate(state):
-            xs, ms, cc, gs = before[s]
-            ox, om, oc = ea_step(xs, ms, cc, gs, hp)
+            xs, ms, cc, gs, vs = before[s]
+            if optimizer == "sgd":
+                ox, om, oc = ea_step(xs, ms, cc, gs, hp)
+            else:
+                ox, om, ov, oc = ea_step_adam(xs, ms, vs, cc, gs, hp, t + 1, decoupled=optimizer == "adamw")
+                for i in range(n):
+                    assert rel_err(f64(h.state(s, i, 1), idx), ov[i]) <= TOL, (s, t, i)
             assert rel_err(f64(c, idx), oc) <= TOL, (s, t)
             for i in range(n):
                 assert rel_err(f64(reps[i], idx), ox[i]) <= TOL, (s, t, i)
@@ -67,6 +74,12 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
 def test_c2_full_size_sampled(variant):
     cfg = synth.CONFIGS["C2"]
     _run_sampled(cfg.n_pipelines, cfg.stage_sizes, 3, variant)
+
+
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+def test_c2_full_size_sampled_adam(optimizer):
+    cfg = synth.CONFIGS["C2"]
+    _run_sampled(cfg.n_pipelines, cfg.stage_sizes, 3, "auto", optimizer=optimizer)
 
 
 def test_c2_full_size_per_stage_launches():
