@@ -208,10 +208,10 @@ def run_ours(args, rank, world, local):
     for _ in range(args.warmup):
         one_step()
     torch.cuda.synchronize()
-    use_graph = not args.no_graph and not spread and args.optimizer == "sgd" and batched
+    use_graph = not args.no_graph and not spread and batched
     if use_graph:
-        # the whole step as one CUDA graph (no per-step host work at all); SGD only:
-        # Adam's bias correction is a host-side per-step coefficient
+        # the whole step as one CUDA graph (no per-step host work at all; Adam's step
+        # counter and bias corrections are advanced on the device inside the graph)
         graph = torch.cuda.CUDAGraph()
         cap = torch.cuda.Stream()
         cap.wait_stream(stream)

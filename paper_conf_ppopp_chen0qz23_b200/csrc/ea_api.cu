@@ -31,7 +31,9 @@ struct ea_ctx {
   std::vector<int64_t> p_pad;   // center capacity
   std::vector<int64_t> stride;  // optimizer-state row stride (floats)
   std::vector<float*> state[2]; // per stage: [replicas][stride]; slot 0 = momentum / Adam m, slot 1 = Adam v
-  std::vector<int64_t> steps;   // per-stage step count t (Adam bias correction)
+  std::vector<int64_t> steps;   // per-stage step count t, host shadow (enqueue order)
+  int64_t* d_steps = nullptr;   // device step counters (authoritative for Adam / P2P; graph-safe)
+  ea::StepCoef* d_coef = nullptr;  // device Adam bias corrections of the current step
   // EA_SPREAD
   cudaStream_t side = nullptr;
   cudaEvent_t ev_in = nullptr, ev_local = nullptr, ev_done = nullptr;
@@ -126,20 +128,10 @@ ea::Hyper make_hyper(const ea_config& c) {
 
 int state_slots(const ea_ctx* h) { return h->cfg.optimizer == EA_OPT_SGD ? 1 : 2; }
 
-// Advance the stage's step count and return the Adam bias corrections for it.
-ea::StepCoef next_coef(ea_ctx* h, int stage) {
-  const int64_t t = ++h->steps[stage];
-  ea::StepCoef sc;
-  if (h->cfg.optimizer == EA_OPT_SGD) {
-    sc.step_size = 0.f;
-    sc.inv_sqrt_bc2 = 0.f;
-    return sc;
-  }
-  const double bc1 = 1.0 - std::pow(h->cfg.beta1, (double)t);
-  const double bc2 = 1.0 - std::pow(h->cfg.beta2, (double)t);
-  sc.step_size = static_cast<float>((double)h->cfg.lr / bc1);
-  sc.inv_sqrt_bc2 = static_cast<float>(1.0 / std::sqrt(bc2));
-  return sc;
+// Device step counters are needed when a kernel consumes the step count:
+// Adam's bias correction and the peer-memory exchange's epoch.
+bool device_steps(const ea_ctx* h) {
+  return h->cfg.optimizer != EA_OPT_SGD || (h->cfg.layout == EA_SPREAD && h->cfg.exchange == EA_XCHG_P2P);
 }
 
 ea_status cuda_fail(ea_ctx* h, cudaError_t e, const char* what) {
@@ -152,6 +144,21 @@ ea_status nccl_fail(ea_ctx* h, ncclResult_t r, const char* what) {
   return EA_ENCCL;
 }
 
+// Count one step of each listed stage: host shadow now, device counters (and
+// Adam coefficients) on `s` ahead of the step's kernel.
+ea_status advance(ea_ctx* h, const int32_t* stages, int count, cudaStream_t s) {
+  for (int j = 0; j < count; ++j) ++h->steps[stages[j]];
+  if (!device_steps(h)) return EA_OK;
+  for (int j0 = 0; j0 < count; j0 += 8) {
+    ea::StageList l;
+    l.count = 0;
+    for (int j = j0; j < count && j < j0 + 8; ++j) l.idx[l.count++] = stages[j];
+    cudaError_t e = ea::launch_advance_steps(h->d_steps, h->d_coef, l, h->cfg.beta1, h->cfg.beta2, (double)h->cfg.lr, s);
+    if (e != cudaSuccess) return cuda_fail(h, e, "step-counter kernel launch");
+  }
+  return EA_OK;
+}
+
 void free_ctx(ea_ctx* h) {
   if (!h) return;
   cudaSetDevice(h->cfg.device);
@@ -161,6 +168,8 @@ void free_ctx(ea_ctx* h) {
     for (float* m : slot) if (m) cudaFree(m);
   if (h->contrib) cudaFree(h->contrib);
   if (h->reduced) cudaFree(h->reduced);
+  if (h->d_steps) cudaFree(h->d_steps);
+  if (h->d_coef) cudaFree(h->d_coef);
   if (h->ev_in) cudaEventDestroy(h->ev_in);
   if (h->ev_local) cudaEventDestroy(h->ev_local);
   if (h->ev_done) cudaEventDestroy(h->ev_done);
@@ -228,13 +237,17 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
         t.m[i] = state_ptr(h, 0, st, i);
         t.v[i] = two ? state_ptr(h, 1, st, i) : nullptr;
       }
-      const ea::StepCoef sc = next_coef(h, st);
-      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, opt, sc, h->num_sms, s);
+      ea_status st2 = advance(h, &stages[j], 1, s);
+      if (st2 != EA_OK) return st2;
+      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, opt, h->d_coef + st, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
     }
     return EA_OK;
   }
   for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
+    const int cnt = count - j0 < ea::kMaxLaunchStages ? count - j0 : ea::kMaxLaunchStages;
+    ea_status st2 = advance(h, stages + j0, cnt, s);
+    if (st2 != EA_OK) return st2;
     ea::StageBatch b;
     b.nstages = 0;
     for (int j = j0; j < count && j < j0 + ea::kMaxLaunchStages; ++j) {
@@ -249,7 +262,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
       }
       r.c = center_ptrs[j];
       r.p = h->p[st];
-      r.sc = next_coef(h, st);
+      r.scp = h->d_coef + st;
     }
     e = ea::launch_colocated_batch(b, n, h->hp, opt, h->variant, h->num_sms, s);
     if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
@@ -272,9 +285,11 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
   float* own = center_ptr + shard * h->cfg.rank;
   if ((e = cudaEventRecord(h->ev_in, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   if ((e = cudaStreamWaitEvent(h->side, h->ev_in, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  const ea::StepCoef sc = next_coef(h, stage);
+  ea_status st2 = advance(h, &stage, 1, h->side);
+  if (st2 != EA_OK) return st2;
   e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr,
-                              h->contrib, h->p[stage], pad, h->hp, h->cfg.optimizer, sc, h->num_sms, h->side);
+                              h->contrib, h->p[stage], pad, h->hp, h->cfg.optimizer, h->d_coef + stage, h->num_sms,
+                              h->side);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
   if ((e = cudaEventRecord(h->ev_local, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   ncclResult_t r = ncclReduceScatter(h->contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
@@ -407,8 +422,10 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   a.slots = h->x_slots[stage];
   a.rank = h->cfg.rank;
   a.world = n;
-  a.sc = next_coef(h, stage);
-  a.epoch = static_cast<uint32_t>(h->steps[stage]);
+  ea_status st2 = advance(h, &stage, 1, s);
+  if (st2 != EA_OK) return st2;
+  a.stepp = h->d_steps + stage;
+  a.scp = h->d_coef + stage;
   a.hp = h->hp;
   a.err = h->err_dev;
   a.timeout_ns = p2p_timeout_ns();
@@ -503,6 +520,14 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   e = cudaSetDevice(c.device);
   if (e != cudaSuccess) { ea_status r = cuda_fail(nullptr, e, "cudaSetDevice"); free_ctx(h); return r; }
   cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, c.device);
+  if ((e = cudaMalloc(&h->d_steps, sizeof(int64_t) * c.n_stages)) != cudaSuccess ||
+      (e = cudaMemset(h->d_steps, 0, sizeof(int64_t) * c.n_stages)) != cudaSuccess ||
+      (e = cudaMalloc(&h->d_coef, sizeof(ea::StepCoef) * c.n_stages)) != cudaSuccess ||
+      (e = cudaMemset(h->d_coef, 0, sizeof(ea::StepCoef) * c.n_stages)) != cudaSuccess) {
+    ea_status r = cuda_fail(nullptr, e, "step counters");
+    free_ctx(h);
+    return r;
+  }
 
   const int reps = replicas_here(h);
   int64_t max_pad = 0;
@@ -666,7 +691,9 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
   int64_t k = 0;  // chunk counter (staging buffer k % 2)
   for (int j = 0; j < count; ++j) {
     const int st = stages[j];
-    const ea::StepCoef sc = next_coef(h, st);
+    ea_status st2 = advance(h, &stages[j], 1, s);
+    if (st2 != EA_OK) return st2;
+    const ea::StepCoef* sc = h->d_coef + st;
     const int64_t ps = h->p[st];
     for (int64_t off = 0; off < ps; off += kHostChunk, ++k) {
       const int64_t len = ps - off < kHostChunk ? ps - off : kHostChunk;
@@ -705,7 +732,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
         }
         r.c = center_ptrs[j] + off;
         r.p = len;
-        r.sc = sc;
+        r.scp = sc;
         e = ea::launch_colocated_batch(bt, n, h->hp, opt, h->variant, h->num_sms, s);
       }
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
@@ -792,10 +819,11 @@ ea_status ea_spread_local(ea_handle h, int32_t stage, float* replica_ptr, const 
     }
   cudaError_t e = cudaSetDevice(dev);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
-  const ea::StepCoef sc = next_coef(h, stage);
+  ea_status st2 = advance(h, &stage, 1, static_cast<cudaStream_t>(stream));
+  if (st2 != EA_OK) return st2;
   e = ea::launch_spread_local(replica_ptr, grad_ptr, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr,
-                              contrib, h->p[stage], h->p_pad[stage], h->hp, h->cfg.optimizer, sc, h->num_sms,
-                              static_cast<cudaStream_t>(stream));
+                              contrib, h->p[stage], h->p_pad[stage], h->hp, h->cfg.optimizer, h->d_coef + stage,
+                              h->num_sms, static_cast<cudaStream_t>(stream));
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
   return EA_OK;
 }
@@ -850,7 +878,14 @@ ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot
 ea_status ea_get_step(ea_handle h, int32_t stage, int64_t* step) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   if (stage < 0 || stage >= h->cfg.n_stages || !step) { set_err(h, "bad stage or NULL out pointer"); return EA_EINVAL; }
-  *step = h->steps[stage];
+  if (!device_steps(h)) {
+    *step = h->steps[stage];
+    return EA_OK;
+  }
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(step, h->d_steps + stage, sizeof(int64_t), cudaMemcpyDeviceToHost);
+  if (e != cudaSuccess) return cuda_fail(h, e, "reading the step counter");
   return EA_OK;
 }
 
@@ -858,6 +893,10 @@ ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   if (stage < 0 || stage >= h->cfg.n_stages || step < 0) { set_err(h, "bad stage or negative step"); return EA_EINVAL; }
   h->steps[stage] = step;
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  if (e == cudaSuccess) e = cudaMemcpy(h->d_steps + stage, &step, sizeof(int64_t), cudaMemcpyHostToDevice);
+  if (e != cudaSuccess) return cuda_fail(h, e, "writing the step counter");
   return EA_OK;
 }
 

@@ -26,11 +26,24 @@ struct Hyper {
   float lr_wd;     // lr * wd (AdamW decoupled decay)
 };
 
-// Per-stage, per-call Adam bias corrections (t = this stage's step count).
+// Per-stage Adam bias corrections for the step being taken (t = the stage's
+// step count).  They live in device memory, written by advance_steps() on the
+// stream right before the step's kernel, so a captured CUDA graph advances t
+// on every replay.
 struct StepCoef {
   float step_size;     // lr / (1 - beta1^t)
   float inv_sqrt_bc2;  // 1 / sqrt(1 - beta2^t)
 };
+
+// Stage list of one advance_steps launch.
+struct StageList {
+  int idx[8];
+  int count;
+};
+
+// On `s`: for every listed stage, ++steps[stage] and recompute coef[stage] (double precision).
+cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, double beta1, double beta2,
+                                 double lr, cudaStream_t s);
 
 constexpr int kMaxReplicas = 64;      // EA_MAX_REPLICAS
 constexpr int kMaxFusedN = 8;         // replicas handled by the compile-time-N kernels
@@ -44,7 +57,7 @@ struct StageRefs {
   float* v[kMaxFusedN];  // Adam second moment (unused by SGD)
   float* c;
   int64_t p;             // elements
-  StepCoef sc;
+  const StepCoef* scp;   // device: this stage's Adam coefficients (unused by SGD)
 };
 
 // Up to kMaxLaunchStages stages updated by ONE launch (same N).
@@ -78,13 +91,13 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
 
 // Co-located step for one stage with any N <= kMaxReplicas (N > 8 path).
 cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
-                                  const StepCoef& sc, int num_sms, cudaStream_t s);
+                                  const StepCoef* scp, int num_sms, cudaStream_t s);
 
 // Spread local step (rows a1-a4 for one replica): updates x and the optimizer
 // state in place and writes r = rho*Delta + beta*(x - x~) into contrib[0..p),
 // zeros into contrib[p..p_pad).
 cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
-                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef& sc, int num_sms,
+                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef* scp, int num_sms,
                                 cudaStream_t s);
 
 // ---- fused peer-memory spread step (ea_p2p.cu)
@@ -108,9 +121,9 @@ struct P2PArgs {
   int64_t chunk;       // floats per chunk (multiple of 4)
   int64_t nchunks, slots;
   int rank, world;
-  uint32_t epoch;      // this stage's step count (>= 1)
+  const int64_t* stepp;  // device: this stage's step count (>= 1), the exchange epoch
   Hyper hp;
-  StepCoef sc;
+  const StepCoef* scp;   // device: Adam coefficients
   uint32_t* err;       // host-mapped error flag (timeouts)
   uint64_t timeout_ns;
 };

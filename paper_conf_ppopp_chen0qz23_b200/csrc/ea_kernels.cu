@@ -120,16 +120,26 @@ __device__ __forceinline__ float4 center_apply(float4 c, float4 acc, float inv_n
                      fmaf(acc.w, inv_n, c.w));
 }
 
+template <int OPT>
+__device__ __forceinline__ StepCoef load_coef(const StepCoef* scp) {
+  if constexpr (OPT == kOptSGD) {
+    return StepCoef{0.f, 0.f};
+  } else {
+    return *scp;
+  }
+}
+
 // Scalar tail of one stage: elements [4*(p/4), p) (fewer than 4), one thread.
 template <int N, int OPT>
 __device__ void stage_tail(const StageRefs& st, const Hyper& hp) {
+  const StepCoef sc = load_coef<OPT>(st.scp);
   for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
     const float c = st.c[j];
     float acc = 0.f;
 #pragma unroll
     for (int i = 0; i < N; ++i) {
       float x = st.x[i][j], m = st.m[i][j], v = OPT == kOptSGD ? 0.f : st.v[i][j];
-      acc += ea_elem<OPT>(x, st.g[i][j], m, v, c, hp, st.sc);
+      acc += ea_elem<OPT>(x, st.g[i][j], m, v, c, hp, sc);
       st.x[i][j] = x;
       st.m[i][j] = m;
       if (OPT != kOptSGD) st.v[i][j] = v;
@@ -227,7 +237,7 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
 #pragma unroll
       for (int i = 0; i < N; ++i) {
         float4 unused;
-        add4(acc, ea_vec<kOptSGD>(x[i][u], g[i][u], m[i][u], unused, c[u], hp, st.sc));
+        add4(acc, ea_vec<kOptSGD>(x[i][u], g[i][u], m[i][u], unused, c[u], hp, StepCoef{0.f, 0.f}));
         mem.st(st.x[i] + 4 * v, x[i][u]);
         mem.st(st.m[i] + 4 * v, m[i][u]);
       }
@@ -251,8 +261,9 @@ __global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b
 template <int U, int OPT>
 __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t, int n, float* __restrict__ center,
                                                            int64_t nvec, int64_t p, const Hyper hp,
-                                                           const StepCoef sc) {
+                                                           const StepCoef* scp) {
   const Mem<0> mem;
+  const StepCoef sc = load_coef<OPT>(scp);
   WaveCursor cur{0, 0};
   int sidx;
   int64_t va, nv;
@@ -418,6 +429,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       issue(s_next, v0_next, nv_next, buf ^ 1);
     }
     const StageRefs& st = b.st[s];
+    const StepCoef sc = load_coef<OPT>(st.scp);
     float* xi = nullptr;
     const float* gi = nullptr;
     float* mi = nullptr;
@@ -453,7 +465,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       const float4 c = in ? s_center[buf][lv] : make_float4(0.f, 0.f, 0.f, 0.f);
       float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
       if (active && in) {
-        r = ea_vec<OPT>(x[k], g[k], m[k], w[k], c, hp, st.sc);
+        r = ea_vec<OPT>(x[k], g[k], m[k], w[k], c, hp, sc);
         const int64_t v = v0 + lv;
         mem.st(xi + 4 * v, x[k]);
         mem.st(mi + 4 * v, m[k]);
@@ -565,7 +577,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
           const float4 g = base[(2 + 3 * i) * T + lv];
           float4 m = base[(3 + 3 * i) * T + lv];
           float4 unused;
-          add4(acc, ea_vec<kOptSGD>(x, g, m, unused, c, hp, st.sc));
+          add4(acc, ea_vec<kOptSGD>(x, g, m, unused, c, hp, StepCoef{0.f, 0.f}));
           mem.st(st.x[i] + 4 * v, x);
           mem.st(st.m[i] + 4 * v, m);
         }
@@ -588,8 +600,9 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
                                                          float* __restrict__ m, float* __restrict__ vs,
                                                          const float* __restrict__ center,
                                                          float* __restrict__ contrib, int64_t nvec, int64_t p,
-                                                         int64_t p_pad, const Hyper hp, const StepCoef sc) {
+                                                         int64_t p_pad, const Hyper hp, const StepCoef* scp) {
   const Mem<0> mem;
+  const StepCoef sc = load_coef<OPT>(scp);
   WaveCursor cur{0, 0};
   int sidx;
   int64_t va, nv;
@@ -779,7 +792,7 @@ cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant,
 
 template <int OPT>
 cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
-                            const StepCoef& sc, int num_sms, cudaStream_t s) {
+                            const StepCoef* sc, int num_sms, cudaStream_t s) {
   constexpr int U = 2;
   const int64_t nvec = p / 4;
   auto k = colocated_wide<U, OPT>;
@@ -790,7 +803,7 @@ cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, int64_t
 
 template <int OPT>
 cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
-                                    float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef& sc,
+                                    float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
   constexpr int U = OPT == kOptSGD ? 4 : 2;
   const int64_t nvec = p / 4;
@@ -801,7 +814,27 @@ cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v
   return cudaGetLastError();
 }
 
+// Step counter + Adam bias corrections, on the stream (graph-capturable).
+__global__ void advance_steps(int64_t* steps, StepCoef* coef, const StageList list, double beta1, double beta2,
+                              double lr) {
+  const int i = threadIdx.x;
+  if (i >= list.count) return;
+  const int s = list.idx[i];
+  const int64_t t = ++steps[s];
+  const double bc1 = 1.0 - pow(beta1, (double)t);
+  const double bc2 = 1.0 - pow(beta2, (double)t);
+  coef[s].step_size = bc1 > 0.0 ? static_cast<float>(lr / bc1) : 0.f;
+  coef[s].inv_sqrt_bc2 = bc2 > 0.0 ? static_cast<float>(1.0 / sqrt(bc2)) : 0.f;
+}
+
 }  // namespace
+
+cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, double beta1, double beta2,
+                                 double lr, cudaStream_t s) {
+  if (list.count <= 0) return cudaSuccess;
+  advance_steps<<<1, 32, 0, s>>>(steps, coef, list, beta1, beta2, lr);
+  return cudaGetLastError();
+}
 
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
@@ -820,7 +853,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
 }
 
 cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
-                                  const StepCoef& sc, int num_sms, cudaStream_t s) {
+                                  const StepCoef* sc, int num_sms, cudaStream_t s) {
   if (p <= 0) return cudaSuccess;
   if (opt == kOptAdam) return launch_wide_opt<kOptAdam>(t, n, center, p, hp, sc, num_sms, s);
   if (opt == kOptAdamW) return launch_wide_opt<kOptAdamW>(t, n, center, p, hp, sc, num_sms, s);
@@ -828,7 +861,7 @@ cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, i
 }
 
 cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
-                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef& sc, int num_sms,
+                                int64_t p, int64_t p_pad, const Hyper& hp, int opt, const StepCoef* sc, int num_sms,
                                 cudaStream_t s) {
   if (p_pad <= 0) return cudaSuccess;
   if (opt == kOptAdam)

@@ -103,6 +103,8 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
   const int64_t Q = a.chunk, nch = a.nchunks, slots = a.slots;
   const int N = a.world, r = a.rank;
   const float inv_n = a.hp.inv_n;
+  const uint32_t epoch = static_cast<uint32_t>(*a.stepp);
+  const StepCoef sc = OPT == kOptSGD ? StepCoef{0.f, 0.f} : *a.scp;
 
   // ---------------- Phase A: local update, push contributions to the owners
   for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
@@ -117,10 +119,10 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
       if (j + 3 < a.p) {
         float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
         float4 w = OPT == kOptSGD ? make_float4(0.f, 0.f, 0.f, 0.f) : ld4(a.v + j);
-        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, a.sc);
-        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, a.sc);
-        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, a.sc);
-        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, a.sc);
+        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
+        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
+        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
+        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
         st4(a.x + j, x);
         st4(a.m + j, m);
         if (OPT != kOptSGD) st4(a.v + j, w);
@@ -131,7 +133,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
           rr[q] = 0.f;
           if (jj < a.p) {
             float x = a.x[jj], m = a.m[jj], w = OPT == kOptSGD ? 0.f : a.v[jj];
-            rr[q] = p2p_elem<OPT>(x, a.g[jj], m, w, a.center[jj], a.hp, a.sc);
+            rr[q] = p2p_elem<OPT>(x, a.g[jj], m, w, a.center[jj], a.hp, sc);
             a.x[jj] = x;
             a.m[jj] = m;
             if (OPT != kOptSGD) a.v[jj] = w;
@@ -155,7 +157,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     if (c >= nch) continue;
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    if (tid == 0) s_ok = wait_at_least(view.arrive[r] + slot, (uint32_t)N * a.epoch, a.timeout_ns, a.err);
+    if (tid == 0) s_ok = wait_at_least(view.arrive[r] + slot, (uint32_t)N * epoch, a.timeout_ns, a.err);
     __syncthreads();
     const float* in = view.inbox[r] + slot * Q;
     float* out = view.outbox[r] + slot * Q;
@@ -174,7 +176,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     __syncthreads();
     if (tid == 0) {
       __threadfence_system();
-      st_release_sys(view.ready[r] + slot, a.epoch);
+      st_release_sys(view.ready[r] + slot, epoch);
     }
     (void)s_ok;
   }
@@ -186,7 +188,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     const int64_t slot = c / N;
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    if (tid == 0) s_ok = wait_at_least(view.ready[o] + slot, a.epoch, a.timeout_ns, a.err);
+    if (tid == 0) s_ok = wait_at_least(view.ready[o] + slot, epoch, a.timeout_ns, a.err);
     __syncthreads();
     const float* src = view.outbox[o] + slot * Q;
     for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) st4(a.center + e0 + 4 * lv, ld_cg(src + 4 * lv));

@@ -412,18 +412,22 @@ def test_step_many_host_pipelined(optimizer, n):
 
 
 # ------------------------------------------------------------------ CUDA graphs
-def test_step_many_captured_in_a_cuda_graph():
-    """ea_step_many is stream-ordered work only, so a whole EA step can be
-    captured once and replayed (SGD: no per-step host state).  Replays must
-    equal the oracle run step by step."""
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw"])
+def test_step_many_captured_in_a_cuda_graph(optimizer):
+    """ea_step_many is stream-ordered work only -- including Adam's step
+    counter and bias corrections, which live on the device -- so a whole EA
+    step can be captured once and replayed.  Replays must equal the oracle run
+    step by step, and the step counter must count replays."""
     n, sizes, steps = 3, [100_003, 4096, 7], 6
-    hp = hyper(n, "combined")
+    lr = synth.LR if optimizer == "sgd" else 1e-3
+    hp = hyper(n, "combined", lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
-    h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum)
+    h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                         weight_decay=hp.weight_decay, optimizer=optimizer)
     oracle, gstreams, xs, cs, gb = [], [], [], [], []
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
-        oracle.append(OracleStage(reps, c))
+        oracle.append(OracleStage(reps, c, optimizer))
         gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
         xs.append([torch.from_numpy(x).to(dev) for x in reps])
         cs.append(torch.from_numpy(c).to(dev))
@@ -448,4 +452,8 @@ def test_step_many_captured_in_a_cuda_graph():
         assert rel_err(to_np(cs[s]), oracle[s].c) <= TOL
         for i in range(n):
             assert rel_err(to_np(xs[s][i]), oracle[s].xs[i]) <= TOL
+            if optimizer != "sgd":
+                assert rel_err(to_np(h.state(s, i, 1)), oracle[s].vs[i]) <= TOL
+        if optimizer != "sgd":
+            assert h.get_step(s) == steps          # device counter: replays, not the one capture
     h.close()
