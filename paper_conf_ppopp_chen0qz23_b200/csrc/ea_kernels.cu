@@ -401,11 +401,13 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
   const int rep = lane / CH, chunk = lane % CH;
   const bool active = rep < N;
 
+  __shared__ StepCoef s_coef[kMaxLaunchStages];  // Adam coefficients of the batch's stages, loaded once
   if (threadIdx.x == 0) {
     mbar_init(&s_bar[0], 1);
     mbar_init(&s_bar[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if (kTwoState && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
   __syncthreads();
 
   auto issue = [&](int s, int64_t v0, int64_t nv, int buf) {
@@ -429,7 +431,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       issue(s_next, v0_next, nv_next, buf ^ 1);
     }
     const StageRefs& st = b.st[s];
-    const StepCoef sc = load_coef<OPT>(st.scp);
+    const StepCoef sc = kTwoState ? s_coef[s] : StepCoef{0.f, 0.f};
     float* xi = nullptr;
     const float* gi = nullptr;
     float* mi = nullptr;

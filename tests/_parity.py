@@ -32,11 +32,22 @@ def to_np(t) -> np.ndarray:
     return t.detach().cpu().numpy()
 
 
+def f32(v: float) -> float:
+    """The value a float32 field of ea_config actually carries."""
+    return float(np.float32(v))
+
+
 def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nesterov=False, betas=(0.9, 0.999),
           eps=1e-8):
+    """Oracle hyper-parameters equal to what the ABI carries (reading c12: the
+    oracle consumes the same fp32 values upcast): alpha, beta, rho, lr,
+    momentum, weight_decay, eps are float32 fields; beta1/beta2 are double.
+    (Adam's Delta = -lr m/(sqrt(v)+eps) has slope ~lr/eps where the gradient
+    is near 0, so the 2e-10 relative gap between 0.01 and float32(0.01) alone
+    moves such an element by ~1e-5 of rms(x).)"""
     a, b, r = synth.mode_coeffs(mode, n, alpha)
-    return Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=momentum, weight_decay=wd, nesterov=nesterov,
-                 beta1=betas[0], beta2=betas[1], eps=eps)
+    return Hyper(alpha=f32(a), beta=f32(b), rho=f32(r), lr=f32(lr), momentum=f32(momentum), weight_decay=f32(wd),
+                 nesterov=nesterov, beta1=betas[0], beta2=betas[1], eps=f32(eps))
 
 
 class OracleStage:

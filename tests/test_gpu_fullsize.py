@@ -13,7 +13,7 @@ import torch
 from oracle.ea_oracle import Hyper, ea_step, ea_step_adam
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
-from tests._parity import TOL, rel_err
+from tests._parity import TOL, hyper, rel_err
 
 pytestmark = pytest.mark.gpu
 
@@ -28,9 +28,9 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
     dev = torch.device("cuda:0")
     a, b, r = synth.mode_coeffs(mode, n)
     lr = synth.LR if optimizer == "sgd" else 1e-3
-    hp = Hyper(alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM, weight_decay=0.0 if optimizer == "sgd" else 1e-2)
+    hp = hyper(n, mode, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
     h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
-                         weight_decay=hp.weight_decay, kernel_variant=variant, optimizer=optimizer)
+                         weight_decay=0.0 if optimizer == "sgd" else 1e-2, kernel_variant=variant, optimizer=optimizer)
     gen = torch.Generator(device=dev)
     gen.manual_seed(7)
     rng = np.random.default_rng(0)
