@@ -764,7 +764,7 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
       default: break;
     }
   }
-  return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 1>(b, hp, num_sms, s);
+  return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 2>(b, hp, num_sms, s);  // <= 128 regs: 2 CTAs/SM
 }
 
 template <int N, int HINT>
