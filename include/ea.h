@@ -67,6 +67,7 @@ extern "C" {
 #define EA_ABI_VERSION 2
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
+#define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
 
 typedef enum {
   EA_OK = 0,
@@ -208,6 +209,14 @@ EA_API ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* st
  * another, so each rank must drive its own stream; ranks that share a device
  * split its SMs.  EA_ESTATE for other layouts/exchanges. */
 EA_API ea_status ea_p2p_connect(ea_handle h, const ea_handle* peers, int32_t world);
+
+/* EA_XCHG_P2P between processes without an NCCL id (the caller moves the
+ * handles, e.g. over a torch process group): ea_p2p_export writes this rank's
+ * exchange-buffer IPC handle (EA_IPC_HANDLE_BYTES); ea_p2p_open takes all
+ * ranks' handles (world x EA_IPC_HANDLE_BYTES, rank-major) and maps the peers
+ * (cudaIpcOpenMemHandle).  Ranks created with an NCCL id do this inside ea_init. */
+EA_API ea_status ea_p2p_export(ea_handle h, uint8_t* handle);
+EA_API ea_status ea_p2p_open(ea_handle h, const uint8_t* handles, int32_t world);
 
 /* Make `stream` wait until every center update enqueued so far is complete,
  * then report any asynchronous CUDA/NCCL error seen so far.  Does not block

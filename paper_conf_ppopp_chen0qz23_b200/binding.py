@@ -122,6 +122,8 @@ SIGNATURES = {
     "ea_step_many_host": (ctypes.c_int, [_VP, ctypes.c_int32, ctypes.POINTER(ctypes.c_int32), _FPP, _FPP, _FPP,
                                          _FPP, _VP]),
     "ea_p2p_connect": (ctypes.c_int, [_VP, ctypes.POINTER(_VP), ctypes.c_int32]),
+    "ea_p2p_export": (ctypes.c_int, [_VP, ctypes.c_void_p]),
+    "ea_p2p_open": (ctypes.c_int, [_VP, ctypes.c_void_p, ctypes.c_int32]),
     "ea_sync": (ctypes.c_int, [_VP, _VP]),
     "ea_spread_local": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP, _VP, _VP]),
     "ea_spread_apply": (ctypes.c_int, [_VP, ctypes.c_int32, _VP, _VP, _VP]),
@@ -372,6 +374,20 @@ class ElasticAveraging:
         arr = (ctypes.c_void_p * len(handles))(*[h._h.value for h in handles])
         for h in handles:
             _check(lib.ea_p2p_connect(h._h, arr, len(handles)), h._h)
+
+    def p2p_export(self) -> bytes:
+        """This rank's exchange-buffer CUDA IPC handle (64 bytes)."""
+        buf = (ctypes.c_uint8 * 64)()
+        _check(self._lib.ea_p2p_export(self._h, buf), self._h)
+        return bytes(buf)
+
+    def p2p_open(self, handles):
+        """Map every rank's exchange buffer from the list of all ranks' handles."""
+        blob = b"".join(handles)
+        if len(blob) != 64 * self.world:
+            raise ValueError("need world x 64-byte handles")
+        buf = (ctypes.c_uint8 * len(blob)).from_buffer_copy(blob)
+        _check(self._lib.ea_p2p_open(self._h, buf, self.world), self._h)
 
     def sync(self, stream=None):
         _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)

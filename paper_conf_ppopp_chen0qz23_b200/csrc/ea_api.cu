@@ -353,15 +353,36 @@ ea_status p2p_alloc(ea_ctx* h) {
 }
 
 // Map every peer's exchange buffer through CUDA IPC (handles all-gathered over NCCL).
-ea_status p2p_ipc_connect(ea_ctx* h) {
+// Open every peer's exchange buffer from the all-gathered IPC handles
+// (world x EA_IPC_HANDLE_BYTES, rank-major).
+ea_status p2p_open_handles(ea_ctx* h, const uint8_t* all) {
   const int n = h->cfg.n_pipelines, r = h->cfg.rank;
+  const size_t hb = sizeof(cudaIpcMemHandle_t);
+  for (int q = 0; q < n; ++q) {
+    if (q == r) continue;
+    cudaIpcMemHandle_t hq;
+    std::memcpy(&hq, all + hb * q, hb);
+    void* p = nullptr;
+    cudaError_t e = cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess);
+    if (e != cudaSuccess) return cuda_fail(h, e, "cudaIpcOpenMemHandle (peer exchange buffer)");
+    h->peer_base[q] = static_cast<char*>(p);
+    h->peer_ipc[q] = 1;
+  }
+  h->same_device_ranks = 1;
+  h->p2p_ready = true;
+  return EA_OK;
+}
+
+// Map every peer's exchange buffer through CUDA IPC (handles all-gathered over NCCL).
+ea_status p2p_ipc_connect(ea_ctx* h) {
+  const int n = h->cfg.n_pipelines;
   cudaIpcMemHandle_t mine;
   cudaError_t e = cudaIpcGetMemHandle(&mine, h->xbuf);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaIpcGetMemHandle");
   const size_t hb = sizeof(cudaIpcMemHandle_t);
   char* dev = nullptr;
   if ((e = cudaMalloc(&dev, hb * (n + 1))) != cudaSuccess) return cuda_fail(h, e, "handle exchange buffer");
-  std::vector<char> all(hb * n);
+  std::vector<uint8_t> all(hb * n);
   ea_status st = EA_OK;
   cudaStream_t s = h->side;
   if ((e = cudaMemcpyAsync(dev + hb * n, &mine, hb, cudaMemcpyHostToDevice, s)) != cudaSuccess) {
@@ -375,19 +396,7 @@ ea_status p2p_ipc_connect(ea_ctx* h) {
   }
   cudaFree(dev);
   if (st != EA_OK) return st;
-  for (int q = 0; q < n; ++q) {
-    if (q == r) continue;
-    cudaIpcMemHandle_t hq;
-    std::memcpy(&hq, all.data() + hb * q, hb);
-    void* p = nullptr;
-    if ((e = cudaIpcOpenMemHandle(&p, hq, cudaIpcMemLazyEnablePeerAccess)) != cudaSuccess)
-      return cuda_fail(h, e, "cudaIpcOpenMemHandle (peer exchange buffer)");
-    h->peer_base[q] = static_cast<char*>(p);
-    h->peer_ipc[q] = 1;
-  }
-  h->same_device_ranks = 1;
-  h->p2p_ready = true;
-  return EA_OK;
+  return p2p_open_handles(h, all.data());
 }
 
 // One stage of the fused peer-memory exchange, on the caller's stream.
@@ -782,6 +791,32 @@ ea_status ea_p2p_connect(ea_handle h, const ea_handle* peers, int32_t world) {
   h->same_device_ranks = same;
   h->p2p_ready = true;
   return EA_OK;
+}
+
+ea_status ea_p2p_export(ea_handle h, uint8_t* handle) {
+  if (!h || !handle) { set_err(h, "NULL handle or output"); return EA_EINVAL; }
+  if (h->cfg.layout != EA_SPREAD || h->cfg.exchange != EA_XCHG_P2P || !h->xbuf) {
+    set_err(h, "ea_p2p_export needs EA_SPREAD with exchange EA_XCHG_P2P");
+    return EA_ESTATE;
+  }
+  static_assert(sizeof(cudaIpcMemHandle_t) == EA_IPC_HANDLE_BYTES, "IPC handle size");
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(handle), h->xbuf);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaIpcGetMemHandle");
+  return EA_OK;
+}
+
+ea_status ea_p2p_open(ea_handle h, const uint8_t* handles, int32_t world) {
+  if (!h || !handles) { set_err(h, "NULL handle or handle list"); return EA_EINVAL; }
+  if (h->cfg.layout != EA_SPREAD || h->cfg.exchange != EA_XCHG_P2P || !h->xbuf) {
+    set_err(h, "ea_p2p_open needs EA_SPREAD with exchange EA_XCHG_P2P");
+    return EA_ESTATE;
+  }
+  if (world != h->cfg.world) { set_err(h, "handle list must have world = %d entries", h->cfg.world); return EA_EINVAL; }
+  if (h->p2p_ready) { set_err(h, "peer exchange already connected"); return EA_ESTATE; }
+  cudaError_t e = cudaSetDevice(h->cfg.device);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
+  return p2p_open_handles(h, handles);
 }
 
 ea_status ea_sync(ea_handle h, void* stream) {

@@ -110,3 +110,19 @@ class CollectiveSpread:
         self.apply_fn(stage, own, reduced)
         parts = list(center.view(self.world, hi - lo).unbind(0))
         dist.all_gather(parts, own.clone(), group=self.group)
+
+
+def connect_p2p(handle, group=None):
+    """Wire an EA_XCHG_P2P handle to its peers over a torch process group
+    (any backend): all-gather the 64-byte CUDA IPC handles and open them.
+    Needed only when the handle was created without an NCCL id."""
+    import torch
+    import torch.distributed as dist
+    mine = handle.p2p_export()
+    world = dist.get_world_size(group)
+    backend = dist.get_backend(group)
+    dev = torch.device("cuda", torch.cuda.current_device()) if backend == "nccl" else torch.device("cpu")
+    t = torch.frombuffer(bytearray(mine), dtype=torch.uint8).to(dev)
+    out = [torch.empty_like(t) for _ in range(world)]
+    dist.all_gather(out, t, group=group)
+    handle.p2p_open([bytes(o.cpu().tolist()) for o in out])

@@ -108,3 +108,69 @@ except EAError as e:
 def test_p2p_missing_rank_times_out_instead_of_hanging():
     out = subprocess.run([sys.executable, "-c", _TIMEOUT_SCRIPT, ROOT], capture_output=True, text=True, timeout=120)
     assert "TIMEOUT REPORTED" in out.stdout, out.stdout + out.stderr
+
+
+def _ipc_worker(rank, world, port, q):
+    """One rank in its own process on cuda:0: IPC handles through gloo, then
+    the fused exchange against the other process (time-sliced on one GPU)."""
+    import numpy as np  # noqa: F401
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    os.environ["AVGPIPE_EA_P2P_TIMEOUT_MS"] = "60000"
+    try:
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+        from paper_conf_ppopp_chen0qz23_b200.parallel import connect_p2p
+        n, sizes, steps = world, [100_003, 70], 5
+        hp = hyper(n, "combined")
+        dev = torch.device("cuda:0")
+        h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                             layout="spread", rank=rank, world=n, exchange="p2p")
+        connect_p2p(h)
+        oracle, gstreams, xs, cs = [], [], [], []
+        for s, p in enumerate(sizes):
+            reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
+            oracle.append(OracleStage(reps, c))
+            gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + s))
+            cc = torch.zeros(h.center_capacity(s), device=dev)
+            cc[:p] = torch.from_numpy(c)
+            cs.append(cc)
+            xs.append(torch.from_numpy(reps[replica_of(rank, s, n)]).to(dev))
+        for t in range(steps):
+            for s in reversed(range(len(sizes))):
+                g = gstreams[s].next()
+                oracle[s].step(g, hp)
+                h.step(s, [xs[s]], [torch.from_numpy(g[replica_of(rank, s, n)]).to(dev)], cs[s])
+        h.sync()
+        torch.cuda.synchronize()
+        for s, p in enumerate(sizes):
+            i = replica_of(rank, s, n)
+            assert rel_err(to_np(xs[s]), oracle[s].xs[i]) <= TOL
+            assert rel_err(to_np(cs[s][:p]), oracle[s].c) <= TOL
+        h.close()
+        q.put((rank, "ok"))
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e)))
+    finally:
+        if dist.is_initialized():
+            dist.destroy_process_group()
+
+
+def test_p2p_exchange_across_processes_via_cuda_ipc():
+    """The multi-process path (cudaIpcGetMemHandle -> all-gather -> cudaIpcOpenMemHandle,
+    system-scope release/acquire across processes) with 2 processes on one GPU."""
+    import socket
+    import torch.multiprocessing as mp
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    procs = [ctx.Process(target=_ipc_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=600) for _ in range(2))
+    for p in procs:
+        p.join(timeout=120)
+    assert all(v == "ok" for v in res.values()), res
