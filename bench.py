@@ -53,6 +53,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--config", default=None, help="override workload key (synth.CONFIGS)")
+    ap.add_argument("--n", type=int, default=None, help="override the number of pipelines (co-located, 1 GPU)")
     return ap.parse_args()
 
 
@@ -159,7 +160,7 @@ def run_ours(args, rank, world, local):
     dev = torch.device("cuda", local)
     key = workload_key(world, args.config)
     cfg = synth.CONFIGS[key]
-    n = cfg.n_pipelines if world == 1 else world
+    n = (args.n or cfg.n_pipelines) if world == 1 else world
     sizes = cfg.stage_sizes
     a, b, r = synth.mode_coeffs(MODE, n)
     lr = synth.LR if args.optimizer == "sgd" else 1e-3
