@@ -227,7 +227,11 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   const int opt = h->cfg.optimizer;
   const bool two = state_slots(h) == 2;
   cudaError_t e = cudaSuccess;
-  if (n > ea::kMaxFusedN) {  // wide N: one launch per stage
+  static const bool force_wide = [] {  // measurement knob: AVGPIPE_EA_FORCE_WIDE=1
+    const char* v = std::getenv("AVGPIPE_EA_FORCE_WIDE");
+    return v && v[0] == '1';
+  }();
+  if (n > ea::kMaxFusedN || force_wide) {  // wide N: one launch per stage
     for (int j = 0; j < count; ++j) {
       const int st = stages[j];
       ea::ReplicaTable t;
