@@ -136,6 +136,19 @@ def workload_key(gpus: int, override):
 
 
 # ----------------------------------------------------------------------------- our arm
+def kernel_name(variant, optimizer, n):
+    """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
+    if n > 8 or (optimizer != "sgd" and n > 4 and variant == "auto"):
+        name = "colocated_wide"
+    elif optimizer != "sgd":
+        name = "colocated_laneshfl"
+    elif variant == "auto":
+        name = "colocated_laneshfl" if n <= 4 else "colocated_regloop"
+    else:
+        name = "colocated_" + variant
+    return name + ("" if optimizer == "sgd" else "<" + optimizer + ">")
+
+
 def bytes_colocated(n, p, optimizer="sgd"):
     """Algorithmic HBM bytes of one co-located launch (fp32): read x~ and, per
     replica, x_i, g_i and the optimizer state; write x_i, the state and x~.
@@ -275,9 +288,7 @@ def run_ours(args, rank, world, local):
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
-                           "kernel": "colocated_" + ("laneshfl" if args.variant == "auto" or args.optimizer != "sgd"
-                                                     else args.variant) + ("" if args.optimizer == "sgd"
-                                                                           else "<" + args.optimizer + ">"),
+                           "kernel": kernel_name(args.variant, args.optimizer, n),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * launches_per_step

@@ -530,7 +530,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
-      mbar_init(&empty[i], kBulkConsumerWarps);
+      mbar_init(&empty[i], 1);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -585,8 +585,9 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
         }
         mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
       }
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&empty[slot]);  // release: this warp's smem reads are done
+      // all consumer warps are done reading the slot, then one release-arrive hands it back
+      asm volatile("bar.sync 1, %0;" ::"n"(32 * kBulkConsumerWarps) : "memory");
+      if (threadIdx.x == 0) mbar_arrive(&empty[slot]);
     }
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
       for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
@@ -841,6 +842,9 @@ cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
+  // library default per N (measured on B200, profiles/r01_nsweep.jsonl): the lane kernel up to N = 4 (the
+  // replicas fill a warp with >= 8 lanes per replica row), the register replica loop beyond
+  if (variant == kVariantAuto) variant = n <= 4 ? kVariantLaneShfl : kVariantRegLoop;
   switch (n) {
     case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
     case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
