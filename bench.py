@@ -143,7 +143,8 @@ def kernel_name(variant, optimizer, n):
     elif optimizer != "sgd":
         name = "colocated_laneshfl"
     elif variant == "auto":
-        name = "colocated_laneshfl" if n <= 4 else "colocated_regloop"
+        name = ("colocated_bulkpipe" if n in (1, 5, 6) else
+                "colocated_laneshfl" if n <= 4 else "colocated_regloop")
     else:
         name = "colocated_" + variant
     return name + ("" if optimizer == "sgd" else "<" + optimizer + ">")

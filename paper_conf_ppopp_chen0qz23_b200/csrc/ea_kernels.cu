@@ -842,9 +842,11 @@ cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
-  // library default per N (measured on B200, profiles/r01_nsweep.jsonl): the lane kernel up to N = 4 (the
-  // replicas fill a warp with >= 8 lanes per replica row), the register replica loop beyond
-  if (variant == kVariantAuto) variant = n <= 4 ? kVariantLaneShfl : kVariantRegLoop;
+  // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl): the bulk-copy pipeline
+  // for N = 1, 5, 6 (0.94 / 1.01 / 0.94 of peak), the lane kernel for N = 2..4 (0.96 / 0.93 / 0.97; a warp
+  // holds >= 8 lanes per replica row), the register replica loop for N = 7, 8 (0.93 / 0.97)
+  if (variant == kVariantAuto)
+    variant = (n == 1 || n == 5 || n == 6) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {
     case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
     case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
