@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=10.0)
     ap.add_argument("--config", default=None, help="override workload key (synth.CONFIGS)")
     ap.add_argument("--n", type=int, default=None, help="override the number of pipelines (co-located, 1 GPU)")
+    ap.add_argument("--layout", choices=("auto", "colocated", "spread"), default="auto",
+                    help="auto: co-located on 1 GPU, spread on N>1; spread on 1 GPU runs the N>1 code path at world 1")
     return ap.parse_args()
 
 
@@ -150,6 +152,15 @@ def kernel_name(variant, optimizer, n):
     return name + ("" if optimizer == "sgd" else "<" + optimizer + ">")
 
 
+def colocated_launches(n, k, args, batched):
+    """Our kernels per co-located step: the fused kernel(s) plus, for Adam, the
+    step-counter kernel that precedes each launch."""
+    adam = args.optimizer != "sgd"
+    per_stage = n > 8 or not batched or (adam and n > 4 and args.variant == "auto")
+    launches = k if per_stage else (k + 7) // 8
+    return launches * (2 if adam else 1)
+
+
 def bytes_colocated(n, p, optimizer="sgd"):
     """Algorithmic HBM bytes of one co-located launch (fp32): read x~ and, per
     replica, x_i, g_i and the optimizer state; write x_i, the state and x~.
@@ -174,13 +185,19 @@ def run_ours(args, rank, world, local):
     dev = torch.device("cuda", local)
     key = workload_key(world, args.config)
     cfg = synth.CONFIGS[key]
-    n = (args.n or cfg.n_pipelines) if world == 1 else world
+    spread = world > 1 or args.layout == "spread"
+    if args.layout == "colocated" and world > 1:
+        raise SystemExit("--layout colocated runs one process per GPU with all N replicas: use --gpus 1")
+    n = (args.n or cfg.n_pipelines) if not spread else world
     sizes = cfg.stage_sizes
     a, b, r = synth.mode_coeffs(MODE, n)
     lr = synth.LR if args.optimizer == "sgd" else 1e-3
     stream = torch.cuda.current_stream(dev)
-    spread = world > 1
     if spread:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        os.environ.setdefault("MASTER_PORT", "29531")
+        os.environ.setdefault("RANK", str(rank))
+        os.environ.setdefault("WORLD_SIZE", str(world))
         dist.init_process_group("nccl", device_id=dev)
         uid = parallel.broadcast_unique_id()
         h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
@@ -292,7 +309,7 @@ def run_ours(args, rank, world, local):
                            "kernel": kernel_name(args.variant, args.optimizer, n),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
-        out["gpu_launches"] = args.steps * launches_per_step
+        out["gpu_launches"] = args.steps * colocated_launches(n, len(sizes), args, batched)
         out["config"]["launch"] = ("CUDA graph replay of ea_step_many (1 kernel/step)" if use_graph
                                    else "ea_step_many (1 launch/step)" if batched else "ea_step per stage")
     else:
@@ -304,7 +321,8 @@ def run_ours(args, rank, world, local):
                            "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None,
                            "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / "
                                    "step time; peak = measured peer copy per direction"}
-        out["gpu_launches"] = args.steps * 2 * len(sizes)
+        per_stage = 2 if args.exchange == "p2p" else (2 if args.optimizer == "sgd" else 3)
+        out["gpu_launches"] = args.steps * per_stage * len(sizes)   # ours only (NCCL kernels excluded)
     out["clocks"] = clk.summary()
     if not spread:
         out["copy_gbs_same_box"] = same_box_copy_gbs(dev)
