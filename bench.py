@@ -30,6 +30,13 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "elastic-avg step params/sec and HBM/NVLink GB/s (% roofline) at 1/2/4/8 B200"
+_JSON_OUT = None
+
+
+def emit(obj):
+    out = _JSON_OUT or sys.stdout
+    out.write(json.dumps(obj) + "\n")
+    out.flush()
 UNIT = "replica-params/s"
 MODE = "combined"   # rho=1, beta=N*alpha, alpha=1/N; every mode moves the same bytes
 
@@ -334,7 +341,7 @@ def run_ours(args, rank, world, local):
         out["cpu_baseline"] = cpu_baseline(cfg, n, seconds=args.cpu_seconds)
     h.close()
     if rank == 0:
-        print(json.dumps(out), flush=True)
+        emit(out)
     if spread:
         dist.destroy_process_group()
 
@@ -455,11 +462,18 @@ def run_reference(args, rank, world):
            "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
            "gpu_launches": 0}
-    print(json.dumps(out), flush=True)
+    emit(out)
 
 
 def main():
     args = parse()
+    # exactly ONE JSON line on stdout: whatever native libraries print there (NCCL's
+    # version banner at communicator init, ...) goes to stderr instead
+    json_out = os.fdopen(os.dup(1), "w")
+    sys.stdout.flush()
+    os.dup2(2, 1)
+    global _JSON_OUT
+    _JSON_OUT = json_out
     rank, world, local = dist_env()
     if world != args.gpus and rank == 0:
         print(f"note: WORLD_SIZE={world} but --gpus={args.gpus}; using WORLD_SIZE", file=sys.stderr)
