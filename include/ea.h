@@ -166,12 +166,15 @@ EA_API int64_t ea_shard_elems(ea_handle h, int32_t stage);
  *   grad_ptrs:    matching gradient pointers (read only).
  *   center_ptr:   x~ of the stage (ea_center_capacity floats), updated in place.
  *   stream:       caller's stream (cudaStream_t); NULL = legacy default stream.
- * EA_COLOCATED: one fused kernel on `stream`.  EA_SPREAD: the side stream
- * waits for `stream`, runs kernel -> reduce-scatter -> shard update ->
- * all-gather; `stream` then waits only for the kernel (x_i ready), so the
- * next forward can start while the center is being exchanged.  Call
- * ea_sync before reading x~ on another stream.  All ranks must call
- * ea_step for the same stages in the same order (NCCL ordering).
+ * EA_COLOCATED: one fused kernel on `stream`.  EA_SPREAD with EA_XCHG_NCCL:
+ * the local kernel (x_i, optimizer state, contribution) runs on `stream`
+ * after this stage's previous all-gather; the exchange (reduce-scatter ->
+ * shard update -> all-gather) runs on the library's side stream and `stream`
+ * does NOT wait for it -- the next forward and the other stages' local steps
+ * proceed while the center is exchanged (never block the
+ * pipelines).  EA_XCHG_P2P: one fused kernel on `stream` (local update and
+ * exchange).  Call ea_sync before reading x~ on any stream.  All ranks must
+ * call ea_step for the same stages in the same order (collective ordering).
  * Pointers must stay valid until the work completes. */
 EA_API ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
                   const float* const* grad_ptrs, float* center_ptr, void* stream);

@@ -36,8 +36,11 @@ struct ea_ctx {
   ea::StepCoef* d_coef = nullptr;  // device Adam bias corrections of the current step
   // EA_SPREAD
   cudaStream_t side = nullptr;
-  cudaEvent_t ev_in = nullptr, ev_local = nullptr, ev_done = nullptr;
-  float* contrib = nullptr;  // max P_pad floats
+  cudaEvent_t ev_done = nullptr;
+  float* contrib = nullptr;  // NCCL exchange: sum_s P_pad(s) floats, one contribution buffer per stage
+  std::vector<size_t> contrib_off;       // per-stage offset into contrib (floats)
+  std::vector<cudaEvent_t> ev_ag;        // per stage: its last all-gather (center final) on the side stream
+  std::vector<cudaEvent_t> ev_loc;       // per stage: its last local kernel on the caller's stream
   float* reduced = nullptr;  // max P_pad/N floats
   ncclComm_t comm = nullptr;
   // EA_SPREAD with exchange == EA_XCHG_P2P (fused peer-memory kernel)
@@ -167,11 +170,11 @@ void free_ctx(ea_ctx* h) {
   for (auto& slot : h->state)
     for (float* m : slot) if (m) cudaFree(m);
   if (h->contrib) cudaFree(h->contrib);
+  for (cudaEvent_t ev : h->ev_ag) if (ev) cudaEventDestroy(ev);
+  for (cudaEvent_t ev : h->ev_loc) if (ev) cudaEventDestroy(ev);
   if (h->reduced) cudaFree(h->reduced);
   if (h->d_steps) cudaFree(h->d_steps);
   if (h->d_coef) cudaFree(h->d_coef);
-  if (h->ev_in) cudaEventDestroy(h->ev_in);
-  if (h->ev_local) cudaEventDestroy(h->ev_local);
   if (h->ev_done) cudaEventDestroy(h->ev_done);
   if (h->side) cudaStreamDestroy(h->side);
   if (h->h2d) cudaStreamSynchronize(h->h2d);
@@ -290,24 +293,28 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
   const int n = h->cfg.n_pipelines;
   const int64_t pad = h->p_pad[stage], shard = pad / n;
   float* own = center_ptr + shard * h->cfg.rank;
-  if ((e = cudaEventRecord(h->ev_in, s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-  if ((e = cudaStreamWaitEvent(h->side, h->ev_in, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
-  ea_status st2 = advance(h, &stage, 1, h->side);
+  float* contrib = h->contrib + h->contrib_off[stage];
+  // Local phase on the CALLER's stream (x_i, state and r_i ready there, in stream order): it reads the
+  // center, so it waits for this stage's previous all-gather (a no-op wait when that finished long ago).
+  if ((e = cudaStreamWaitEvent(s, h->ev_ag[stage], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  ea_status st2 = advance(h, &stage, 1, s);
   if (st2 != EA_OK) return st2;
-  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr,
-                              h->contrib, h->p[stage], pad, h->hp, h->cfg.optimizer, h->d_coef + stage, h->num_sms,
-                              h->side);
+  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr, contrib,
+                              h->p[stage], pad, h->hp, h->cfg.optimizer, h->d_coef + stage, h->num_sms, s);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
-  if ((e = cudaEventRecord(h->ev_local, h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-  ncclResult_t r = ncclReduceScatter(h->contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
+  if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  // Exchange on the side stream: reduce-scatter -> owner-shard update -> in-place all-gather.  The caller's
+  // stream does not wait for it; the next local step of this stage (or ea_sync) does.
+  if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
+    return cuda_fail(h, e, "cudaStreamWaitEvent");
+  ncclResult_t r = ncclReduceScatter(contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
                                      h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
   e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, h->side);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
   r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
-  // The caller's stream waits only for x_i (the next forward may start now).
-  if ((e = cudaStreamWaitEvent(s, h->ev_local, 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  if ((e = cudaEventRecord(h->ev_ag[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   return EA_OK;
 }
 
@@ -546,12 +553,14 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   }
 
   const int reps = replicas_here(h);
-  int64_t max_pad = 0;
+  int64_t max_pad = 0, sum_pad = 0;
   for (int s = 0; s < c.n_stages; ++s) {
     const int64_t ps = h->p[s];
     const int64_t pad = c.layout == EA_SPREAD ? round_up(ps, 32LL * c.n_pipelines) : ps;
     h->p_pad.push_back(pad);
     if (pad > max_pad) max_pad = pad;
+    h->contrib_off.push_back(static_cast<size_t>(sum_pad));
+    sum_pad += pad;
     const int64_t stride = round_up(ps, 64);
     h->stride.push_back(stride);
     for (int slot = 0; slot < state_slots(h); ++slot) {
@@ -569,14 +578,24 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   }
   if (c.layout == EA_SPREAD) {
     if ((e = cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking)) != cudaSuccess ||
-        (e = cudaEventCreateWithFlags(&h->ev_in, cudaEventDisableTiming)) != cudaSuccess ||
-        (e = cudaEventCreateWithFlags(&h->ev_local, cudaEventDisableTiming)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_done, cudaEventDisableTiming)) != cudaSuccess ||
-        (e = cudaMalloc(&h->contrib, sizeof(float) * max_pad)) != cudaSuccess ||
+        (c.exchange == EA_XCHG_NCCL && (e = cudaMalloc(&h->contrib, sizeof(float) * sum_pad)) != cudaSuccess) ||
         (e = cudaMalloc(&h->reduced, sizeof(float) * (max_pad / c.n_pipelines))) != cudaSuccess) {
       ea_status r = cuda_fail(nullptr, e, "spread resources");
       free_ctx(h);
       return r;
+    }
+    for (int st = 0; st < c.n_stages; ++st) {
+      cudaEvent_t a = nullptr, b = nullptr;
+      if ((e = cudaEventCreateWithFlags(&a, cudaEventDisableTiming)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&b, cudaEventDisableTiming)) != cudaSuccess) {
+        if (a) cudaEventDestroy(a);
+        ea_status r = cuda_fail(nullptr, e, "per-stage events");
+        free_ctx(h);
+        return r;
+      }
+      h->ev_ag.push_back(a);
+      h->ev_loc.push_back(b);
     }
     if (nccl_id) {  // NULL: external-collective mode (phase calls only)
       ncclUniqueId uid;
