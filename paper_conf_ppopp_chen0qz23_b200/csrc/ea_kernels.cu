@@ -510,16 +510,20 @@ constexpr int kBulkConsumerWarps = 8;
 constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 
 template <int N>
+constexpr int default_bulk_tile() { return (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128; }  // slot <= ~56 KB
+
+template <int N, int TILE = default_bulk_tile<N>()>
 struct BulkGeom {
-  static constexpr int kTile = (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128;  // keep a slot <= ~56 KB
-  static constexpr int kSlotVec = (3 * N + 1) * kTile;                        // float4 per slot
-  static constexpr int kStages = (kSlotVec * 16 * 4 <= 200 * 1024) ? 4 : 3;
+  static constexpr int kTile = TILE;                      // float4 per array per tile
+  static constexpr int kSlotVec = (3 * N + 1) * kTile;    // float4 per slot
+  static constexpr int kFit = (200 * 1024) / (kSlotVec * 16);
+  static constexpr int kStages = kFit > 6 ? 6 : (kFit < 2 ? 2 : kFit);
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
 
-template <int N, int HINT>
+template <int N, int HINT, int TILE = default_bulk_tile<N>()>
 __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
-  using G = BulkGeom<N>;
+  using G = BulkGeom<N, TILE>;
   constexpr int T = G::kTile, S = G::kStages;
   extern __shared__ __align__(128) float4 smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * G::kSlotVec);
@@ -768,10 +772,10 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
   return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 2>(b, hp, num_sms, s);  // <= 128 regs: 2 CTAs/SM
 }
 
-template <int N, int HINT>
-cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using G = BulkGeom<N>;
-  auto k = colocated_bulkpipe<N, HINT>;
+template <int N, int HINT, int TILE>
+cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  using G = BulkGeom<N, TILE>;
+  auto k = colocated_bulkpipe<N, HINT, TILE>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
   if (e != cudaSuccess) return e;
   int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
@@ -779,6 +783,29 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
   if (grid > units) grid = units;
   k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp);
   return cudaGetLastError();
+}
+
+// Tile knob for measurement: AVGPIPE_EA_BULK_TILE = 64 | 128 | 256 float4 per array.
+int bulk_tile() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_BULK_TILE");
+    return e ? std::atoi(e) : 0;
+  }();
+  return v;
+}
+
+template <int N, int HINT>
+cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  if constexpr (HINT == 0) {
+    switch (bulk_tile()) {
+      case 64: return launch_bulkpipe_t<N, HINT, 64>(b, hp, num_sms, s);
+      case 128: return launch_bulkpipe_t<N, HINT, 128>(b, hp, num_sms, s);
+      case 256: if ((3 * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 256>(b, hp, num_sms, s);
+                break;
+      default: break;
+    }
+  }
+  return launch_bulkpipe_t<N, HINT, default_bulk_tile<N>()>(b, hp, num_sms, s);
 }
 
 template <int N>
