@@ -800,8 +800,12 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
     switch (bulk_tile()) {
       case 64: return launch_bulkpipe_t<N, HINT, 64>(b, hp, num_sms, s);
       case 128: return launch_bulkpipe_t<N, HINT, 128>(b, hp, num_sms, s);
-      case 256: if ((3 * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 256>(b, hp, num_sms, s);
-                break;
+      case 256:
+        if constexpr ((3 * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 256>(b, hp, num_sms, s);
+        break;
+      case 512:
+        if constexpr ((3 * N + 1) * 512 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 512>(b, hp, num_sms, s);
+        break;
       default: break;
     }
   }
