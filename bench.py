@@ -152,7 +152,7 @@ def kernel_name(variant, optimizer, n):
     elif optimizer != "sgd":
         name = "colocated_laneshfl"
     elif variant == "auto":
-        name = ("colocated_bulkpipe" if n in (1, 5, 6) else
+        name = ("colocated_bulkpipe" if n in (1, 5, 6, 7) else
                 "colocated_laneshfl" if n <= 4 else "colocated_regloop")
     else:
         name = "colocated_" + variant

@@ -509,8 +509,11 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
 constexpr int kBulkConsumerWarps = 8;
 constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 
+// Default tile (float4 per array per bulk copy), measured on B200 (profiles/r01_bulk_tiles.jsonl): 4 KB
+// copies except N = 4, 5 (2 KB copies, deeper ring) -- larger copies need fewer stages to keep the
+// same bytes in flight and reach DRAM as longer bursts.
 template <int N>
-constexpr int default_bulk_tile() { return (3 * N + 1) * 256 * 16 <= 57344 ? 256 : 128; }  // slot <= ~56 KB
+constexpr int default_bulk_tile() { return (N == 4 || N == 5) ? 128 : 256; }
 
 template <int N, int TILE = default_bulk_tile<N>()>
 struct BulkGeom {
@@ -873,11 +876,11 @@ cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
-  // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl): the bulk-copy pipeline
-  // for N = 1, 5, 6 (0.94 / 1.01 / 0.94 of peak), the lane kernel for N = 2..4 (0.96 / 0.93 / 0.97; a warp
-  // holds >= 8 lanes per replica row), the register replica loop for N = 7, 8 (0.93 / 0.97)
+  // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl, r01_bulk_tiles.jsonl):
+  // the bulk-copy pipeline for N = 1, 5, 6, 7 (0.93 / 1.01 / 0.95 / 0.95 of peak), the lane kernel for
+  // N = 2..4 (0.96 / 0.93 / 0.97; a warp holds >= 8 lanes per replica row), the register loop for N = 8 (0.97)
   if (variant == kVariantAuto)
-    variant = (n == 1 || n == 5 || n == 6) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
+    variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {
     case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
     case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
