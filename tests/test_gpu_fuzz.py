@@ -29,12 +29,12 @@ def _case(seed):
               lr=float(rng.uniform(1e-3, 0.1)) if opt == "sgd" else float(rng.uniform(1e-4, 3e-3)),
               momentum=momentum, weight_decay=float(rng.choice([0.0, 1e-4, 1e-2])), nesterov=nesterov,
               betas=(float(rng.uniform(0.8, 0.95)), float(rng.uniform(0.99, 0.9999))), eps=1e-8)
-    variant = str(rng.choice(["auto", "regloop", "laneshfl", "bulkpipe"]))
+    variant = str(rng.choice(["auto", "auto", "regloop", "laneshfl", "bulkpipe"]))
     form = str(rng.choice(["step", "many", "host"]))
     return n, sizes, opt, hp, variant, form
 
 
-@pytest.mark.parametrize("seed", range(40))
+@pytest.mark.parametrize("seed", range(120))
 def test_random_configuration(seed):
     n, sizes, opt, hp, variant, form = _case(seed)
     dev = torch.device("cuda:0")

@@ -127,7 +127,7 @@ def test_adam_replica_counts_and_sizes(optimizer, n):
     _run_colocated(n, sizes[:1], 10, "paper", optimizer=optimizer, lr=1e-3, variants=("auto",))
 
 
-@pytest.mark.parametrize("n", [1, 3, 5, 8, 12])
+@pytest.mark.parametrize("n", [1, 3, 5, 6, 7, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_replica_counts(n, mode):
     _run_colocated(n, [65_539, 4097], 30, mode)
