@@ -512,25 +512,30 @@ constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 // Default tile (float4 per array per bulk copy), measured on B200 (profiles/r01_bulk_tiles.jsonl): 4 KB
 // copies except N = 4, 5 (2 KB copies, deeper ring) -- larger copies need fewer stages to keep the
 // same bytes in flight and reach DRAM as longer bursts.
-template <int N>
-constexpr int default_bulk_tile() { return (N == 4 || N == 5) ? 128 : 256; }
+template <int N, int A = 3>
+constexpr int default_bulk_tile() {
+  return A == 3 ? ((N == 4 || N == 5) ? 128 : 256) : ((A * N + 1) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128);
+}
 
-template <int N, int TILE = default_bulk_tile<N>()>
+// A = streams per replica in the slot: 3 (x, g, m) for SGD, 4 (x, g, m, v) for Adam.
+template <int N, int TILE, int A>
 struct BulkGeom {
   static constexpr int kTile = TILE;                      // float4 per array per tile
-  static constexpr int kSlotVec = (3 * N + 1) * kTile;    // float4 per slot
+  static constexpr int kSlotVec = (A * N + 1) * kTile;    // float4 per slot
   static constexpr int kFit = (200 * 1024) / (kSlotVec * 16);
   static constexpr int kStages = kFit > 6 ? 6 : (kFit < 2 ? 2 : kFit);
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
 
-template <int N, int HINT, int TILE = default_bulk_tile<N>()>
+template <int N, int HINT, int OPT, int TILE>
 __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
-  using G = BulkGeom<N, TILE>;
+  constexpr int A = OPT == kOptSGD ? 3 : 4;
+  using G = BulkGeom<N, TILE, A>;
   constexpr int T = G::kTile, S = G::kStages;
   extern __shared__ __align__(128) float4 smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * G::kSlotVec);
   uint64_t* empty = full + S;
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
   const Mem<HINT> mem;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
@@ -541,6 +546,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if (OPT != kOptSGD && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
   __syncthreads();
 
   if (warp == kBulkConsumerWarps) {
@@ -556,13 +562,14 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
         float4* base = smem + slot * G::kSlotVec;
         const uint32_t bytes = static_cast<uint32_t>(nv * 16);
         const StageRefs& st = b.st[s];
-        mbar_expect_tx(&full[slot], bytes * (3 * N + 1));
+        mbar_expect_tx(&full[slot], bytes * (A * N + 1));
         bulk_g2s(base, st.c + 4 * v0, bytes, &full[slot]);
 #pragma unroll
         for (int i = 0; i < N; ++i) {
-          bulk_g2s(base + (1 + 3 * i) * T, st.x[i] + 4 * v0, bytes, &full[slot]);
-          bulk_g2s(base + (2 + 3 * i) * T, st.g[i] + 4 * v0, bytes, &full[slot]);
-          bulk_g2s(base + (3 + 3 * i) * T, st.m[i] + 4 * v0, bytes, &full[slot]);
+          bulk_g2s(base + (1 + A * i) * T, st.x[i] + 4 * v0, bytes, &full[slot]);
+          bulk_g2s(base + (2 + A * i) * T, st.g[i] + 4 * v0, bytes, &full[slot]);
+          bulk_g2s(base + (3 + A * i) * T, st.m[i] + 4 * v0, bytes, &full[slot]);
+          if (A == 4) bulk_g2s(base + (4 + A * i) * T, st.v[i] + 4 * v0, bytes, &full[slot]);
         }
       }
     }
@@ -576,19 +583,21 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
       mbar_wait(&full[slot], (k / S) & 1);
       const float4* base = smem + slot * G::kSlotVec;
       const StageRefs& st = b.st[s];
+      const StepCoef sc = OPT == kOptSGD ? StepCoef{0.f, 0.f} : s_coef[s];
       for (int lv = threadIdx.x; lv < nv; lv += 32 * kBulkConsumerWarps) {
         const float4 c = base[lv];
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
         const int64_t v = v0 + lv;
 #pragma unroll
         for (int i = 0; i < N; ++i) {
-          float4 x = base[(1 + 3 * i) * T + lv];
-          const float4 g = base[(2 + 3 * i) * T + lv];
-          float4 m = base[(3 + 3 * i) * T + lv];
-          float4 unused;
-          add4(acc, ea_vec<kOptSGD>(x, g, m, unused, c, hp, StepCoef{0.f, 0.f}));
+          float4 x = base[(1 + A * i) * T + lv];
+          const float4 g = base[(2 + A * i) * T + lv];
+          float4 m = base[(3 + A * i) * T + lv];
+          float4 w = A == 4 ? base[(4 + A * i) * T + lv] : make_float4(0.f, 0.f, 0.f, 0.f);
+          add4(acc, ea_vec<OPT>(x, g, m, w, c, hp, sc));
           mem.st(st.x[i] + 4 * v, x);
           mem.st(st.m[i] + 4 * v, m);
+          if (A == 4) mem.st(st.v[i] + 4 * v, w);
         }
         mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
       }
@@ -597,7 +606,7 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
       if (threadIdx.x == 0) mbar_arrive(&empty[slot]);
     }
     if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-      for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
+      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
   }
 }
 
@@ -775,10 +784,10 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
   return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 2>(b, hp, num_sms, s);  // <= 128 regs: 2 CTAs/SM
 }
 
-template <int N, int HINT, int TILE>
+template <int N, int HINT, int OPT, int TILE>
 cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using G = BulkGeom<N, TILE>;
-  auto k = colocated_bulkpipe<N, HINT, TILE>;
+  using G = BulkGeom<N, TILE, OPT == kOptSGD ? 3 : 4>;
+  auto k = colocated_bulkpipe<N, HINT, OPT, TILE>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
   if (e != cudaSuccess) return e;
   int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
@@ -788,7 +797,7 @@ cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms,
   return cudaGetLastError();
 }
 
-// Tile knob for measurement: AVGPIPE_EA_BULK_TILE = 64 | 128 | 256 float4 per array.
+// Tile knob for measurement: AVGPIPE_EA_BULK_TILE = 64 | 128 | 256 | 512 float4 per array.
 int bulk_tile() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_BULK_TILE");
@@ -797,31 +806,35 @@ int bulk_tile() {
   return v;
 }
 
-template <int N, int HINT>
+template <int N, int HINT, int OPT>
 cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  constexpr int A = OPT == kOptSGD ? 3 : 4;
   if constexpr (HINT == 0) {
     switch (bulk_tile()) {
-      case 64: return launch_bulkpipe_t<N, HINT, 64>(b, hp, num_sms, s);
-      case 128: return launch_bulkpipe_t<N, HINT, 128>(b, hp, num_sms, s);
+      case 64: return launch_bulkpipe_t<N, HINT, OPT, 64>(b, hp, num_sms, s);
+      case 128: return launch_bulkpipe_t<N, HINT, OPT, 128>(b, hp, num_sms, s);
       case 256:
-        if constexpr ((3 * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 256>(b, hp, num_sms, s);
+        if constexpr ((A * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, OPT, 256>(b, hp, num_sms, s);
         break;
       case 512:
-        if constexpr ((3 * N + 1) * 512 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, 512>(b, hp, num_sms, s);
+        if constexpr ((A * N + 1) * 512 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, OPT, 512>(b, hp, num_sms, s);
         break;
       default: break;
     }
   }
-  return launch_bulkpipe_t<N, HINT, default_bulk_tile<N>()>(b, hp, num_sms, s);
+  return launch_bulkpipe_t<N, HINT, OPT, default_bulk_tile<N, A>()>(b, hp, num_sms, s);
 }
 
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (opt != kOptSGD && variant == kVariantBulkPipe)
+    return opt == kOptAdam ? launch_bulkpipe<N, 0, kOptAdam>(b, hp, num_sms, s)
+                           : launch_bulkpipe<N, 0, kOptAdamW>(b, hp, num_sms, s);
   if (opt == kOptAdam) return launch_laneshfl<N, 0, kOptAdam>(b, hp, num_sms, s);
   if (opt == kOptAdamW) return launch_laneshfl<N, 0, kOptAdamW>(b, hp, num_sms, s);
   const bool hint = l2_hint() != 0;
   if (variant == kVariantBulkPipe)
-    return hint ? launch_bulkpipe<N, 1>(b, hp, num_sms, s) : launch_bulkpipe<N, 0>(b, hp, num_sms, s);
+    return hint ? launch_bulkpipe<N, 1, kOptSGD>(b, hp, num_sms, s) : launch_bulkpipe<N, 0, kOptSGD>(b, hp, num_sms, s);
   if (variant == kVariantRegLoop)
     return hint ? launch_regloop<N, 1>(b, hp, num_sms, s) : launch_regloop<N, 0>(b, hp, num_sms, s);
   return hint ? launch_laneshfl<N, 1, kOptSGD>(b, hp, num_sms, s) : launch_laneshfl<N, 0, kOptSGD>(b, hp, num_sms, s);
@@ -879,6 +892,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl, r01_bulk_tiles.jsonl):
   // the bulk-copy pipeline for N = 1, 5, 6, 7 (0.93 / 1.01 / 0.95 / 0.95 of peak), the lane kernel for
   // N = 2..4 (0.96 / 0.93 / 0.97; a warp holds >= 8 lanes per replica row), the register loop for N = 8 (0.97)
+  if (variant == kVariantAuto && opt != kOptSGD) variant = kVariantLaneShfl;
   if (variant == kVariantAuto)
     variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {

@@ -127,6 +127,15 @@ def test_adam_replica_counts_and_sizes(optimizer, n):
     _run_colocated(n, sizes[:1], 10, "paper", optimizer=optimizer, lr=1e-3, variants=("auto",))
 
 
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+@pytest.mark.parametrize("n", [1, 2, 4, 5, 8])
+def test_adam_bulk_pipeline(optimizer, n):
+    """Adam/AdamW through the bulk-copy pipeline (x, g, m, v of every replica in the slot)."""
+    sizes = [100_003, 7, 4096]
+    _run_colocated(n, sizes, 12, "combined", optimizer=optimizer, lr=1e-3, wd=1e-2, many=True,
+                   variants=("bulkpipe",))
+
+
 @pytest.mark.parametrize("n", [1, 3, 5, 6, 7, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_replica_counts(n, mode):
