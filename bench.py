@@ -147,10 +147,11 @@ def workload_key(gpus: int, override):
 # ----------------------------------------------------------------------------- our arm
 def kernel_name(variant, optimizer, n):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
-    if n > 8 or (optimizer != "sgd" and n > 4 and variant == "auto"):
+    if n > 8 or (optimizer != "sgd" and n > 6 and variant == "auto"):
         name = "colocated_wide"
     elif optimizer != "sgd":
-        name = "colocated_laneshfl"
+        name = ("colocated_laneshfl" if (n <= 2 and variant == "auto") or variant == "laneshfl"
+                else "colocated_" + ("bulkpipe" if variant == "auto" else variant))
     elif variant == "auto":
         name = ("colocated_bulkpipe" if n in (1, 5, 6, 7) else
                 "colocated_laneshfl" if n <= 4 else "colocated_regloop")
@@ -163,7 +164,7 @@ def colocated_launches(n, k, args, batched):
     """Our kernels per co-located step: the fused kernel(s) plus, for Adam, the
     step-counter kernel that precedes each launch."""
     adam = args.optimizer != "sgd"
-    per_stage = n > 8 or not batched or (adam and n > 4 and args.variant == "auto")
+    per_stage = n > 8 or not batched or (adam and n > 6 and args.variant == "auto")
     launches = k if per_stage else (k + 7) // 8
     return launches * (2 if adam else 1)
 

@@ -234,9 +234,9 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
     const char* v = std::getenv("AVGPIPE_EA_FORCE_WIDE");
     return v && v[0] == '1';
   }();
-  // Adam with N > 4: the lane kernel's per-lane state (4 streams x 4 passes) costs occupancy; the
-  // replica-loop kernel measured faster (0.914 vs 0.727 of peak at N = 8, profiles/r01_nsweep.jsonl)
-  const bool adam_wide = opt != EA_OPT_SGD && n > 4 && h->variant == 0;
+  // Adam with N > 6: the replica-loop kernel measured fastest (0.919 of peak at N = 8 vs 0.75 bulk-copy
+  // pipeline and 0.73 lane kernel, profiles/r01_adam_nsweep.jsonl)
+  const bool adam_wide = opt != EA_OPT_SGD && n > 6 && h->variant == 0;
   if (n > ea::kMaxFusedN || force_wide || adam_wide) {  // wide N: one launch per stage
     for (int j = 0; j < count; ++j) {
       const int st = stages[j];

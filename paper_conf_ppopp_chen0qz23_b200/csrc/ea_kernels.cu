@@ -892,7 +892,9 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl, r01_bulk_tiles.jsonl):
   // the bulk-copy pipeline for N = 1, 5, 6, 7 (0.93 / 1.01 / 0.95 / 0.95 of peak), the lane kernel for
   // N = 2..4 (0.96 / 0.93 / 0.97; a warp holds >= 8 lanes per replica row), the register loop for N = 8 (0.97)
-  if (variant == kVariantAuto && opt != kOptSGD) variant = kVariantLaneShfl;
+  // Adam(W) (profiles/r01_adam_nsweep.jsonl): the lane kernel for N <= 2 (0.91 / 0.94), the bulk-copy
+  // pipeline for N = 3..6 (0.89 / 0.96 / 0.94 / 0.92); N > 6 goes to the replica-loop kernel (ea_api.cu)
+  if (variant == kVariantAuto && opt != kOptSGD) variant = n <= 2 ? kVariantLaneShfl : kVariantBulkPipe;
   if (variant == kVariantAuto)
     variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {
