@@ -61,8 +61,19 @@ struct ea_ctx {
   std::string err;
 };
 
-// Elements per pipelined chunk of the host-buffer path (a multiple of 64).
+// Elements per pipelined chunk of the host-buffer path (a multiple of 64).  AVGPIPE_EA_HOST_CHUNK
+// (elements, measurement knob) overrides it up to the staging capacity.
 constexpr int64_t kHostChunk = 4 << 20;
+
+int64_t host_chunk() {
+  static int64_t v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_HOST_CHUNK");
+    long long c = e ? std::atoll(e) : 0;
+    if (c <= 0 || c > kHostChunk) return kHostChunk;
+    return static_cast<int64_t>((c + 63) / 64 * 64);
+  }();
+  return v;
+}
 // Floats per exchange chunk of the fused peer-memory spread kernel (32 KB).
 constexpr int64_t kP2PChunk = 8192;
 
@@ -730,8 +741,9 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
     if (st2 != EA_OK) return st2;
     const ea::StepCoef* sc = h->d_coef + st;
     const int64_t ps = h->p[st];
-    for (int64_t off = 0; off < ps; off += kHostChunk, ++k) {
-      const int64_t len = ps - off < kHostChunk ? ps - off : kHostChunk;
+    const int64_t chunk = host_chunk();
+    for (int64_t off = 0; off < ps; off += chunk, ++k) {
+      const int64_t len = ps - off < chunk ? ps - off : chunk;
       const int b = static_cast<int>(k & 1);
       float* stage_buf = h->staging[b];
       // H2D of this chunk's gradients once the kernel that last read this buffer is done
