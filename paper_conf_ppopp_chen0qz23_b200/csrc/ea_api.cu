@@ -757,7 +757,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
       if ((e = cudaEventRecord(h->ev_h2d[b], h->h2d)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
       if ((e = cudaStreamWaitEvent(s, h->ev_h2d[b], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
       // the fused step on [off, off+len) of the stage (elementwise: any chunk is a valid sub-problem)
-      if (n > ea::kMaxFusedN) {
+      if (n > ea::kMaxFusedN || (opt != EA_OPT_SGD && n > 6 && h->variant == 0)) {
         ea::ReplicaTable t;
         for (int i = 0; i < n; ++i) {
           t.x[i] = replica_ptrs[(size_t)j * n + i] + off;
