@@ -136,6 +136,13 @@ def test_adam_bulk_pipeline(optimizer, n):
                    variants=("bulkpipe",))
 
 
+@pytest.mark.parametrize("n,optimizer", [(33, "sgd"), (64, "sgd"), (64, "adamw")])
+def test_maximum_replica_count(n, optimizer):
+    """EA_MAX_REPLICAS = 64 co-located replicas (the replica-loop kernel's pointer table)."""
+    _run_colocated(n, [20_003, 5], 6, "combined", optimizer=optimizer, lr=1e-3 if optimizer != "sgd" else synth.LR,
+                   many=True, variants=("auto",))
+
+
 @pytest.mark.parametrize("n", [1, 3, 5, 6, 7, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_replica_counts(n, mode):
