@@ -83,8 +83,11 @@ def test_p2p_exchange_adam(n, optimizer):
     _run(n, [300_001, 17], 12, "combined", optimizer)
 
 
-def test_p2p_exchange_c1_100_steps():
-    _run(2, [1_000_000, 1_000_003], 100, "combined")
+@pytest.mark.parametrize("n", [2, 4, 8])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_p2p_exchange_c1_100_steps(n, mode):
+    """The north-star gate in the spread layout: C1 sizes + the 1,000,003 tail stage, 100 steps, N = 2/4/8."""
+    _run(n, [1_000_000, 1_000_003], 100, mode)
 
 
 _TIMEOUT_SCRIPT = r'''

@@ -178,11 +178,10 @@ def _placement(rank, stage, n):
 
 @pytest.mark.parametrize("n,optimizer", [(2, "sgd"), (3, "sgd"), (4, "sgd"), (8, "sgd"), (2, "adam"), (4, "adamw")])
 @pytest.mark.parametrize("mode", synth.MODES)
-def test_spread_decomposition_virtual_ranks(n, mode, optimizer):
+def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 64), steps=20):
     """N ranks on one GPU, external-collective mode: the real local and shard
     kernels, with the reduce-scatter / all-gather done by the test."""
-    sizes = [200_003, 64]
-    steps = 20
+    sizes = list(sizes)
     hp = hyper(n, mode, lr=synth.LR if optimizer == "sgd" else 1e-3, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     hs = [ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
@@ -236,6 +235,13 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer):
             assert torch.all(centers[s][r][p:] == 0), "center padding must stay zero"
     for h in hs:
         h.close()
+
+
+@pytest.mark.parametrize("n", [2, 4, 8])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_spread_decomposition_c1_100_steps(n, mode):
+    """North-star gate for the NCCL layout's kernels: C1 + tail stage, 100 steps, N = 2/4/8 virtual ranks."""
+    test_spread_decomposition_virtual_ranks(n, mode, "sgd", sizes=(1_000_000, 1_000_003), steps=100)
 
 
 def test_spread_nccl_world1_and_stream_order():
