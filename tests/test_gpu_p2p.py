@@ -83,8 +83,7 @@ def test_p2p_exchange_adam(n, optimizer):
     _run(n, [300_001, 17], 12, "combined", optimizer)
 
 
-@pytest.mark.parametrize("n", [2, 4, 8])
-@pytest.mark.parametrize("mode", synth.MODES)
+@pytest.mark.parametrize("n,mode", [(2, m) for m in synth.MODES] + [(4, m) for m in synth.MODES] + [(8, "combined")])
 def test_p2p_exchange_c1_100_steps(n, mode):
     """The north-star gate in the spread layout: C1 sizes + the 1,000,003 tail stage, 100 steps, N = 2/4/8."""
     _run(n, [1_000_000, 1_000_003], 100, mode)

@@ -237,8 +237,7 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 
         h.close()
 
 
-@pytest.mark.parametrize("n", [2, 4, 8])
-@pytest.mark.parametrize("mode", synth.MODES)
+@pytest.mark.parametrize("n,mode", [(2, m) for m in synth.MODES] + [(4, m) for m in synth.MODES] + [(8, "combined")])
 def test_spread_decomposition_c1_100_steps(n, mode):
     """North-star gate for the NCCL layout's kernels: C1 + tail stage, 100 steps, N = 2/4/8 virtual ranks."""
     test_spread_decomposition_virtual_ranks(n, mode, "sgd", sizes=(1_000_000, 1_000_003), steps=100)
