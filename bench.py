@@ -300,6 +300,7 @@ def run_ours(args, rank, world, local):
     out["config"] = {"workload": cfg.name, "n_pipelines": n, "n_stages": len(sizes), "params": total_params,
                      "stage_params": sizes, "layout": "spread" if spread else "colocated", "mode": MODE,
                      "exchange": args.exchange if spread else None,
+                     "nccl_env": {k: v for k, v in os.environ.items() if k.startswith("NCCL_")} if spread else None,
                      "optimizer": "sgd-momentum(0.9)" if args.optimizer == "sgd" else args.optimizer,
                      "kernel": args.variant,
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}

@@ -19,8 +19,18 @@
 #include <string>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "../../include/ea.h"
 #include "ea_internal.h"
+
+namespace {
+// NVTX range around each ABI call that enqueues work (visible in nsys timelines).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 
 struct ea_ctx {
   ea_config cfg{};
@@ -648,6 +658,7 @@ int64_t ea_shard_elems(ea_handle h, int32_t stage) {
 
 ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const float* const* grad_ptrs,
                   float* center_ptr, void* stream) {
+  NvtxRange range("ea_step");
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   ea_status st = check_stage_ptrs(h, stage, replica_ptrs, grad_ptrs, center_ptr);
   if (st != EA_OK) return st;
@@ -664,6 +675,7 @@ ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs, const 
 
 ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
                        const float* const* grad_ptrs, float* const* center_ptrs, void* stream) {
+  NvtxRange range("ea_step_many");
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   if (count < 0 || (count > 0 && (!stages || !replica_ptrs || !grad_ptrs || !center_ptrs))) {
     set_err(h, "ea_step_many: bad count or NULL array");
@@ -696,6 +708,7 @@ ea_status ea_step_many(ea_handle h, int32_t count, const int32_t* stages, float*
 ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
                             const float* const* host_grad_ptrs, float* const* center_ptrs,
                             float* const* host_center_out, void* stream) {
+  NvtxRange range("ea_step_many_host");
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   if (h->cfg.layout != EA_COLOCATED) { set_err(h, "ea_step_many_host needs EA_COLOCATED"); return EA_ESTATE; }
   if (count < 0 || (count > 0 && (!stages || !replica_ptrs || !host_grad_ptrs || !center_ptrs || !host_center_out))) {
@@ -858,6 +871,7 @@ ea_status ea_p2p_open(ea_handle h, const uint8_t* handles, int32_t world) {
 }
 
 ea_status ea_sync(ea_handle h, void* stream) {
+  NvtxRange range("ea_sync");
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   cudaError_t e = cudaSetDevice(h->cfg.device);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
