@@ -331,3 +331,50 @@ def test_p2_adam_zero_gradients_decay():
         xs, ms, vs, c = ea_step_adam(xs, ms, vs, c, [np.zeros(p)] * n, hp, t + 1)
     np.testing.assert_allclose(np.mean(xs, axis=0) - c, (1 - alpha - n * alpha) ** 10 * d0, rtol=1e-9, atol=1e-16)
     np.testing.assert_allclose(sum(xs) + c, total0, rtol=0, atol=1e-13)
+
+
+# ---------------------------------------------------------------- stale center (row f4, reading c28)
+from oracle.ea_oracle import ea_step_stale  # noqa: E402
+
+
+def test_stale_with_equal_centers_is_the_synchronous_step():
+    rng = np.random.default_rng(31)
+    n, p = 3, 100
+    xs, _, c = _rand_state(rng, n, p)
+    ms = [rng.normal(0, 1e-2, p) for _ in range(n)]
+    g = [rng.normal(0, 1e-2, p) for _ in range(n)]
+    hp = Hyper(alpha=0.3, beta=0.9, rho=1.0, lr=0.05, momentum=0.9)
+    a = ea_step(xs, ms, c, g, hp)
+    b = ea_step_stale(xs, ms, c, c, g, hp)
+    for i in range(n):
+        np.testing.assert_array_equal(a[0][i], b[0][i])
+    np.testing.assert_array_equal(a[2], b[2])
+    np.testing.assert_array_equal(b[3], c)
+
+
+@pytest.mark.parametrize("n,alpha,rho", [(2, 0.5, 1.0), (3, 0.2, 0.0), (4, 0.1, 1.0)])
+def test_stale_zero_gradient_state_space_closed_form(n, alpha, rho):
+    """Zero gradients/momentum: (mean x_{t+1}, x~_{t+1}, x~_t) = A (mean x_t, x~_t, x~_{t-1}) with
+    A = [[1-a, 0, a], [b, 1, -b], [0, 1, 0]]  (beta = b), so the trajectory is a matrix power;
+    Sum x + x~ is conserved when beta = N alpha; deviations e_i decay by (1 - alpha)."""
+    rng = np.random.default_rng(32)
+    p, steps = 50, 12
+    beta = n * alpha
+    xs, ms, c = _rand_state(rng, n, p)
+    c = c + rng.normal(0, 1e-3, p)
+    hp = Hyper(alpha=alpha, beta=beta, rho=rho, lr=0.05, momentum=0.9)
+    A = np.array([[1 - alpha, 0.0, alpha], [beta, 1.0, -beta], [0.0, 1.0, 0.0]])
+    s0 = np.stack([np.mean(xs, axis=0), c, c])                 # x~_{-1} := x~_0
+    e0 = [x - np.mean(xs, axis=0) for x in xs]
+    total0 = sum(xs) + c
+    cur_x, cur_m, cur_c, prev_c = xs, ms, c, c
+    for t in range(1, steps + 1):
+        cur_x, cur_m, cur_c, prev_c = ea_step_stale(cur_x, cur_m, cur_c, prev_c, [np.zeros(p)] * n, hp)
+        st = np.linalg.matrix_power(A, t) @ s0
+        np.testing.assert_allclose(np.mean(cur_x, axis=0), st[0], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(cur_c, st[1], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(prev_c, st[2], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(sum(cur_x) + cur_c, total0, rtol=0, atol=1e-12)
+        for i in range(n):
+            np.testing.assert_allclose(cur_x[i] - np.mean(cur_x, axis=0), (1 - alpha) ** t * e0[i], rtol=1e-9,
+                                       atol=1e-15)
