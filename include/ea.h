@@ -64,7 +64,7 @@ extern "C" {
 #define EA_API
 #endif
 
-#define EA_ABI_VERSION 2
+#define EA_ABI_VERSION 3
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
@@ -119,6 +119,10 @@ typedef struct {
                                    that 1-beta2 keeps full precision (0.999f would be off by 1.3e-5) */
   float eps;                    /* Adam(W): denominator epsilon > 0 (torch default 1e-8) */
   int32_t exchange;             /* EA_SPREAD: ea_exchange (ignored for EA_COLOCATED) */
+  int32_t staleness;            /* 0: synchronous center (c3); 1: the replicas see the center one step
+                                   late, x~_{t-1}, as with the paper's asynchronous queues (
+                                   reading c28, row f4).  1 needs EA_COLOCATED and EA_OPT_SGD; the
+                                   library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step). */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;

@@ -24,7 +24,7 @@ VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3}
 OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
-ABI_VERSION = 2
+ABI_VERSION = 3
 
 
 class LibraryNotBuilt(RuntimeError):
@@ -59,6 +59,7 @@ class EAConfig(ctypes.Structure):
         ("beta2", ctypes.c_double),
         ("eps", ctypes.c_float),
         ("exchange", ctypes.c_int32),
+        ("staleness", ctypes.c_int32),
     ]
 
 
@@ -278,7 +279,7 @@ class ElasticAveraging:
                  weight_decay: float = 0.0, nesterov: bool = False, layout: str = "colocated", rank: int = 0,
                  world: int = 1, device: Optional[int] = None, kernel_variant: str = "auto",
                  nccl_id: Optional[bytes] = None, optimizer: str = "sgd", betas=(0.9, 0.999), eps: float = 1e-8,
-                 exchange: str = "nccl"):
+                 exchange: str = "nccl", staleness: int = 0):
         import torch
         self._lib = load_library()
         self.n = int(n_pipelines)
@@ -293,7 +294,7 @@ class ElasticAveraging:
                        1.0 / self.n if alpha is None else float(alpha), float(beta), float(rho), float(lr),
                        float(momentum), float(weight_decay), int(bool(nesterov)), LAYOUTS[layout], int(rank),
                        int(world), self.device, VARIANTS[kernel_variant], OPTIMIZERS[optimizer],
-                       float(betas[0]), float(betas[1]), float(eps), EXCHANGES[exchange])
+                       float(betas[0]), float(betas[1]), float(eps), EXCHANGES[exchange], int(staleness))
         self._cfg = cfg
         self.rank, self.world = int(rank), int(world)
         idbuf = None

@@ -41,6 +41,8 @@ struct ea_ctx {
   std::vector<int64_t> p_pad;   // center capacity
   std::vector<int64_t> stride;  // optimizer-state row stride (floats)
   std::vector<float*> state[2]; // per stage: [replicas][stride]; slot 0 = momentum / Adam m, slot 1 = Adam v
+  std::vector<float*> prev;     // staleness 1: per stage x~_{t-1} (P_s floats)
+  std::vector<char> prev_init;  // per stage: prev holds a value (else x~_{-1} := x~_0 at the first step)
   std::vector<int64_t> steps;   // per-stage step count t, host shadow (enqueue order)
   int64_t* d_steps = nullptr;   // device step counters (authoritative for Adam / P2P; graph-safe)
   ea::StepCoef* d_coef = nullptr;  // device Adam bias corrections of the current step
@@ -190,6 +192,7 @@ void free_ctx(ea_ctx* h) {
   if (h->comm) ncclCommDestroy(h->comm);
   for (auto& slot : h->state)
     for (float* m : slot) if (m) cudaFree(m);
+  for (float* m : h->prev) if (m) cudaFree(m);
   if (h->contrib) cudaFree(h->contrib);
   for (cudaEvent_t ev : h->ev_ag) if (ev) cudaEventDestroy(ev);
   for (cudaEvent_t ev : h->ev_loc) if (ev) cudaEventDestroy(ev);
@@ -258,7 +261,8 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // Adam with N > 6: the replica-loop kernel measured fastest (0.919 of peak at N = 8 vs 0.75 bulk-copy
   // pipeline and 0.73 lane kernel, profiles/r01_adam_nsweep.jsonl)
   const bool adam_wide = opt != EA_OPT_SGD && n > 6 && h->variant == 0;
-  if (n > ea::kMaxFusedN || force_wide || adam_wide) {  // wide N: one launch per stage
+  const bool stale = h->cfg.staleness == 1;
+  if (n > ea::kMaxFusedN || force_wide || adam_wide || stale) {  // replica loop: one launch per stage
     for (int j = 0; j < count; ++j) {
       const int st = stages[j];
       ea::ReplicaTable t;
@@ -270,7 +274,16 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
       }
       ea_status st2 = advance(h, &stages[j], 1, s);
       if (st2 != EA_OK) return st2;
-      e = ea::launch_colocated_wide(t, n, center_ptrs[j], h->p[st], h->hp, opt, h->d_coef + st, h->num_sms, s);
+      float* prev = nullptr;
+      if (stale) {
+        prev = h->prev[st];
+        if (!h->prev_init[st]) {  // x~_{-1} := x~_0 (c28)
+          e = cudaMemcpyAsync(prev, center_ptrs[j], sizeof(float) * h->p[st], cudaMemcpyDeviceToDevice, s);
+          if (e != cudaSuccess) return cuda_fail(h, e, "stale-center init");
+          h->prev_init[st] = 1;
+        }
+      }
+      e = ea::launch_colocated_wide(t, n, center_ptrs[j], prev, h->p[st], h->hp, opt, h->d_coef + st, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
     }
     return EA_OK;
@@ -542,6 +555,11 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   }
   if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
   if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
+  if (c.staleness != 0 && c.staleness != 1) { set_err(nullptr, "staleness must be 0 or 1"); return EA_EINVAL; }
+  if (c.staleness == 1 && (c.layout != EA_COLOCATED || c.optimizer != EA_OPT_SGD)) {
+    set_err(nullptr, "staleness 1 is supported for EA_COLOCATED with EA_OPT_SGD");
+    return EA_EINVAL;
+  }
   if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {
     set_err(nullptr, "peer-memory exchange supports world <= %d", ea::kMaxWorld);
     return EA_EINVAL;
@@ -595,6 +613,16 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
         return r;
       }
       h->state[slot].push_back(m);
+    }
+    if (c.staleness == 1) {
+      float* pv = nullptr;
+      if ((e = cudaMalloc(&pv, sizeof(float) * stride)) != cudaSuccess) {
+        ea_status r = cuda_fail(nullptr, e, "stale-center allocation");
+        free_ctx(h);
+        return r;
+      }
+      h->prev.push_back(pv);
+      h->prev_init.push_back(0);
     }
   }
   if (c.layout == EA_SPREAD) {
@@ -711,6 +739,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
   NvtxRange range("ea_step_many_host");
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
   if (h->cfg.layout != EA_COLOCATED) { set_err(h, "ea_step_many_host needs EA_COLOCATED"); return EA_ESTATE; }
+  if (h->cfg.staleness != 0) { set_err(h, "ea_step_many_host does not support staleness 1"); return EA_ESTATE; }
   if (count < 0 || (count > 0 && (!stages || !replica_ptrs || !host_grad_ptrs || !center_ptrs || !host_center_out))) {
     set_err(h, "ea_step_many_host: bad count or NULL array");
     return EA_EINVAL;
@@ -778,7 +807,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
           t.m[i] = state_ptr(h, 0, st, i) + off;
           t.v[i] = two ? state_ptr(h, 1, st, i) + off : nullptr;
         }
-        e = ea::launch_colocated_wide(t, n, center_ptrs[j] + off, len, h->hp, opt, sc, h->num_sms, s);
+        e = ea::launch_colocated_wide(t, n, center_ptrs[j] + off, nullptr, len, h->hp, opt, sc, h->num_sms, s);
       } else {
         ea::StageBatch bt;
         bt.nstages = 1;

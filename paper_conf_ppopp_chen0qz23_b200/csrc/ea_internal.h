@@ -89,9 +89,10 @@ enum KernelVariant : int {
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s);
 
-// Co-located step for one stage with any N <= kMaxReplicas (N > 8 path).
-cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
-                                  const StepCoef* scp, int num_sms, cudaStream_t s);
+// Co-located step for one stage with any N <= kMaxReplicas (replica loop).  prev != nullptr: stale
+// center (row f4): replicas use prev (x~_{t-1}), center is updated from x~_t, prev <- x~_t.
+cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, float* prev, int64_t p, const Hyper& hp,
+                                  int opt, const StepCoef* scp, int num_sms, cudaStream_t s);
 
 // Spread local step (rows a1-a4 for one replica): updates x and the optimizer
 // state in place and writes r = rho*Delta + beta*(x - x~) into contrib[0..p),

@@ -257,27 +257,34 @@ __global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
 }
 
-// Runtime-N fallback (N > 8): one stage, replicas visited in a loop.
+// Runtime-N replica loop (N > 8, Adam N > 6, the stale center): one stage,
+// replicas visited in a loop.  prev != nullptr selects the stale center of
+// row f4 (reading c28): the replicas use x~_{t-1} (prev) for dilution and
+// gap, the center is updated from x~_t, and prev becomes x~_t.
 template <int U, int OPT>
 __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t, int n, float* __restrict__ center,
-                                                           int64_t nvec, int64_t p, const Hyper hp,
-                                                           const StepCoef* scp) {
+                                                           float* __restrict__ prev, int64_t nvec, int64_t p,
+                                                           const Hyper hp, const StepCoef* scp) {
   const Mem<0> mem;
   const StepCoef sc = load_coef<OPT>(scp);
+  const bool stale = prev != nullptr;
   WaveCursor cur{0, 0};
   int sidx;
   int64_t va, nv;
   while (wave_item_f(1, [&](int) { return nvec; }, (int64_t)kThreads * U, cur, sidx, va, nv)) {
     const int64_t ve = va + nv;
     for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
-      float4 c[U], acc[U];
+      float4 c[U], cu[U], acc[U];
       bool ok[U];
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int64_t v = base + (int64_t)u * kThreads;
         ok[u] = v < ve;
         acc[u] = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (ok[u]) c[u] = mem.ld(center + 4 * v);
+        if (ok[u]) {
+          c[u] = mem.ld(center + 4 * v);
+          cu[u] = stale ? mem.ld(prev + 4 * v) : c[u];   // the center the replicas see
+        }
       }
       for (int i = 0; i < n; ++i) {
         float4 x[U], g[U], m[U], w[U];
@@ -295,7 +302,7 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
         for (int u = 0; u < U; ++u) {
           if (!ok[u]) continue;
           const int64_t v = base + (int64_t)u * kThreads;
-          add4(acc[u], ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc));
+          add4(acc[u], ea_vec<OPT>(x[u], g[u], m[u], w[u], cu[u], hp, sc));
           mem.st(t.x[i] + 4 * v, x[u]);
           mem.st(t.m[i] + 4 * v, m[u]);
           if (OPT != kOptSGD) mem.st(t.v[i] + 4 * v, w[u]);
@@ -304,22 +311,27 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int64_t v = base + (int64_t)u * kThreads;
-        if (ok[u]) mem.st(center + 4 * v, center_apply(c[u], acc[u], hp.inv_n));
+        if (ok[u]) {
+          mem.st(center + 4 * v, center_apply(c[u], acc[u], hp.inv_n));
+          if (stale) mem.st(prev + 4 * v, c[u]);
+        }
       }
     }
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
     for (int64_t j = 4 * nvec; j < p; ++j) {
       const float c = center[j];
+      const float cused = stale ? prev[j] : c;
       float acc = 0.f;
       for (int i = 0; i < n; ++i) {
         float x = t.x[i][j], m = t.m[i][j], v = OPT == kOptSGD ? 0.f : t.v[i][j];
-        acc += ea_elem<OPT>(x, t.g[i][j], m, v, c, hp, sc);
+        acc += ea_elem<OPT>(x, t.g[i][j], m, v, cused, hp, sc);
         t.x[i][j] = x;
         t.m[i][j] = m;
         if (OPT != kOptSGD) t.v[i][j] = v;
       }
       center[j] = fmaf(acc, hp.inv_n, c);
+      if (stale) prev[j] = c;
     }
   }
 }
@@ -841,13 +853,13 @@ cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant,
 }
 
 template <int OPT>
-cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp,
+cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, float* prev, int64_t p, const Hyper& hp,
                             const StepCoef* sc, int num_sms, cudaStream_t s) {
   constexpr int U = 2;
   const int64_t nvec = p / 4;
   auto k = colocated_wide<U, OPT>;
   const int64_t units = (nvec + kThreads * U - 1) / (kThreads * U);
-  k<<<persistent_grid(k, units < 1 ? 1 : units, num_sms), kThreads, 0, s>>>(t, n, center, nvec, p, hp, sc);
+  k<<<persistent_grid(k, units < 1 ? 1 : units, num_sms), kThreads, 0, s>>>(t, n, center, prev, nvec, p, hp, sc);
   return cudaGetLastError();
 }
 
@@ -910,12 +922,12 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   }
 }
 
-cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, int64_t p, const Hyper& hp, int opt,
-                                  const StepCoef* sc, int num_sms, cudaStream_t s) {
+cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, float* prev, int64_t p, const Hyper& hp,
+                                  int opt, const StepCoef* sc, int num_sms, cudaStream_t s) {
   if (p <= 0) return cudaSuccess;
-  if (opt == kOptAdam) return launch_wide_opt<kOptAdam>(t, n, center, p, hp, sc, num_sms, s);
-  if (opt == kOptAdamW) return launch_wide_opt<kOptAdamW>(t, n, center, p, hp, sc, num_sms, s);
-  return launch_wide_opt<kOptSGD>(t, n, center, p, hp, sc, num_sms, s);
+  if (opt == kOptAdam) return launch_wide_opt<kOptAdam>(t, n, center, prev, p, hp, sc, num_sms, s);
+  if (opt == kOptAdamW) return launch_wide_opt<kOptAdamW>(t, n, center, prev, p, hp, sc, num_sms, s);
+  return launch_wide_opt<kOptSGD>(t, n, center, prev, p, hp, sc, num_sms, s);
 }
 
 cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, const float* center, float* contrib,

@@ -12,7 +12,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from oracle.ea_oracle import Hyper, ea_step, ea_step_adam
+from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_stale
 from paper_conf_ppopp_chen0qz23_b200 import synth
 
 TOL = 1e-5
@@ -53,17 +53,21 @@ def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nes
 class OracleStage:
     """float64 oracle state of one stage (optimizer 'sgd' | 'adam' | 'adamw')."""
 
-    def __init__(self, reps, center, optimizer="sgd"):
+    def __init__(self, reps, center, optimizer="sgd", staleness=0):
         self.xs = [np.asarray(x, dtype=np.float64) for x in reps]
         self.ms = [np.zeros_like(self.xs[0]) for _ in reps]
         self.vs = [np.zeros_like(self.xs[0]) for _ in reps]
         self.c = np.asarray(center, dtype=np.float64)
+        self.c_prev = self.c.copy()        # x~_{-1} := x~_0 (c28)
         self.opt = optimizer
+        self.staleness = staleness
         self.t = 0
 
     def step(self, grads, hp):
         self.t += 1
-        if self.opt == "sgd":
+        if self.staleness == 1:
+            self.xs, self.ms, self.c, self.c_prev = ea_step_stale(self.xs, self.ms, self.c, self.c_prev, grads, hp)
+        elif self.opt == "sgd":
             self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)
         else:
             self.xs, self.ms, self.vs, self.c = ea_step_adam(self.xs, self.ms, self.vs, self.c, grads, hp, self.t,

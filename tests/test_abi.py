@@ -52,10 +52,10 @@ def test_abi_version(lib):
 
 
 def test_config_struct_layout_matches_header():
-    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, [pad], 2 doubles, 1 float, [pad]  (x86-64 alignment)
-    assert ctypes.sizeof(binding.EAConfig) == 96
+    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, [pad], 2 doubles, float, 2 int32, [pad] (x86-64)
+    assert ctypes.sizeof(binding.EAConfig) == 104
     assert binding.EAConfig.beta1.offset == 72 and binding.EAConfig.eps.offset == 88
-    assert binding.EAConfig.exchange.offset == 92
+    assert binding.EAConfig.exchange.offset == 92 and binding.EAConfig.staleness.offset == 96
     assert binding.EAConfig.stage_params.offset == 8
     assert ctypes.sizeof(binding.EAOp) == 8
 
@@ -64,7 +64,7 @@ def _cfg(**kw):
     sp = (ctypes.c_int64 * 2)(1000, 1001)
     base = dict(n_pipelines=2, n_stages=2, stage_params=sp, alpha=0.5, beta=0.0, rho=1.0, lr=0.05, momentum=0.9,
                 weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0, optimizer=0,
-                beta1=0.9, beta2=0.999, eps=1e-8, exchange=0)
+                beta1=0.9, beta2=0.999, eps=1e-8, exchange=0, staleness=0)
     base.update(kw)
     c = binding.EAConfig(**base)
     c._keep = sp
@@ -88,6 +88,9 @@ def _cfg(**kw):
     (dict(lr=float("nan")), "finite"),
     (dict(optimizer=3), "optimizer"),
     (dict(exchange=5), "exchange"),
+    (dict(staleness=2), "staleness"),
+    (dict(staleness=1, optimizer=1), "staleness 1"),
+    (dict(staleness=1, layout=1, world=2, rank=0), "staleness 1"),
     (dict(layout=1, world=17, n_pipelines=17, rank=0, exchange=1), "world <="),
     (dict(optimizer=1, beta1=1.0), "betas"),
     (dict(optimizer=2, beta2=-0.5), "betas"),

@@ -25,7 +25,7 @@ VARIANTS = ("regloop", "laneshfl", "bulkpipe")  # Adam(W): lane kernel whatever 
 
 
 def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nesterov=False, wd=0.0, lr=synth.LR,
-                   momentum=synth.MOMENTUM, seed=0, many=False, optimizer="sgd"):
+                   momentum=synth.MOMENTUM, seed=0, many=False, optimizer="sgd", staleness=0):
     hp = hyper(n, mode, alpha=alpha, lr=lr, momentum=momentum, wd=wd, nesterov=nesterov)
     dev = torch.device("cuda:0")
     oracle, gstreams = [], []
@@ -33,14 +33,15 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
     handles = {}
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + 97 * seed + s)
-        oracle.append(OracleStage(reps, c, optimizer))
+        oracle.append(OracleStage(reps, c, optimizer, staleness))
         gstreams.append(synth.GradStream(n, p, seed=synth.GRAD_SEED + 97 * seed + s))
         for v in variants:
             gpu[v].append(([torch.from_numpy(x).to(dev) for x in reps], torch.from_numpy(c).to(dev)))
     for v in variants:
         handles[v] = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr,
                                       momentum=hp.momentum, weight_decay=hp.weight_decay, nesterov=hp.nesterov,
-                                      kernel_variant=v, optimizer=optimizer, betas=(hp.beta1, hp.beta2), eps=hp.eps)
+                                      kernel_variant=v, optimizer=optimizer, betas=(hp.beta1, hp.beta2), eps=hp.eps,
+                                      staleness=staleness)
     gbuf = [[torch.empty(p, device=dev) for _ in range(n)] for p in sizes]
     order = list(reversed(range(len(sizes))))
     for t in range(steps):
@@ -134,6 +135,19 @@ def test_adam_bulk_pipeline(optimizer, n):
     sizes = [100_003, 7, 4096]
     _run_colocated(n, sizes, 12, "combined", optimizer=optimizer, lr=1e-3, wd=1e-2, many=True,
                    variants=("bulkpipe",))
+
+
+# ------------------------------------------------------------------ stale center (row f4)
+@pytest.mark.parametrize("n", [1, 2, 4, 8, 12])
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_stale_center(n, mode):
+    """staleness 1 (reading c28): replicas dilute with x~_{t-1}, the center moves from x~_t."""
+    _run_colocated(n, [100_003, 7, 4096], 40, mode, variants=("auto",), staleness=1, many=True)
+    _run_colocated(n, [65_537], 20, mode, variants=("auto",), staleness=1, nesterov=True, wd=1e-3)
+
+
+def test_stale_center_c1_100_steps():
+    _run_colocated(2, [1_000_000, 1_000_003], 100, "combined", variants=("auto",), staleness=1, many=True)
 
 
 @pytest.mark.parametrize("n,optimizer", [(33, "sgd"), (64, "sgd"), (64, "adamw")])
