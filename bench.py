@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
     ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw"), default="sgd",
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
+    ap.add_argument("--staleness", type=int, choices=(0, 1), default=0,
+                    help="1: replicas see the center one step late (row f4; co-located SGD)")
     ap.add_argument("--exchange", choices=("nccl", "p2p"), default="nccl",
                     help="N>1 spread exchange: NCCL RS/AG or the fused peer-memory kernel")
     ap.add_argument("--no-graph", action="store_true",
@@ -145,8 +147,10 @@ def workload_key(gpus: int, override):
 
 
 # ----------------------------------------------------------------------------- our arm
-def kernel_name(variant, optimizer, n):
+def kernel_name(variant, optimizer, n, staleness=0):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
+    if staleness:
+        return "colocated_wide<stale>"
     if n > 8 or (optimizer != "sgd" and n > 6 and variant == "auto"):
         name = "colocated_wide"
     elif optimizer != "sgd":
@@ -164,7 +168,7 @@ def colocated_launches(n, k, args, batched):
     """Our kernels per co-located step: the fused kernel(s) plus, for Adam, the
     step-counter kernel that precedes each launch."""
     adam = args.optimizer != "sgd"
-    per_stage = n > 8 or not batched or (adam and n > 6 and args.variant == "auto")
+    per_stage = n > 8 or not batched or (adam and n > 6 and args.variant == "auto") or args.staleness
     launches = k if per_stage else (k + 7) // 8
     return launches * (2 if adam else 1)
 
@@ -219,7 +223,8 @@ def run_ours(args, rank, world, local):
             state.append((reps, grads, cc))
     else:
         h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
-                             device=local, kernel_variant=args.variant, optimizer=args.optimizer)
+                             device=local, kernel_variant=args.variant, optimizer=args.optimizer,
+                             staleness=args.staleness)
         state = [synth.device_state(n, p, dev, seed=s) for s, p in enumerate(sizes)]
         state = [(reps, grads, c) for (reps, c, grads) in state]
     order = parallel.stage_order(len(sizes))
@@ -305,7 +310,7 @@ def run_ours(args, rank, world, local):
                      "kernel": args.variant,
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
     if not spread:
-        step_bytes = sum(bytes_colocated(n, p, args.optimizer) for p in sizes)
+        step_bytes = sum(bytes_colocated(n, p, args.optimizer) + 8 * p * args.staleness for p in sizes)
         launches_per_step = 1 if batched else len(sizes)
         kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(launches_per_step)]
         # per launch (batched: all stages; per-stage: averaged over the equal-sized stages)
@@ -315,7 +320,7 @@ def run_ours(args, rank, world, local):
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
-                           "kernel": kernel_name(args.variant, args.optimizer, n),
+                           "kernel": kernel_name(args.variant, args.optimizer, n, args.staleness),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         out["gpu_launches"] = args.steps * colocated_launches(n, len(sizes), args, batched)
