@@ -529,7 +529,7 @@ constexpr int default_bulk_tile() {
   return A == 3 ? ((N == 4 || N == 5) ? 128 : 256) : ((A * N + 1) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128);
 }
 
-constexpr int kMaxBulkStages = 8;  // ring depth cap
+constexpr int kMaxBulkStages = 6;  // ring depth cap (8 measured slower: profiles/r01_bulk_n4_tiles.jsonl)
 
 // A = streams per replica in the slot: 3 (x, g, m) for SGD, 4 (x, g, m, v) for Adam.
 template <int N, int TILE, int A>
@@ -826,12 +826,6 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
   if constexpr (HINT == 0) {
     switch (bulk_tile()) {
       case 64: return launch_bulkpipe_t<N, HINT, OPT, 64>(b, hp, num_sms, s);
-      case 96: if constexpr (N == 4 && OPT == kOptSGD) return launch_bulkpipe_t<N, HINT, OPT, 96>(b, hp, num_sms, s);
-               break;
-      case 160: if constexpr (N == 4 && OPT == kOptSGD) return launch_bulkpipe_t<N, HINT, OPT, 160>(b, hp, num_sms, s);
-                break;
-      case 192: if constexpr (N == 4 && OPT == kOptSGD) return launch_bulkpipe_t<N, HINT, OPT, 192>(b, hp, num_sms, s);
-                break;
       case 128: return launch_bulkpipe_t<N, HINT, OPT, 128>(b, hp, num_sms, s);
       case 256:
         if constexpr ((A * N + 1) * 256 * 16 * 2 <= 200 * 1024) return launch_bulkpipe_t<N, HINT, OPT, 256>(b, hp, num_sms, s);
