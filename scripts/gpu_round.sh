@@ -24,4 +24,7 @@ timeout 900 ncu --set full --clock-control none --import-source on -k regex:colo
     python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full_default.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:colocated -s 5 -c 1 -o gpurun_out/prof_adam -f \
     python bench.py --steps 3 --warmup 3 --no-e2e --no-cpu-baseline --optimizer adam > gpurun_out/ncu_full_adam.log 2>&1
+
+# large-model points on one GPU (co-located)
+timeout 900 python bench.py --config C5 --n 2 --no-e2e --no-cpu-baseline --steps 50 > gpurun_out/bench_c5n2.json 2>> gpurun_out/bench.err
 echo done
