@@ -342,8 +342,8 @@ def run_ours(args, rank, world, local):
         out["copy_gbs_same_box"] = same_box_copy_gbs(dev)
     if not spread and not args.no_e2e:
         out["e2e"] = e2e_colocated(h, state, sizes, n, args, stream, dev, order)
-    elif spread:
-        out["e2e"] = None
+    elif spread and not args.no_e2e:
+        out["e2e"] = e2e_spread(h, state, sizes, args, stream, dev, order, rank, world)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         out["cpu_baseline"] = cpu_baseline(cfg, n, seconds=args.cpu_seconds)
     h.close()
@@ -408,6 +408,49 @@ def e2e_colocated(h, state, sizes, n, args, stream, dev, order):
             "h2d_bytes_per_step": 4 * n * sum(sizes), "d2h_bytes_per_step": 4 * sum(sizes),
             "path": "ea_step_many_host: pinned host grads -> device (chunked, copy stream), fused kernel per chunk, "
                     "center chunks -> pinned host (second copy stream)"}
+
+
+def e2e_spread(h, state, sizes, args, stream, dev, order, rank, world):
+    """Spread layout end to end through the public API: every step each rank
+    copies its replica's gradients of every stage from pinned HOST memory
+    (non_blocking, on the step stream), runs ea_step per stage (local kernel +
+    exchange on the library side stream), joins the exchange (ea_sync) and
+    reads its owned center shard of every stage back to pinned host memory.
+    Timed with CUDA events on the step stream, max over ranks."""
+    import torch
+    import torch.distributed as dist
+    host_g = [state[s][1][0].cpu().pin_memory() for s in range(len(sizes))]
+    shard = [h.shard_elems(s) for s in range(len(sizes))]
+    host_c = [torch.empty(shard[s], dtype=torch.float32).pin_memory() for s in range(len(sizes))]
+
+    def step():
+        for s in order:
+            reps, grads, cc = state[s]
+            grads[0].copy_(host_g[s], non_blocking=True)
+            h.step(s, reps, grads, cc, stream=stream)
+        h.sync(stream)
+        for s in order:
+            cc = state[s][2]
+            host_c[s].copy_(cc[rank * shard[s]:(rank + 1) * shard[s]], non_blocking=True)
+
+    for _ in range(3):
+        step()
+    torch.cuda.synchronize()
+    dist.barrier()
+    t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    t0.record(stream)
+    for _ in range(args.e2e_steps):
+        step()
+    t1.record(stream)
+    torch.cuda.synchronize()
+    ms = t0.elapsed_time(t1) / args.e2e_steps
+    tt = torch.tensor([ms], device=dev)
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    ms = float(tt.item())
+    return {"value": world * sum(sizes) / (ms * 1e-3), "unit": UNIT, "ms_per_step": ms,
+            "h2d_bytes_per_step": 4 * world * sum(sizes), "d2h_bytes_per_step": 4 * world * sum(shard),
+            "path": "per rank: pinned host grads -> device (non_blocking copy on the step stream), ea_step per "
+                    "stage, ea_sync, owned center shards -> pinned host; bytes summed over ranks"}
 
 
 # ----------------------------------------------------------------------------- oracle (CPU) legs

@@ -1,0 +1,64 @@
+"""bench.py's JSON contract, checked on CPU: the reference arm (the float64
+oracle on host cores) prints exactly one JSON line with the driver's keys,
+and under torchrun only rank 0 prints.  Also the algorithmic byte counts the
+roofline divides by ((20N+8)P co-located SGD, 28P spread)."""
+import json
+import os
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+import bench  # noqa: E402
+
+KEYS = {"metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+        "vs_baseline", "dtype", "data", "config", "impl", "cpu_baseline", "e2e", "gpu_launches"}
+
+
+def _json_lines(out: str):
+    return [json.loads(l) for l in out.splitlines() if l.strip().startswith("{")]
+
+
+def test_reference_arm_one_json_line():
+    r = subprocess.run([sys.executable, "bench.py", "--impl", "reference", "--steps", "3", "--warmup", "3"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr
+    lines = [l for l in r.stdout.splitlines() if l.strip()]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert KEYS <= set(d), KEYS - set(d)
+    assert d["impl"] == "reference" and d["unit"] == bench.UNIT and d["metric"] == bench.METRIC
+    assert d["config"]["workload"].startswith("C2")
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["value"] == d["value"]
+    assert d["value"] > 0 and d["steps"] == 3
+
+
+def test_reference_arm_under_torchrun_rank0_only():
+    r = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29617", "bench.py", "--impl", "reference",
+                        "--gpus", "2", "--steps", "3", "--warmup", "3"],
+                       cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = _json_lines(r.stdout)
+    assert len(lines) == 1, r.stdout
+    assert lines[0]["n_gpus"] == 2 and lines[0]["config"]["n_pipelines"] == 2
+
+
+@pytest.mark.parametrize("n", [1, 2, 4, 8, 12])
+def test_algorithmic_bytes(n):
+    p = 1000
+    # read x~ + N x (x, g, m); write N x (x, m) + x~
+    assert bench.bytes_colocated(n, p) == 4 * p * ((1 + 3 * n) + (2 * n + 1))
+    # Adam: + v read and written per replica
+    assert bench.bytes_colocated(n, p, "adam") == 4 * p * ((1 + 4 * n) + (3 * n + 1))
+    # spread: read x, g, m, x~; write x, m, r
+    assert bench.bytes_spread_local(p) == 4 * p * 7
+    assert bench.bytes_spread_local(p, "adam") == 4 * p * 9
+
+
+def test_default_workload_is_configs1():
+    assert bench.workload_key(1, None) == "C2"
+    assert bench.workload_key(8, None) == "C4"
