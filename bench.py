@@ -278,7 +278,7 @@ def run_ours(args, rank, world, local):
         dist.barrier()
     # per-launch events for the dominant kernel (co-located: every ea_step is one kernel)
     ev = None
-    if not spread:
+    if not spread or args.exchange == "nccl":   # spread + NCCL: events bracket each stage's local kernel
         ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
                for _ in (range(1) if batched else sizes)] for _ in range(args.steps)]
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -331,10 +331,29 @@ def run_ours(args, rank, world, local):
         nv_bytes = sum(2 * (n - 1) / n * 4 * h.center_capacity(s) for s in range(len(sizes)))
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         nv_gbs = nv_bytes / (ms * 1e-3) / 1e9
-        out["roofline"] = {"bound": "nvlink", "achieved": nv_gbs, "peak": NVLINK_PEAK_GBS, "unit": "GB/s",
-                           "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None,
-                           "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / "
-                                   "step time; peak = measured peer copy per direction"}
+        nvlink = {"bound": "nvlink", "achieved": nv_gbs, "peak": NVLINK_PEAK_GBS, "unit": "GB/s",
+                  "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None,
+                  "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / "
+                          "step time; peak = measured peer copy per direction"}
+        local = None
+        if ev is not None:
+            # the local kernel (rows a1-a4) runs on the caller's stream between each stage's events;
+            # the exchange runs on the library's side stream, outside them
+            kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(len(sizes))]
+            avg_ms = sum(kern_ms) / len(kern_ms)
+            per_launch_bytes = step_bytes / len(sizes)
+            achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
+            local = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                     "traffic": None, "kernel": "spread_bulkpipe" + ("" if args.optimizer == "sgd" else
+                                                                     "<" + args.optimizer + ">"),
+                     "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
+                     "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
+        if world == 1 and local is not None:
+            out["roofline"] = local     # no NVLink traffic at world 1: the local kernel is the bound
+        else:
+            out["roofline"] = nvlink
+            if local is not None:
+                out["local_kernel_roofline"] = local
         per_stage = 2 if args.exchange == "p2p" else (2 if args.optimizer == "sgd" else 3)
         out["gpu_launches"] = args.steps * per_stage * len(sizes)   # ours only (NCCL kernels excluded)
     out["clocks"] = clk.summary()

@@ -541,8 +541,26 @@ struct BulkGeom {
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
 
-template <int N, int HINT, int OPT, int TILE>
-__global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
+// Scalar tail of the spread bulk pipeline (one thread): elements [4*(p/4), p) and the zero padding
+// [p, p_pad) of the contribution (reading c18: zero padding is a fixed point of the exchange).
+template <int OPT>
+__device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
+  const StepCoef sc = load_coef<OPT>(st.scp);
+  for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
+    float x = st.x[0][j], m = st.m[0][j], v = OPT == kOptSGD ? 0.f : st.v[0][j];
+    contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
+    st.x[0][j] = x;
+    st.m[0][j] = m;
+    if (OPT != kOptSGD) st.v[0][j] = v;
+  }
+  for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
+}
+
+// SPREAD = false: co-located stages (x~ updated in place).  SPREAD = true: the spread layout's local
+// step (N = 1, one stage): x~ is only read and the contribution r goes to `contrib` (rows a1-a4).
+template <int N, int HINT, int OPT, int TILE, bool SPREAD>
+__device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& hp, float* __restrict__ contrib,
+                                              int64_t p_pad) {
   constexpr int A = OPT == kOptSGD ? 3 : 4;
   using G = BulkGeom<N, TILE, A>;
   constexpr int T = G::kTile, S = G::kStages;
@@ -613,15 +631,35 @@ __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const Stag
           mem.st(st.m[i] + 4 * v, m);
           if (A == 4) mem.st(st.v[i] + 4 * v, w);
         }
-        mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
+        if constexpr (SPREAD)
+          mem.st(contrib + 4 * v, acc);
+        else
+          mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
       }
       // all consumer warps are done reading the slot, then one release-arrive hands it back
       asm volatile("bar.sync 1, %0;" ::"n"(32 * kBulkConsumerWarps) : "memory");
       if (threadIdx.x == 0) mbar_arrive(&empty[slot]);
     }
-    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+    if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
+      if constexpr (SPREAD)
+        spread_tail<OPT>(b.st[0], contrib, p_pad, hp);
+      else
+        for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+    }
   }
+}
+
+template <int N, int HINT, int OPT, int TILE>
+__global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
+  bulkpipe_body<N, HINT, OPT, TILE, false>(b, hp, nullptr, 0);
+}
+
+// Spread local step (one replica) through the same bulk-copy pipeline: 4 input streams (x, g, state, x~;
+// + v for Adam) arrive by cp.async.bulk into the smem ring; x, state and r leave by 128-bit stores.
+template <int OPT, int TILE>
+__global__ void __launch_bounds__(kBulkThreads, 1) spread_bulkpipe(const StageBatch b, const Hyper hp,
+                                                                   float* __restrict__ contrib, int64_t p_pad) {
+  bulkpipe_body<1, 0, OPT, TILE, true>(b, hp, contrib, p_pad);
 }
 
 // ============================================================================
@@ -865,10 +903,50 @@ cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, float* 
   return cudaGetLastError();
 }
 
+// Spread local kernel knob (measurement): AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel
+// (spread_local); default: the bulk-copy pipeline (spread_bulkpipe).
+int spread_reg() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_SPREAD_KERNEL");
+    return (e && e[0] == 'r') ? 1 : 0;
+  }();
+  return v;
+}
+
+template <int OPT>
+cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
+                               cudaStream_t s) {
+  constexpr int A = OPT == kOptSGD ? 3 : 4;
+  constexpr int TILE = default_bulk_tile<1, A>();
+  using G = BulkGeom<1, TILE, A>;
+  auto k = spread_bulkpipe<OPT, TILE>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
+  if (e != cudaSuccess) return e;
+  StageBatch b;
+  b.nstages = 1;
+  StageRefs& r = b.st[0];
+  for (int i = 0; i < kMaxFusedN; ++i) {
+    r.x[i] = i == 0 ? x : nullptr;
+    r.g[i] = i == 0 ? g : nullptr;
+    r.m[i] = i == 0 ? m : nullptr;
+    r.v[i] = i == 0 ? v : nullptr;
+  }
+  r.c = const_cast<float*>(center);  // read only (SPREAD)
+  r.p = p;
+  r.scp = sc;
+  int64_t grid = num_sms;
+  const int64_t units = (p / 4 + TILE - 1) / TILE;
+  if (grid > units) grid = units < 1 ? 1 : units;
+  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp, contrib, p_pad);
+  return cudaGetLastError();
+}
+
 template <int OPT>
 cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
                                     float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
+  if (!spread_reg()) return launch_spread_bulk<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   constexpr int U = OPT == kOptSGD ? 4 : 2;
   const int64_t nvec = p / 4;
   auto k = spread_local<U, OPT>;
