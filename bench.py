@@ -318,8 +318,11 @@ def run_ours(args, rank, world, local):
         avg_ms = sum(kern_ms) / len(kern_ms)
         achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
+        q = sorted(kern_ms)
+        pct = {f"p{k}": q[min(len(q) - 1, len(q) * k // 100)] for k in (10, 50, 90)}
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
+                           "launch_ms_pct": pct,
                            "kernel": kernel_name(args.variant, args.optimizer, n, args.staleness),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                            "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
@@ -497,9 +500,38 @@ def cpu_baseline(cfg, n, seconds=10.0):
         el = time.perf_counter() - t0
         if el >= seconds:
             break
-    return {"value": n * p * steps / el, "unit": UNIT, "cores": 1, "kind": "oracle",
-            "sample": f"{steps} oracle steps of one {p}-element stage x N={n} (float64 numpy, 1 thread), "
-                      f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0))}
+    out = {"value": n * p * steps / el, "unit": UNIT, "cores": 1, "kind": "oracle",
+           "sample": f"{steps} oracle steps of one {p}-element stage x N={n} (float64 numpy, 1 thread), "
+                     f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0))}
+    out["all_cores"] = cpu_baseline_all_cores(xs, ms, c, g, hp, seconds=seconds / 2)
+    return out
+
+
+def cpu_baseline_all_cores(xs, ms, c, g, hp, seconds=5.0):
+    """The same oracle step, unchanged, called on contiguous element ranges by a
+    thread pool with one worker per host core (the update is elementwise over j,
+    and numpy's ufuncs release the GIL) -- SURVEY §8(d)'s all-core variant."""
+    from concurrent.futures import ThreadPoolExecutor
+    from oracle.ea_oracle import ea_step
+    cores = len(os.sched_getaffinity(0))
+    p, n = len(c), len(xs)
+    bounds = [(p * k // cores, p * (k + 1) // cores) for k in range(cores)]
+
+    def part(b):
+        a, e = b
+        return ea_step([x[a:e] for x in xs], [m[a:e] for m in ms], c[a:e], [gi[a:e] for gi in g], hp)
+
+    steps, t0 = 0, time.perf_counter()
+    with ThreadPoolExecutor(max_workers=cores) as pool:
+        while True:
+            list(pool.map(part, bounds))
+            steps += 1
+            el = time.perf_counter() - t0
+            if el >= seconds:
+                break
+    return {"value": n * p * steps / el, "unit": UNIT, "cores": cores, "kind": "oracle",
+            "sample": f"{steps} oracle steps of one {p}-element stage x N={n}, split into {cores} element ranges "
+                      f"on {cores} threads (float64 numpy), {el:.1f} s"}
 
 
 def run_reference(args, rank, world):
