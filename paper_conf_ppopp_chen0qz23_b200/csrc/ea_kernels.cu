@@ -205,11 +205,12 @@ __device__ __forceinline__ bool wave_item(const StageBatch& b, int64_t C, WaveCu
 // registers, reduces the N contributions in registers and writes x_i, m_i
 // and x~ once.  Work unit: kThreads*U float4 per block, scheduled by wave_item.
 // ============================================================================
-template <int N, int U, int HINT>
+template <int N, int U, int HINT, int OPT>
 __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, int64_t ve, const Hyper& hp,
-                                              const Mem<HINT>& mem) {
+                                              const Mem<HINT>& mem, const StepCoef& sc) {
+  constexpr bool kTwo = OPT != kOptSGD;  // Adam(W): second moment v
   for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
-    float4 c[U], x[N][U], g[N][U], m[N][U];
+    float4 c[U], x[N][U], g[N][U], m[N][U], w[kTwo ? N : 1][U];
     bool ok[U];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -226,6 +227,7 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
           x[i][u] = mem.ld(st.x[i] + 4 * v);
           g[i][u] = mem.ld_ro(st.g[i] + 4 * v);
           m[i][u] = mem.ld(st.m[i] + 4 * v);
+          if constexpr (kTwo) w[i][u] = mem.ld(st.v[i] + 4 * v);
         }
       }
     }
@@ -236,25 +238,35 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
       float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
 #pragma unroll
       for (int i = 0; i < N; ++i) {
-        float4 unused;
-        add4(acc, ea_vec<kOptSGD>(x[i][u], g[i][u], m[i][u], unused, c[u], hp, StepCoef{0.f, 0.f}));
+        float4 unused = make_float4(0.f, 0.f, 0.f, 0.f);
+        float4& wv = kTwo ? w[kTwo ? i : 0][u] : unused;
+        add4(acc, ea_vec<OPT>(x[i][u], g[i][u], m[i][u], wv, c[u], hp, sc));
         mem.st(st.x[i] + 4 * v, x[i][u]);
         mem.st(st.m[i] + 4 * v, m[i][u]);
+        if constexpr (kTwo) mem.st(st.v[i] + 4 * v, wv);
       }
       mem.st(st.c + 4 * v, center_apply(c[u], acc, hp.inv_n));
     }
   }
 }
 
-template <int N, int U, int HINT>
+// SGD: __launch_bounds__(256) (<= 255 registers; 2+ CTAs/SM at N <= 4).  Adam(W) keeps (4N+1) float4 per
+// thread in flight (N = 8: 132 registers of loads), one 256-thread CTA per SM.
+template <int N, int U, int HINT, int OPT>
 __global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b, const Hyper hp) {
   const Mem<HINT> mem;
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
+  if (OPT != kOptSGD) {
+    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+    __syncthreads();
+  }
   WaveCursor cur{0, 0};
   int s;
   int64_t v0, nv;
-  while (wave_item(b, (int64_t)kThreads * U, cur, s, v0, nv)) regloop_range<N, U, HINT>(b.st[s], v0, v0 + nv, hp, mem);
+  while (wave_item(b, (int64_t)kThreads * U, cur, s, v0, nv))
+    regloop_range<N, U, HINT, OPT>(b.st[s], v0, v0 + nv, hp, mem, OPT == kOptSGD ? StepCoef{0.f, 0.f} : s_coef[s]);
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, kOptSGD>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
 
 // Runtime-N replica loop (N > 8, Adam N > 6, the stale center): one stage,
@@ -775,9 +787,9 @@ int64_t units_of(const StageBatch& b, int64_t chunk) {
   return units < 1 ? 1 : units;
 }
 
-template <int N, int HINT, int U>
+template <int N, int HINT, int U, int OPT = kOptSGD>
 cudaError_t launch_regloop_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  auto k = colocated_regloop<N, U, HINT>;
+  auto k = colocated_regloop<N, U, HINT, OPT>;
   k<<<persistent_grid(k, units_of(b, kThreads * U), num_sms), kThreads, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
@@ -879,6 +891,9 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
 
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (opt != kOptSGD && variant == kVariantRegLoop)
+    return opt == kOptAdam ? launch_regloop_u<N, 0, 1, kOptAdam>(b, hp, num_sms, s)
+                           : launch_regloop_u<N, 0, 1, kOptAdamW>(b, hp, num_sms, s);
   if (opt != kOptSGD && variant == kVariantBulkPipe)
     return opt == kOptAdam ? launch_bulkpipe<N, 0, kOptAdam>(b, hp, num_sms, s)
                            : launch_bulkpipe<N, 0, kOptAdamW>(b, hp, num_sms, s);

@@ -137,6 +137,16 @@ def test_adam_bulk_pipeline(optimizer, n):
                    variants=("bulkpipe",))
 
 
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+@pytest.mark.parametrize("n", [1, 2, 3, 5, 7, 8])
+def test_adam_register_loop(optimizer, n):
+    """Adam/AdamW through the register-loop kernel (all (4N+1) float4 loads of a thread hoisted)."""
+    sizes = [100_003, 7, 4096, 1_000_001]
+    _run_colocated(n, sizes, 12, "combined", optimizer=optimizer, lr=1e-3, wd=1e-2, many=True,
+                   variants=("regloop",))
+    _run_colocated(n, sizes[:1], 8, "paper", optimizer=optimizer, lr=1e-3, variants=("regloop",))
+
+
 # ------------------------------------------------------------------ stale center (row f4)
 @pytest.mark.parametrize("n", [1, 2, 4, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
