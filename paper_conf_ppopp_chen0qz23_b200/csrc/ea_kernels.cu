@@ -251,9 +251,17 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
 }
 
 // SGD: __launch_bounds__(256) (<= 255 registers; 2+ CTAs/SM at N <= 4).  Adam(W) keeps (4N+1) float4 per
-// thread in flight (N = 8: 132 registers of loads), one 256-thread CTA per SM.
+// thread in flight (N = 8: 132 registers of loads).  Bytes in flight per SM = resident threads x loads per
+// thread, so Adam at N = 5 asks for 2 CTAs/SM (<= 128 registers, 32 B spilled) instead of 1 CTA at 137 (N = 6 would
+// spill 120 B).
+template <int N, int OPT>
+constexpr int regloop_min_blocks() {
+  return (OPT != kOptSGD && N == 5) ? 2 : 0;  // 0: no minimum (ptxas default heuristics)
+}
+
 template <int N, int U, int HINT, int OPT>
-__global__ void __launch_bounds__(kThreads) colocated_regloop(const StageBatch b, const Hyper hp) {
+__global__ void __launch_bounds__(kThreads, regloop_min_blocks<N, OPT>()) colocated_regloop(const StageBatch b,
+                                                                                            const Hyper hp) {
   const Mem<HINT> mem;
   __shared__ StepCoef s_coef[kMaxLaunchStages];
   if (OPT != kOptSGD) {
@@ -572,7 +580,7 @@ __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, 
 // step (N = 1, one stage): x~ is only read and the contribution r goes to `contrib` (rows a1-a4).
 template <int N, int HINT, int OPT, int TILE, bool SPREAD>
 __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& hp, float* __restrict__ contrib,
-                                              int64_t p_pad) {
+                                              int64_t p_pad, int issue_lanes) {
   constexpr int A = OPT == kOptSGD ? 3 : 4;
   using G = BulkGeom<N, TILE, A>;
   constexpr int T = G::kTile, S = G::kStages;
@@ -594,27 +602,30 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
   __syncthreads();
 
   if (warp == kBulkConsumerWarps) {
-    // ---------------- producer: one thread issues every bulk copy
-    if (lane == 0) {
-      WaveCursor cur{0, 0};
-      int s;
-      int64_t v0, nv;
-      for (int k = 0; wave_item(b, T, cur, s, v0, nv); ++k) {
-        const int slot = k % S;
-        mbar_wait(&empty[slot], ((k / S) & 1) ^ 1);
-        fence_proxy_async();  // the consumers' generic-proxy reads of this slot precede the bulk writes
-        float4* base = smem + slot * G::kSlotVec;
-        const uint32_t bytes = static_cast<uint32_t>(nv * 16);
-        const StageRefs& st = b.st[s];
-        mbar_expect_tx(&full[slot], bytes * (A * N + 1));
-        bulk_g2s(base, st.c + 4 * v0, bytes, &full[slot]);
-#pragma unroll
-        for (int i = 0; i < N; ++i) {
-          bulk_g2s(base + (1 + A * i) * T, st.x[i] + 4 * v0, bytes, &full[slot]);
-          bulk_g2s(base + (2 + A * i) * T, st.g[i] + 4 * v0, bytes, &full[slot]);
-          bulk_g2s(base + (3 + A * i) * T, st.m[i] + 4 * v0, bytes, &full[slot]);
-          if (A == 4) bulk_g2s(base + (4 + A * i) * T, st.v[i] + 4 * v0, bytes, &full[slot]);
+    // ---------------- producer warp: lane 0 arms the slot's barrier, then lane q issues the bulk copy of
+    // stream q (q = 0: x~; 1 + A*i + {0,1,2,3}: x_i, g_i, state_i, v_i), so the A*N+1 copies of a slot
+    // leave in parallel instead of from one thread (the cursor is warp-uniform)
+    WaveCursor cur{0, 0};
+    int s;
+    int64_t v0, nv;
+    for (int k = 0; wave_item(b, T, cur, s, v0, nv); ++k) {
+      const int slot = k % S;
+      mbar_wait(&empty[slot], ((k / S) & 1) ^ 1);
+      fence_proxy_async();  // the consumers' generic-proxy reads of this slot precede the bulk writes
+      float4* base = smem + slot * G::kSlotVec;
+      const uint32_t bytes = static_cast<uint32_t>(nv * 16);
+      const StageRefs& st = b.st[s];
+      if (lane == 0) mbar_expect_tx(&full[slot], bytes * (A * N + 1));
+      __syncwarp();
+      for (int q = lane; q < A * N + 1 && lane < issue_lanes; q += issue_lanes) {
+        const float* src;
+        if (q == 0) {
+          src = st.c;
+        } else {
+          const int i = (q - 1) / A, kind = (q - 1) % A;
+          src = kind == 0 ? st.x[i] : kind == 1 ? st.g[i] : kind == 2 ? st.m[i] : st.v[i];
         }
+        bulk_g2s(base + q * T, src + 4 * v0, bytes, &full[slot]);
       }
     }
   } else {
@@ -662,16 +673,18 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
 }
 
 template <int N, int HINT, int OPT, int TILE>
-__global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp) {
-  bulkpipe_body<N, HINT, OPT, TILE, false>(b, hp, nullptr, 0);
+__global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp,
+                                                                      int issue_lanes) {
+  bulkpipe_body<N, HINT, OPT, TILE, false>(b, hp, nullptr, 0, issue_lanes);
 }
 
 // Spread local step (one replica) through the same bulk-copy pipeline: 4 input streams (x, g, state, x~;
 // + v for Adam) arrive by cp.async.bulk into the smem ring; x, state and r leave by 128-bit stores.
 template <int OPT, int TILE>
 __global__ void __launch_bounds__(kBulkThreads, 1) spread_bulkpipe(const StageBatch b, const Hyper hp,
-                                                                   float* __restrict__ contrib, int64_t p_pad) {
-  bulkpipe_body<1, 0, OPT, TILE, true>(b, hp, contrib, p_pad);
+                                                                   float* __restrict__ contrib, int64_t p_pad,
+                                                                   int issue_lanes) {
+  bulkpipe_body<1, 0, OPT, TILE, true>(b, hp, contrib, p_pad, issue_lanes);
 }
 
 // ============================================================================
@@ -848,6 +861,17 @@ cudaError_t launch_laneshfl(const StageBatch& b, const Hyper& hp, int num_sms, c
   return launch_laneshfl_t<N, HINT, OPT, kLanePasses, 2>(b, hp, num_sms, s);  // <= 128 regs: 2 CTAs/SM
 }
 
+// Copy-issue knob for measurement: AVGPIPE_EA_BULK_ISSUE=1 issues every bulk copy of a slot from one
+// producer lane (the first design); default: the 32 producer lanes issue them in parallel.
+int bulk_issue_lanes() {
+  static int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_BULK_ISSUE");
+    const int k = e ? std::atoi(e) : 32;
+    return (k >= 1 && k <= 32) ? k : 32;
+  }();
+  return v;
+}
+
 template <int N, int HINT, int OPT, int TILE>
 cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   using G = BulkGeom<N, TILE, OPT == kOptSGD ? 3 : 4>;
@@ -857,7 +881,7 @@ cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms,
   int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
   const int64_t units = units_of(b, G::kTile);
   if (grid > units) grid = units;
-  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp);
+  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp, bulk_issue_lanes());
   return cudaGetLastError();
 }
 
@@ -953,7 +977,7 @@ cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, con
   int64_t grid = num_sms;
   const int64_t units = (p / 4 + TILE - 1) / TILE;
   if (grid > units) grid = units < 1 ? 1 : units;
-  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp, contrib, p_pad);
+  k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp, contrib, p_pad, bulk_issue_lanes());
   return cudaGetLastError();
 }
 
