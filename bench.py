@@ -154,8 +154,9 @@ def kernel_name(variant, optimizer, n, staleness=0):
     if n > 8 or (optimizer != "sgd" and n > 6 and variant == "auto"):
         name = "colocated_wide"
     elif optimizer != "sgd":
-        name = ("colocated_laneshfl" if (n <= 2 and variant == "auto") or variant == "laneshfl"
-                else "colocated_" + ("bulkpipe" if variant == "auto" else variant))
+        if variant == "auto":
+            variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else "bulkpipe")
+        name = "colocated_" + variant
     elif variant == "auto":
         name = ("colocated_bulkpipe" if n in (1, 5, 6, 7) else
                 "colocated_laneshfl" if n <= 4 else "colocated_regloop")

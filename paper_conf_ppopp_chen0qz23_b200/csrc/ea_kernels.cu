@@ -541,12 +541,13 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
 constexpr int kBulkConsumerWarps = 8;
 constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 
-// Default tile (float4 per array per bulk copy), measured on B200 (profiles/r01_bulk_tiles.jsonl): 4 KB
-// copies except N = 4, 5 (2 KB copies, deeper ring) -- larger copies need fewer stages to keep the
-// same bytes in flight and reach DRAM as longer bursts.
+// Default tile (float4 per array per bulk copy), measured on B200 with the copies issued from all 32
+// producer lanes (profiles/r01_s2_bulk_lanes_tiles.jsonl, r01_s2_issue_ab.jsonl): 4 KB copies whenever a
+// two-stage ring of them fits in 200 KB (SGD N <= 8, Adam N <= 6), else 2 KB.  Smaller copies lose: the ring
+// depth is capped, so bytes in flight per SM shrink with the tile (1 KB: 0.27-0.69 of peak).
 template <int N, int A = 3>
 constexpr int default_bulk_tile() {
-  return A == 3 ? ((N == 4 || N == 5) ? 128 : 256) : ((A * N + 1) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128);
+  return (A * N + 1) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128;
 }
 
 constexpr int kMaxBulkStages = 6;  // ring depth cap (8 measured slower: profiles/r01_bulk_n4_tiles.jsonl)
@@ -1020,12 +1021,14 @@ cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
-  // library default per N, measured on B200 (C2 sizes, profiles/r01_nsweep*.jsonl, r01_bulk_tiles.jsonl):
-  // the bulk-copy pipeline for N = 1, 5, 6, 7 (0.93 / 1.01 / 0.95 / 0.95 of peak), the lane kernel for
-  // N = 2..4 (0.96 / 0.93 / 0.97; a warp holds >= 8 lanes per replica row), the register loop for N = 8 (0.97)
-  // Adam(W) (profiles/r01_adam_nsweep.jsonl): the lane kernel for N <= 2 (0.91 / 0.94), the bulk-copy
-  // pipeline for N = 3..6 (0.89 / 0.96 / 0.94 / 0.92); N > 6 goes to the replica-loop kernel (ea_api.cu)
-  if (variant == kVariantAuto && opt != kOptSGD) variant = n <= 2 ? kVariantLaneShfl : kVariantBulkPipe;
+  // library default per N, measured on B200 (C2 sizes; profiles/r01_nsweep*.jsonl, r01_s2_*.jsonl):
+  // SGD: the bulk-copy pipeline for N = 1, 5, 6, 7 (0.88-0.96 / 0.95 / 0.96 / 0.955 of peak), the lane kernel
+  // for N = 2..4 (0.96 / 0.93 / 0.97-0.99; a warp holds >= 8 lanes per replica row), the register loop for
+  // N = 8 (0.98-0.99).  Adam(W): the lane kernel for N = 1 (0.915), the register loop for N = 2, 3 (0.96 /
+  // 0.95; bulk pipeline 0.88 / 0.90), the bulk-copy pipeline for N = 4..6 (0.97 / 0.95 / 0.93); N > 6 goes to
+  // the replica-loop kernel (ea_api.cu)
+  if (variant == kVariantAuto && opt != kOptSGD)
+    variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : kVariantBulkPipe);
   if (variant == kVariantAuto)
     variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {
