@@ -378,3 +378,74 @@ def test_stale_zero_gradient_state_space_closed_form(n, alpha, rho):
         for i in range(n):
             np.testing.assert_allclose(cur_x[i] - np.mean(cur_x, axis=0), (1 - alpha) ** t * e0[i], rtol=1e-9,
                                        atol=1e-15)
+
+
+# ---------------------------------------------------------------- stale center with Adam / AdamW (f4 + f1)
+from oracle.ea_oracle import ea_step_adam_stale  # noqa: E402
+
+
+@pytest.mark.parametrize("decoupled", [False, True])
+def test_adam_stale_with_equal_centers_is_the_synchronous_adam_step(decoupled):
+    rng = np.random.default_rng(33)
+    n, p = 3, 100
+    xs, _, c = _rand_state(rng, n, p)
+    ms = [rng.normal(0, 1e-3, p) for _ in range(n)]
+    vs = [rng.uniform(0, 1e-4, p) for _ in range(n)]
+    g = [rng.normal(0, 1e-2, p) for _ in range(n)]
+    hp = Hyper(alpha=0.3, beta=0.9, rho=1.0, lr=1e-3, weight_decay=1e-2)
+    a = ea_step_adam(xs, ms, vs, c, g, hp, 4, decoupled=decoupled)
+    b = ea_step_adam_stale(xs, ms, vs, c, c, g, hp, 4, decoupled=decoupled)
+    for i in range(n):
+        np.testing.assert_array_equal(a[0][i], b[0][i])
+        np.testing.assert_array_equal(a[1][i], b[1][i])
+        np.testing.assert_array_equal(a[2][i], b[2][i])
+    np.testing.assert_array_equal(a[3], b[3])
+    np.testing.assert_array_equal(b[4], c)
+
+
+def test_adam_stale_alpha0_is_independent_torch_adam():
+    """alpha = 0: the stale reference never feeds back, so every replica is torch.optim.Adam (float64)."""
+    torch = pytest.importorskip("torch")
+    rng = np.random.default_rng(34)
+    n, p, steps = 2, 40, 6
+    xs, _, c = _rand_state(rng, n, p)
+    hp = Hyper(alpha=0.0, beta=0.7, rho=1.0, lr=1e-2, weight_decay=1e-2)
+    grads = [[rng.normal(0, 1e-2, p) for _ in range(n)] for _ in range(steps)]
+    ref = []
+    for i in range(n):
+        w = torch.tensor(xs[i], dtype=torch.float64, requires_grad=True)
+        opt = torch.optim.Adam([w], lr=hp.lr, betas=(hp.beta1, hp.beta2), eps=hp.eps, weight_decay=hp.weight_decay)
+        for t in range(steps):
+            w.grad = torch.tensor(grads[t][i], dtype=torch.float64)
+            opt.step()
+        ref.append(w.detach().numpy())
+    cur = (xs, [np.zeros(p)] * n, [np.zeros(p)] * n, c, c)
+    for t in range(steps):
+        x_, m_, v_, c_new, c_old = ea_step_adam_stale(cur[0], cur[1], cur[2], cur[3], cur[4], grads[t], hp, t + 1)
+        cur = (x_, m_, v_, c_new, c_old)
+    for i in range(n):
+        np.testing.assert_allclose(cur[0][i], ref[i], rtol=1e-13, atol=1e-15)
+
+
+@pytest.mark.parametrize("n,alpha,rho", [(2, 0.5, 1.0), (3, 0.2, 0.0)])
+def test_adam_stale_zero_gradient_state_space_closed_form(n, alpha, rho):
+    """Zero gradients and moments give Delta = 0 under Adam too, so the stale state-space closed form
+    (mean x, x~_t, x~_{t-1}) = A^t s_0 holds with A = [[1-a, 0, a], [b, 1, -b], [0, 1, 0]]."""
+    rng = np.random.default_rng(35)
+    p, steps = 50, 10
+    beta = n * alpha
+    xs, _, c = _rand_state(rng, n, p)
+    c = c + rng.normal(0, 1e-3, p)
+    hp = Hyper(alpha=alpha, beta=beta, rho=rho, lr=1e-3)
+    A = np.array([[1 - alpha, 0.0, alpha], [beta, 1.0, -beta], [0.0, 1.0, 0.0]])
+    s0 = np.stack([np.mean(xs, axis=0), c, c])
+    total0 = sum(xs) + c
+    z = [np.zeros(p)] * n
+    cur_x, cur_m, cur_v, cur_c, prev_c = xs, z, z, c, c
+    for t in range(1, steps + 1):
+        cur_x, cur_m, cur_v, cur_c, prev_c = ea_step_adam_stale(cur_x, cur_m, cur_v, cur_c, prev_c, z, hp, t)
+        st = np.linalg.matrix_power(A, t) @ s0
+        np.testing.assert_allclose(np.mean(cur_x, axis=0), st[0], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(cur_c, st[1], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(prev_c, st[2], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(sum(cur_x) + cur_c, total0, rtol=0, atol=1e-12)
