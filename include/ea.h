@@ -121,7 +121,7 @@ typedef struct {
   int32_t exchange;             /* EA_SPREAD: ea_exchange (ignored for EA_COLOCATED) */
   int32_t staleness;            /* 0: synchronous center (c3); 1: the replicas see the center one step
                                    late, x~_{t-1}, as with the paper's asynchronous queues (
-                                   reading c28, row f4).  1 needs EA_COLOCATED and EA_OPT_SGD; the
+                                   reading c28, row f4).  1 needs EA_COLOCATED (any optimizer); the
                                    library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step). */
 } ea_config;
 

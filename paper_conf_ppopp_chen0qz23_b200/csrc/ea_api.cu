@@ -556,8 +556,8 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
   if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
   if (c.staleness != 0 && c.staleness != 1) { set_err(nullptr, "staleness must be 0 or 1"); return EA_EINVAL; }
-  if (c.staleness == 1 && (c.layout != EA_COLOCATED || c.optimizer != EA_OPT_SGD)) {
-    set_err(nullptr, "staleness 1 is supported for EA_COLOCATED with EA_OPT_SGD");
+  if (c.staleness == 1 && c.layout != EA_COLOCATED) {
+    set_err(nullptr, "staleness 1 is supported for EA_COLOCATED");
     return EA_EINVAL;
   }
   if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {

@@ -12,7 +12,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_stale
+from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_adam_stale, ea_step_stale
 from paper_conf_ppopp_chen0qz23_b200 import synth
 
 TOL = 1e-5
@@ -65,8 +65,11 @@ class OracleStage:
 
     def step(self, grads, hp):
         self.t += 1
-        if self.staleness == 1:
+        if self.staleness == 1 and self.opt == "sgd":
             self.xs, self.ms, self.c, self.c_prev = ea_step_stale(self.xs, self.ms, self.c, self.c_prev, grads, hp)
+        elif self.staleness == 1:
+            self.xs, self.ms, self.vs, self.c, self.c_prev = ea_step_adam_stale(
+                self.xs, self.ms, self.vs, self.c, self.c_prev, grads, hp, self.t, decoupled=self.opt == "adamw")
         elif self.opt == "sgd":
             self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)
         else:

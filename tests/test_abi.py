@@ -89,7 +89,6 @@ def _cfg(**kw):
     (dict(optimizer=3), "optimizer"),
     (dict(exchange=5), "exchange"),
     (dict(staleness=2), "staleness"),
-    (dict(staleness=1, optimizer=1), "staleness 1"),
     (dict(staleness=1, layout=1, world=2, rank=0), "staleness 1"),
     (dict(layout=1, world=17, n_pipelines=17, rank=0, exchange=1), "world <="),
     (dict(optimizer=1, beta1=1.0), "betas"),

@@ -156,6 +156,15 @@ def test_stale_center(n, mode):
     _run_colocated(n, [65_537], 20, mode, variants=("auto",), staleness=1, nesterov=True, wd=1e-3)
 
 
+@pytest.mark.parametrize("optimizer", ["adam", "adamw"])
+@pytest.mark.parametrize("n", [1, 3, 8, 12])
+def test_stale_center_adam(optimizer, n):
+    """staleness 1 with Adam / AdamW as the local optimizer (readings c28 + c21)."""
+    _run_colocated(n, [100_003, 7, 4096], 30, "combined", variants=("auto",), staleness=1, many=True,
+                   optimizer=optimizer, lr=1e-3, wd=1e-2)
+    _run_colocated(n, [65_537], 15, "paper", variants=("auto",), staleness=1, optimizer=optimizer, lr=1e-3)
+
+
 def test_stale_center_c1_100_steps():
     _run_colocated(2, [1_000_000, 1_000_003], 100, "combined", variants=("auto",), staleness=1, many=True)
 
