@@ -322,7 +322,9 @@ def run_ours(args, rank, world, local):
         q = sorted(kern_ms)
         pct = {f"p{k}": q[min(len(q) - 1, len(q) * k // 100)] for k in (10, 50, 90)}
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                           "frac": achieved / peak, "traffic": traffic_from_profiles(cfg.name),
+                           "frac": achieved / peak,
+                           "traffic": traffic_from_profiles(cfg.name, kernel_name(args.variant, args.optimizer, n,
+                                                                                  args.staleness)),
                            "launch_ms_pct": pct,
                            "kernel": kernel_name(args.variant, args.optimizer, n, args.staleness),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
@@ -396,12 +398,14 @@ def same_box_copy_gbs(dev, nbytes=2 << 30, reps=10):
     return 2 * nbytes / (best * 1e-3) / 1e9
 
 
-def traffic_from_profiles(workload):
+def traffic_from_profiles(workload, kernel):
+    """ncu dram__bytes_read.sum + dram__bytes_write.sum per launch of this exact
+    (workload, kernel), from profiles/traffic.json; None when not captured."""
     path = os.path.join(ROOT, "profiles", "traffic.json")
     if not os.path.exists(path):
         return None
     d = json.load(open(path))
-    return d.get(workload, {}).get("dram_bytes_per_launch")
+    return d.get(f"{workload}|{kernel}", {}).get("dram_bytes_per_launch")
 
 
 def e2e_colocated(h, state, sizes, n, args, stream, dev, order):

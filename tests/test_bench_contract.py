@@ -62,3 +62,15 @@ def test_algorithmic_bytes(n):
 def test_default_workload_is_configs1():
     assert bench.workload_key(1, None) == "C2"
     assert bench.workload_key(8, None) == "C4"
+
+
+@pytest.mark.parametrize("optimizer", ["sgd", "adam"])
+def test_traffic_is_keyed_by_kernel(optimizer):
+    """roofline.traffic comes from an ncu capture of the SAME kernel: within 5% below the algorithmic
+    bytes (dirty L2 lines at the end of an isolated launch are not yet written back), never another
+    kernel's number."""
+    wl = "C2-resnet50-25M-N4-K4"
+    t = bench.traffic_from_profiles(wl, bench.kernel_name("auto", optimizer, 4))
+    alg = bench.bytes_colocated(4, 25_000_000, optimizer)
+    assert t is not None and 0.95 * alg <= t <= alg * 1.01
+    assert bench.traffic_from_profiles(wl, "no_such_kernel") is None
