@@ -277,6 +277,41 @@ __global__ void __launch_bounds__(kThreads, regloop_min_blocks<N, OPT>()) coloca
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
 
+template <int U>
+struct WideRep {
+  float4 x[U], g[U], m[U], w[U];
+};
+
+template <int U, int OPT>
+__device__ __forceinline__ void wide_load(const ReplicaTable& t, int i, int64_t base, const bool* ok,
+                                          const Mem<0>& mem, WideRep<U>& r) {
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    const int64_t v = base + (int64_t)u * kThreads;
+    if (ok[u]) {
+      r.x[u] = mem.ld(t.x[i] + 4 * v);
+      r.g[u] = mem.ld_ro(t.g[i] + 4 * v);
+      r.m[u] = mem.ld(t.m[i] + 4 * v);
+      if (OPT != kOptSGD) r.w[u] = mem.ld(t.v[i] + 4 * v);
+    }
+  }
+}
+
+template <int U, int OPT>
+__device__ __forceinline__ void wide_proc(const ReplicaTable& t, int i, int64_t base, const bool* ok,
+                                          const Mem<0>& mem, WideRep<U>& r, const float4* cu, float4* acc,
+                                          const Hyper& hp, const StepCoef& sc) {
+#pragma unroll
+  for (int u = 0; u < U; ++u) {
+    if (!ok[u]) continue;
+    const int64_t v = base + (int64_t)u * kThreads;
+    add4(acc[u], ea_vec<OPT>(r.x[u], r.g[u], r.m[u], r.w[u], cu[u], hp, sc));
+    mem.st(t.x[i] + 4 * v, r.x[u]);
+    mem.st(t.m[i] + 4 * v, r.m[u]);
+    if (OPT != kOptSGD) mem.st(t.v[i] + 4 * v, r.w[u]);
+  }
+}
+
 // Runtime-N replica loop (N > 8, Adam N > 6, the stale center): one stage,
 // replicas visited in a loop.  prev != nullptr selects the stale center of
 // row f4 (reading c28): the replicas use x~_{t-1} (prev) for dilution and
@@ -306,28 +341,18 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
           cu[u] = stale ? mem.ld(prev + 4 * v) : c[u];   // the center the replicas see
         }
       }
-      for (int i = 0; i < n; ++i) {
-        float4 x[U], g[U], m[U], w[U];
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int64_t v = base + (int64_t)u * kThreads;
-          if (ok[u]) {
-            x[u] = mem.ld(t.x[i] + 4 * v);
-            g[u] = mem.ld_ro(t.g[i] + 4 * v);
-            m[u] = mem.ld(t.m[i] + 4 * v);
-            if (OPT != kOptSGD) w[u] = mem.ld(t.v[i] + 4 * v);
-          }
-        }
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          if (!ok[u]) continue;
-          const int64_t v = base + (int64_t)u * kThreads;
-          add4(acc[u], ea_vec<OPT>(x[u], g[u], m[u], w[u], cu[u], hp, sc));
-          mem.st(t.x[i] + 4 * v, x[u]);
-          mem.st(t.m[i] + 4 * v, m[u]);
-          if (OPT != kOptSGD) mem.st(t.v[i] + 4 * v, w[u]);
-        }
+      // software-pipelined replica loop: replica i+1's loads are in flight while replica i is updated
+      // (replicas never alias, ABI contract), two register buffers with compile-time names
+      WideRep<U> ra, rb;
+      wide_load<U, OPT>(t, 0, base, ok, mem, ra);
+      int i = 0;
+      for (; i + 1 < n; i += 2) {
+        wide_load<U, OPT>(t, i + 1, base, ok, mem, rb);
+        wide_proc<U, OPT>(t, i, base, ok, mem, ra, cu, acc, hp, sc);
+        if (i + 2 < n) wide_load<U, OPT>(t, i + 2, base, ok, mem, ra);
+        wide_proc<U, OPT>(t, i + 1, base, ok, mem, rb, cu, acc, hp, sc);
       }
+      if (i < n) wide_proc<U, OPT>(t, i, base, ok, mem, ra, cu, acc, hp, sc);
 #pragma unroll
       for (int u = 0; u < U; ++u) {
         const int64_t v = base + (int64_t)u * kThreads;
