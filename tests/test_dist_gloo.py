@@ -7,7 +7,7 @@ bounds, collective calls and stage order.  The composition must equal the
 co-located oracle step (the oracle is layout-agnostic).
 """
 import os
-import socket
+import tempfile
 
 import numpy as np
 import pytest
@@ -20,11 +20,9 @@ from paper_conf_ppopp_chen0qz23_b200 import parallel, synth
 
 
 def _free_port():
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
-    return port
+    """A fresh file:// rendezvous (no TCP port to race for between tests)."""
+    d = tempfile.mkdtemp(prefix="gloo_")
+    return "file://" + os.path.join(d, "store")
 
 
 def test_placement_is_a_latin_square():
@@ -50,9 +48,7 @@ def test_padding_and_shards():
 
 
 def _worker(rank, world, port, q):
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
-    dist.init_process_group("gloo", rank=rank, world_size=world)
+    dist.init_process_group("gloo", init_method=port, rank=rank, world_size=world)
     try:
         n = world
         a, b, r = synth.mode_coeffs("combined", n)

@@ -5,7 +5,7 @@ reference (full model, same micro-batches, loss/M summed); the peak stash of
 each stage must be min(a_k+1, M); with the dynamic controller
 all stages agree on the advance after every iteration (c16 feasibility)."""
 import os
-import socket
+import tempfile
 
 import pytest
 import torch
@@ -30,10 +30,8 @@ def _data(N, M, seed=0):
 
 
 def _worker(rank, K, N, M, extra, dynamic, port, q):
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
     try:
-        dist.init_process_group("gloo", rank=rank, world_size=K)
+        dist.init_process_group("gloo", init_method=port, rank=rank, world_size=K)
         from paper_conf_ppopp_chen0qz23_b200.pipeline import PipelineStage
         models = [_model(100 + i) for i in range(N)]
         stage_mods = [m[rank] for m in models]
@@ -57,11 +55,14 @@ def _worker(rank, K, N, M, extra, dynamic, port, q):
             dist.destroy_process_group()
 
 
+def _file_store():
+    """A fresh file:// rendezvous (no TCP port to race for between tests)."""
+    d = tempfile.mkdtemp(prefix="gloo_")
+    return "file://" + os.path.join(d, "store")
+
+
 def _run(K, N, M, extra, dynamic=False):
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
+    port = _file_store()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     procs = [ctx.Process(target=_worker, args=(r, K, N, M, extra, dynamic, port, q)) for r in range(K)]
