@@ -117,11 +117,9 @@ def _ipc_worker(rank, world, port, q):
     the fused exchange against the other process (time-sliced on one GPU)."""
     import numpy as np  # noqa: F401
     import torch.distributed as dist
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
     os.environ["AVGPIPE_EA_P2P_TIMEOUT_MS"] = "60000"
     try:
-        dist.init_process_group("gloo", rank=rank, world_size=world)
+        dist.init_process_group("gloo", init_method=port, rank=rank, world_size=world)
         from paper_conf_ppopp_chen0qz23_b200.parallel import connect_p2p
         n, sizes, steps = world, [100_003, 70], 5
         hp = hyper(n, "combined")
@@ -161,12 +159,9 @@ def _ipc_worker(rank, world, port, q):
 def test_p2p_exchange_across_processes_via_cuda_ipc():
     """The multi-process path (cudaIpcGetMemHandle -> all-gather -> cudaIpcOpenMemHandle,
     system-scope release/acquire across processes) with 2 processes on one GPU."""
-    import socket
+    import tempfile
     import torch.multiprocessing as mp
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
+    port = "file://" + os.path.join(tempfile.mkdtemp(prefix="gloo_"), "store")   # no TCP port race
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     procs = [ctx.Process(target=_ipc_worker, args=(r, 2, port, q)) for r in range(2)]

@@ -5,7 +5,6 @@ on the stage's parameters (views into flat buffers the kernel updates in
 place).  Compared with a single-process reference: the full model's autograd
 plus the float64 oracle step (rounded to fp32 storage) -- rows f2 + a1-a5."""
 import os
-import socket
 
 import numpy as np
 import pytest
@@ -50,10 +49,8 @@ def _flatten(mod, device):
 
 
 def _worker(rank, port, q):
-    os.environ["MASTER_ADDR"] = "127.0.0.1"
-    os.environ["MASTER_PORT"] = str(port)
     try:
-        dist.init_process_group("gloo", rank=rank, world_size=K)
+        dist.init_process_group("gloo", init_method=port, rank=rank, world_size=K)
         from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
         from paper_conf_ppopp_chen0qz23_b200.pipeline import PipelineStage
         dev = torch.device("cuda:0")
@@ -116,10 +113,8 @@ def _reference():
 
 
 def test_pipeline_with_elastic_averaging_matches_reference():
-    s = socket.socket()
-    s.bind(("127.0.0.1", 0))
-    port = s.getsockname()[1]
-    s.close()
+    import tempfile
+    port = "file://" + os.path.join(tempfile.mkdtemp(prefix="gloo_"), "store")   # no TCP port race
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     procs = [ctx.Process(target=_worker, args=(r, port, q)) for r in range(K)]
