@@ -398,6 +398,23 @@ def same_box_copy_gbs(dev, nbytes=2 << 30, reps=10):
     return 2 * nbytes / (best * 1e-3) / 1e9
 
 
+def same_box_h2d_gbs(dev, pinned, reps=5):
+    """Pinned host -> device copy bandwidth of this box (best of `reps` copies of
+    the given pinned tensor): the PCIe bound of the e2e line."""
+    import torch
+    d = torch.empty_like(pinned, device=dev)
+    best = None
+    for _ in range(reps + 1):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        d.copy_(pinned, non_blocking=True)
+        e1.record()
+        e1.synchronize()
+        t = e0.elapsed_time(e1)
+        best = t if best is None else min(best, t)
+    return pinned.numel() * pinned.element_size() / (best * 1e-3) / 1e9
+
+
 def traffic_from_profiles(workload, kernel):
     """ncu dram__bytes_read.sum + dram__bytes_write.sum per launch of this exact
     (workload, kernel), from profiles/traffic.json; None when not captured."""
@@ -431,8 +448,12 @@ def e2e_colocated(h, state, sizes, n, args, stream, dev, order):
     t1.record(stream)
     torch.cuda.synchronize()
     ms = t0.elapsed_time(t1) / args.e2e_steps
+    h2d = 4 * n * sum(sizes)
+    pcie = same_box_h2d_gbs(dev, host_g[0][0])
     return {"value": n * sum(sizes) / (ms * 1e-3), "unit": UNIT, "ms_per_step": ms,
-            "h2d_bytes_per_step": 4 * n * sum(sizes), "d2h_bytes_per_step": 4 * sum(sizes),
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": 4 * sum(sizes),
+            "h2d_gbs": h2d / (ms * 1e-3) / 1e9, "h2d_gbs_same_box": pcie,
+            "pcie_frac": h2d / (ms * 1e-3) / 1e9 / pcie,
             "path": "ea_step_many_host: pinned host grads -> device (chunked, copy stream), fused kernel per chunk, "
                     "center chunks -> pinned host (second copy stream)"}
 
