@@ -32,8 +32,6 @@ namespace ea {
 namespace {
 
 constexpr int kP2PThreads = 256;
-constexpr int kU = 4;    // float4 per thread in flight per stream, phases A and C
-constexpr int kUB = 2;   // phase B (N contributions each)
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -108,63 +106,42 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
   const uint32_t epoch = static_cast<uint32_t>(*a.stepp);
   const StepCoef sc = OPT == kOptSGD ? StepCoef{0.f, 0.f} : *a.scp;
 
-  // ---------------- Phase A: local update, push contributions to the owners.  Each thread hoists the loads
-  // of kU float4 (x, g, state, x~) before any arithmetic: bytes in flight, not instructions, bound a single
-  // rank's kernel (one kernel per GPU owns the whole HBM, unlike the N virtual ranks of the 1-GPU proxy).
+  // ---------------- Phase A: local update, push contributions to the owners
   for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
     const int o = static_cast<int>(c % N);
     const int64_t slot = c / N;
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    const int64_t nv4 = len / 4;
     float* dst = view.inbox[o] + ((int64_t)r * slots + slot) * Q;
-    for (int64_t lb = tid; lb < nv4; lb += (int64_t)kP2PThreads * kU) {
-      float4 x[kU], g[kU], m[kU], c4[kU], w[kU];
-      bool full[kU];
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        const int64_t j = e0 + 4 * lv;
-        full[u] = lv < nv4 && j + 3 < a.p;
-        if (full[u]) {
-          x[u] = ld4(a.x + j);
-          g[u] = ld4(a.g + j);
-          m[u] = ld4(a.m + j);
-          c4[u] = ld4(a.center + j);
-          w[u] = OPT == kOptSGD ? make_float4(0.f, 0.f, 0.f, 0.f) : ld4(a.v + j);
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        if (lv >= nv4) continue;
-        const int64_t j = e0 + 4 * lv;
-        float4 rv;
-        if (full[u]) {
-          rv.x = p2p_elem<OPT>(x[u].x, g[u].x, m[u].x, w[u].x, c4[u].x, a.hp, sc);
-          rv.y = p2p_elem<OPT>(x[u].y, g[u].y, m[u].y, w[u].y, c4[u].y, a.hp, sc);
-          rv.z = p2p_elem<OPT>(x[u].z, g[u].z, m[u].z, w[u].z, c4[u].z, a.hp, sc);
-          rv.w = p2p_elem<OPT>(x[u].w, g[u].w, m[u].w, w[u].w, c4[u].w, a.hp, sc);
-          st4(a.x + j, x[u]);
-          st4(a.m + j, m[u]);
-          if (OPT != kOptSGD) st4(a.v + j, w[u]);
-        } else {  // the ragged end of the replica and the zero padding of the center
-          float rr[4];
-          for (int q = 0; q < 4; ++q) {
-            const int64_t jj = j + q;
-            rr[q] = 0.f;
-            if (jj < a.p) {
-              float xs = a.x[jj], ms = a.m[jj], ws = OPT == kOptSGD ? 0.f : a.v[jj];
-              rr[q] = p2p_elem<OPT>(xs, a.g[jj], ms, ws, a.center[jj], a.hp, sc);
-              a.x[jj] = xs;
-              a.m[jj] = ms;
-              if (OPT != kOptSGD) a.v[jj] = ws;
-            }
+    for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) {
+      const int64_t j = e0 + 4 * lv;
+      float4 rv;
+      if (j + 3 < a.p) {
+        float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
+        float4 w = OPT == kOptSGD ? make_float4(0.f, 0.f, 0.f, 0.f) : ld4(a.v + j);
+        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
+        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
+        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
+        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
+        st4(a.x + j, x);
+        st4(a.m + j, m);
+        if (OPT != kOptSGD) st4(a.v + j, w);
+      } else {  // the ragged end of the replica and the zero padding of the center
+        float rr[4];
+        for (int q = 0; q < 4; ++q) {
+          const int64_t jj = j + q;
+          rr[q] = 0.f;
+          if (jj < a.p) {
+            float x = a.x[jj], m = a.m[jj], w = OPT == kOptSGD ? 0.f : a.v[jj];
+            rr[q] = p2p_elem<OPT>(x, a.g[jj], m, w, a.center[jj], a.hp, sc);
+            a.x[jj] = x;
+            a.m[jj] = m;
+            if (OPT != kOptSGD) a.v[jj] = w;
           }
-          rv = make_float4(rr[0], rr[1], rr[2], rr[3]);
         }
-        st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
+        rv = make_float4(rr[0], rr[1], rr[2], rr[3]);
       }
+      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
     }
     __syncthreads();
     if (tid == 0) {
@@ -180,43 +157,21 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     if (c >= nch) continue;
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    const int64_t nv4 = len / 4;
     if (tid == 0) s_ok = wait_at_least(view.arrive[r] + slot, (uint32_t)N * epoch, a.timeout_ns, a.err);
     __syncthreads();
     const float* in = view.inbox[r] + slot * Q;
     float* out = view.outbox[r] + slot * Q;
-    for (int64_t lb = tid; lb < nv4; lb += (int64_t)kP2PThreads * kUB) {
-      float4 sum[kUB], cv[kUB];
-#pragma unroll
-      for (int u = 0; u < kUB; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        sum[u] = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (lv < nv4) cv[u] = ld4(a.center + e0 + 4 * lv);
-      }
+    for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) {
+      float4 sum = make_float4(0.f, 0.f, 0.f, 0.f);
       for (int src = 0; src < N; ++src) {
-        float4 t[kUB];
-#pragma unroll
-        for (int u = 0; u < kUB; ++u) {
-          const int64_t lv = lb + (int64_t)u * kP2PThreads;
-          if (lv < nv4) t[u] = ld_cg(in + (int64_t)src * slots * Q + 4 * lv);
-        }
-#pragma unroll
-        for (int u = 0; u < kUB; ++u) {
-          const int64_t lv = lb + (int64_t)u * kP2PThreads;
-          if (lv < nv4) {
-            sum[u].x += t[u].x; sum[u].y += t[u].y; sum[u].z += t[u].z; sum[u].w += t[u].w;
-          }
-        }
+        const float4 t = ld_cg(in + (int64_t)src * slots * Q + 4 * lv);
+        sum.x += t.x; sum.y += t.y; sum.z += t.z; sum.w += t.w;
       }
-#pragma unroll
-      for (int u = 0; u < kUB; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        if (lv >= nv4) continue;
-        const float4 nc = make_float4(fmaf(sum[u].x, inv_n, cv[u].x), fmaf(sum[u].y, inv_n, cv[u].y),
-                                      fmaf(sum[u].z, inv_n, cv[u].z), fmaf(sum[u].w, inv_n, cv[u].w));
-        st4(a.center + e0 + 4 * lv, nc);
-        st4(out + 4 * lv, nc);
-      }
+      float4 cv = ld4(a.center + e0 + 4 * lv);
+      cv = make_float4(fmaf(sum.x, inv_n, cv.x), fmaf(sum.y, inv_n, cv.y), fmaf(sum.z, inv_n, cv.z),
+                       fmaf(sum.w, inv_n, cv.w));
+      st4(a.center + e0 + 4 * lv, cv);
+      st4(out + 4 * lv, cv);
     }
     __syncthreads();
     if (tid == 0) {
@@ -233,23 +188,10 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     const int64_t slot = c / N;
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    const int64_t nv4 = len / 4;
     if (tid == 0) s_ok = wait_at_least(view.ready[o] + slot, epoch, a.timeout_ns, a.err);
     __syncthreads();
     const float* src = view.outbox[o] + slot * Q;
-    for (int64_t lb = tid; lb < nv4; lb += (int64_t)kP2PThreads * kU) {
-      float4 t[kU];
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        if (lv < nv4) t[u] = ld_cg(src + 4 * lv);
-      }
-#pragma unroll
-      for (int u = 0; u < kU; ++u) {
-        const int64_t lv = lb + (int64_t)u * kP2PThreads;
-        if (lv < nv4) st4(a.center + e0 + 4 * lv, t[u]);
-      }
-    }
+    for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) st4(a.center + e0 + 4 * lv, ld_cg(src + 4 * lv));
     __syncthreads();
   }
 }
