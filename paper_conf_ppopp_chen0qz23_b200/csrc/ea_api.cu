@@ -60,6 +60,7 @@ struct ea_ctx {
   size_t xbuf_bytes = 0;
   std::vector<size_t> x_inbox, x_outbox, x_arrive, x_ready;  // per-stage byte offsets into xbuf
   std::vector<int64_t> x_nchunks, x_slots;
+  int64_t x_chunk = 0;  // floats per exchange chunk (p2p_chunk() at ea_init; every rank must agree)
   std::vector<char*> peer_base;   // world entries, as mapped on this device (self = xbuf)
   std::vector<char> peer_ipc;     // 1 = opened with cudaIpcOpenMemHandle (closed at destroy)
   bool p2p_ready = false;
@@ -86,8 +87,15 @@ int64_t host_chunk() {
   }();
   return v;
 }
-// Floats per exchange chunk of the fused peer-memory spread kernel (32 KB).
-constexpr int64_t kP2PChunk = 8192;
+
+// Floats per exchange chunk of the fused peer-memory spread kernel (default 8192 = 32 KB).
+// Measurement knob AVGPIPE_EA_P2P_CHUNK (a multiple of 1024 floats, 1024..65536); every rank of an
+// exchange must use the same value (it fixes the layout of the peers' inboxes).
+int64_t p2p_chunk() {
+  const char* e = std::getenv("AVGPIPE_EA_P2P_CHUNK");
+  const long long v = e ? std::atoll(e) : 0;
+  return (v >= 1024 && v <= 65536 && v % 1024 == 0) ? v : 8192;
+}
 
 namespace {
 
@@ -376,6 +384,7 @@ ea_status p2p_alloc(ea_ctx* h) {
     off += (bytes + 255) / 256 * 256;
     return at;
   };
+  const int64_t kP2PChunk = h->x_chunk = p2p_chunk();
   for (int s = 0; s < h->cfg.n_stages; ++s) {
     const int64_t nch = (h->p_pad[s] + kP2PChunk - 1) / kP2PChunk;
     const int64_t slots = (nch + n - 1) / n;
@@ -474,7 +483,7 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   a.center = center_ptr;
   a.p = h->p[stage];
   a.p_pad = h->p_pad[stage];
-  a.chunk = kP2PChunk;
+  a.chunk = h->x_chunk;
   a.nchunks = h->x_nchunks[stage];
   a.slots = h->x_slots[stage];
   a.rank = h->cfg.rank;
@@ -487,7 +496,7 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   a.err = h->err_dev;
   a.timeout_ns = p2p_timeout_ns();
   // all ranks' kernels must be resident together: ranks sharing this device share its SMs
-  int max_ctas = h->num_sms * ea::p2p_blocks_per_sm() / h->same_device_ranks;
+  int max_ctas = h->num_sms * ea::p2p_blocks_per_sm(h->cfg.optimizer) / h->same_device_ranks;
   if (max_ctas < 1) max_ctas = 1;
   cudaError_t e = ea::launch_spread_p2p(a, v, h->cfg.optimizer, max_ctas, s);
   if (e != cudaSuccess) return cuda_fail(h, e, "peer-memory exchange kernel launch");

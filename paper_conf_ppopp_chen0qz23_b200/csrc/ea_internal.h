@@ -130,7 +130,7 @@ struct P2PArgs {
 };
 
 cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);
-int p2p_blocks_per_sm();
+int p2p_blocks_per_sm(int opt);
 
 // Spread shard epilogue (row a5): shard[k] += reduced[k] * inv_n for k < count.
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,

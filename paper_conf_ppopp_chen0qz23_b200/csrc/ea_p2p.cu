@@ -209,12 +209,20 @@ cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int m
   return cudaGetLastError();
 }
 
-int p2p_blocks_per_sm() {
+template <int OPT>
+int blocks_per_sm_t() {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<kOptAdam>, kP2PThreads, 0) != cudaSuccess ||
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT>, kP2PThreads, 0) != cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   return per_sm;
+}
+
+// Resident CTAs per SM of the instance that will run (SGD 32 registers: 8; Adam(W) 48: 5).  The grid never
+// exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
+int p2p_blocks_per_sm(int opt) {
+  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD>();
+  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam>() : blocks_per_sm_t<kOptAdamW>();
 }
 
 }  // namespace ea
