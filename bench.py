@@ -76,6 +76,23 @@ def dist_env():
     return rank, world, local
 
 
+def shared_gpu_test_mode():
+    """AVGPIPE_BENCH_SHARED_GPU=1 (tests only): every rank on cuda:0, a gloo control group, the P2P
+    exchange wired over CUDA IPC -- exercises the N>1 code path of this script on a one-GPU box, where
+    NCCL refuses two ranks on one device.  The ranks' kernels are time-sliced, so its numbers mean nothing."""
+    return os.environ.get("AVGPIPE_BENCH_SHARED_GPU") == "1"
+
+
+def max_over_ranks(ms, dev):
+    """Max of a per-rank device time over the process group (NCCL: a device tensor; gloo: host)."""
+    import torch
+    import torch.distributed as dist
+    on_dev = dist.get_backend() == "nccl"
+    tt = torch.tensor([ms], device=dev if on_dev else "cpu")
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    return float(tt.item())
+
+
 def measured_peaks():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     if os.path.exists(path):
@@ -194,6 +211,9 @@ def run_ours(args, rank, world, local):
     from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
     from paper_conf_ppopp_chen0qz23_b200 import parallel
 
+    shared = shared_gpu_test_mode()
+    if shared:
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     key = workload_key(world, args.config)
@@ -211,11 +231,19 @@ def run_ours(args, rank, world, local):
         os.environ.setdefault("MASTER_PORT", "29531")
         os.environ.setdefault("RANK", str(rank))
         os.environ.setdefault("WORLD_SIZE", str(world))
-        dist.init_process_group("nccl", device_id=dev)
-        uid = parallel.broadcast_unique_id()
+        if shared:
+            if args.exchange != "p2p" and world > 1:
+                raise SystemExit("AVGPIPE_BENCH_SHARED_GPU=1 needs --exchange p2p (NCCL refuses two ranks on one GPU)")
+            dist.init_process_group("gloo")
+            uid = None
+        else:
+            dist.init_process_group("nccl", device_id=dev)
+            uid = parallel.broadcast_unique_id()
         h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
                              layout="spread", rank=rank, world=world, device=local, nccl_id=uid,
                              optimizer=args.optimizer, exchange=args.exchange)
+        if shared and world > 1:
+            parallel.connect_p2p(h)      # IPC handles over the gloo group
         state = []
         for s, p in enumerate(sizes):
             reps, c0, grads = synth.device_state(1, p, dev, seed=1000 * s)   # same center on every rank
@@ -292,9 +320,7 @@ def run_ours(args, rank, world, local):
         torch.cuda.synchronize()
     ms = t0.elapsed_time(t1) / args.steps
     if spread:
-        tt = torch.tensor([ms], device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        ms = float(tt.item())
+        ms = max_over_ranks(ms, dev)
     total_params = sum(sizes)
     value = n * total_params / (ms * 1e-3)
     peak, peak_src = measured_peaks()
@@ -491,10 +517,7 @@ def e2e_spread(h, state, sizes, args, stream, dev, order, rank, world):
         step()
     t1.record(stream)
     torch.cuda.synchronize()
-    ms = t0.elapsed_time(t1) / args.e2e_steps
-    tt = torch.tensor([ms], device=dev)
-    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    ms = float(tt.item())
+    ms = max_over_ranks(t0.elapsed_time(t1) / args.e2e_steps, dev)
     return {"value": world * sum(sizes) / (ms * 1e-3), "unit": UNIT, "ms_per_step": ms,
             "h2d_bytes_per_step": 4 * world * sum(sizes), "d2h_bytes_per_step": 4 * world * sum(shard),
             "path": "per rank: pinned host grads -> device (non_blocking copy on the step stream), ea_step per "

@@ -43,3 +43,26 @@ def test_bench_spread_world1_line(opt):
     r = d["roofline"]     # world 1: the local kernel's HBM roofline
     assert r["bound"] == "hbm" and r["kernel"].startswith("spread_bulkpipe") and r["frac"] > 0
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 4 * 2_000_000
+
+
+def test_bench_world2_line_on_one_gpu():
+    """bench.py's N>1 path (torchrun, 2 ranks, spread layout, max over ranks, rank-0 JSON line, e2e)
+    on a one-GPU box: both ranks on cuda:0 with the P2P exchange over CUDA IPC and a gloo control
+    group (AVGPIPE_BENCH_SHARED_GPU=1; NCCL refuses two ranks on one device).  Crash guard only:
+    the two ranks' kernels are time-sliced."""
+    import socket
+    with socket.socket() as sk:
+        sk.bind(("127.0.0.1", 0))
+        port = str(sk.getsockname()[1])
+    env = dict(os.environ, AVGPIPE_BENCH_SHARED_GPU="1", AVGPIPE_EA_P2P_TIMEOUT_MS="120000")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", port, "bench.py", "--gpus", "2", "--exchange", "p2p",
+           "--config", "C1", "--steps", "3", "--warmup", "3", "--e2e-steps", "2"]
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
+    assert r.returncode == 0, r.stderr[-3000:]
+    lines = [l for l in r.stdout.splitlines() if l.strip().startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert KEYS <= set(d), KEYS - set(d)
+    assert d["n_gpus"] == 2 and d["config"]["layout"] == "spread" and d["config"]["exchange"] == "p2p"
+    assert d["roofline"]["bound"] == "nvlink" and d["value"] > 0 and d["e2e"]["value"] > 0
