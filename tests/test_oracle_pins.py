@@ -449,3 +449,85 @@ def test_adam_stale_zero_gradient_state_space_closed_form(n, alpha, rho):
         np.testing.assert_allclose(cur_c, st[1], rtol=1e-12, atol=1e-15)
         np.testing.assert_allclose(prev_c, st[2], rtol=1e-12, atol=1e-15)
         np.testing.assert_allclose(sum(cur_x) + cur_c, total0, rtol=0, atol=1e-12)
+
+
+# ---------------------------------------------------------------- ASGD (row f1, reading c29)
+@pytest.mark.parametrize("wd,lambd,t0", [(0.0, 1e-4, 1e6), (1e-2, 5e-2, 3.0), (0.0, 2e-1, 0.0)])
+@pytest.mark.parametrize("beta,rho", [(0.0, 1.0), (2.0, 0.0), (0.7, 0.3)])
+def test_p1_asgd_alpha0_is_independent_torch_asgd(wd, lambd, t0, beta, rho):
+    """alpha = 0 => N independent torch.optim.ASGD trajectories, iterate AND average ax
+    (library routine; t0 small so the running average with mu < 1 is exercised)."""
+    from oracle.ea_oracle import ea_step_asgd
+    rng = np.random.default_rng(31)
+    n, p, steps, lr, a = 3, 211, 14, 0.5, 0.75
+    xs, _, c = _rand_state(rng, n, p)
+    gs = _grads(rng, n, p, steps)
+    hp = Hyper(alpha=0.0, beta=beta, rho=rho, lr=lr, weight_decay=wd, asgd_lambd=lambd, asgd_alpha=a, asgd_t0=t0)
+    ox, oa, oc = [x.copy() for x in xs], [np.zeros(p) for _ in range(n)], c.copy()
+    for t in range(steps):
+        ox, oa, oc = ea_step_asgd(ox, oa, oc, gs[t], hp, t + 1)
+    # torch keeps ASGD's eta and mu as scalar tensors of the default dtype: float64 here, so the library
+    # routine runs entirely in float64 like the oracle
+    prev = torch.get_default_dtype()
+    torch.set_default_dtype(torch.float64)
+    try:
+        for i in range(n):
+            w = torch.nn.Parameter(torch.tensor(xs[i], dtype=torch.float64))
+            opt = torch.optim.ASGD([w], lr=lr, lambd=lambd, alpha=a, t0=t0, weight_decay=wd)
+            for t in range(steps):
+                w.grad = torch.tensor(gs[t][i], dtype=torch.float64)
+                opt.step()
+            np.testing.assert_allclose(ox[i], w.detach().numpy(), rtol=1e-13, atol=1e-16)
+            np.testing.assert_allclose(oa[i], opt.state[w]["ax"].numpy(), rtol=1e-13, atol=1e-16)
+    finally:
+        torch.set_default_dtype(prev)
+
+
+def test_asgd_average_is_the_mean_of_the_iterates():
+    """t0 = 0: mu_t = 1/max(1, t-1), so after t >= 2 steps the average is the arithmetic mean of the
+    optimizer's iterates x_2 .. x_t (the definition of averaged SGD, ref [27]), computed here from the
+    replica trajectory itself (alpha = 0)."""
+    from oracle.ea_oracle import ea_step_asgd
+    rng = np.random.default_rng(32)
+    n, p, steps = 2, 64, 9
+    xs, _, c = _rand_state(rng, n, p)
+    hp = Hyper(alpha=0.0, beta=0.0, rho=1.0, lr=0.3, asgd_lambd=1e-2, asgd_t0=0.0)
+    traj = [[] for _ in range(n)]
+    axs = [np.zeros(p) for _ in range(n)]
+    for t, g in enumerate(_grads(rng, n, p, steps)):
+        xs, axs, c = ea_step_asgd(xs, axs, c, g, hp, t + 1)
+        for i in range(n):
+            traj[i].append(xs[i])
+    for i in range(n):
+        np.testing.assert_allclose(axs[i], np.mean(traj[i][1:], axis=0), rtol=1e-13, atol=1e-17)
+
+
+def test_asgd_zero_gradients_closed_form():
+    """Zero gradients, N = 1, alpha = 0: x_t = x_0 * prod_k (1 - lambd*eta_k) with
+    eta_k = lr / (1 + lambd*lr*(k-1))**a -- the decay term alone, hand-evaluated."""
+    from oracle.ea_oracle import ea_step_asgd
+    rng = np.random.default_rng(33)
+    p, steps, lr, lambd, a = 50, 12, 0.4, 0.1, 0.75
+    x0 = rng.normal(0, 0.02, p)
+    hp = Hyper(alpha=0.0, beta=0.0, rho=1.0, lr=lr, asgd_lambd=lambd, asgd_alpha=a)
+    xs, axs, c = [x0.copy()], [np.zeros(p)], x0.copy()
+    f = 1.0
+    for k in range(1, steps + 1):
+        xs, axs, c = ea_step_asgd(xs, axs, c, [np.zeros(p)], hp, k)
+        f *= 1.0 - lambd * lr / (1.0 + lambd * lr * (k - 1)) ** a
+        np.testing.assert_allclose(xs[0], x0 * f, rtol=1e-14, atol=0)
+        np.testing.assert_allclose(c, x0 * f, rtol=1e-14, atol=0)   # N = 1, rho = 1: x~ follows x
+
+
+def test_p3_asgd_center_stays_the_average():
+    """'stays the average' with ASGD as the local optimizer (rho = 1, centered init)."""
+    from oracle.ea_oracle import ea_step_asgd
+    rng = np.random.default_rng(34)
+    n, p = 4, 150
+    xs, _, _ = _rand_state(rng, n, p)
+    c = np.mean(xs, axis=0)
+    hp = Hyper(alpha=1 / n, beta=0.4, rho=1.0, lr=0.2, weight_decay=1e-3, asgd_lambd=1e-2, asgd_t0=2.0)
+    axs = [np.zeros(p)] * n
+    for t, g in enumerate(_grads(rng, n, p, 20)):
+        xs, axs, c = ea_step_asgd(xs, axs, c, g, hp, t + 1)
+        np.testing.assert_allclose(c, np.mean(xs, axis=0), rtol=0, atol=1e-15)
