@@ -48,8 +48,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
     ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
-    ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw"), default="sgd",
-                    help="local optimizer (BASELINE configs: SGD+momentum; Adam is row f1)")
+    ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw", "asgd"), default="sgd",
+                    help="local optimizer (BASELINE configs: SGD+momentum; Adam(W) and ASGD are row f1)")
     ap.add_argument("--staleness", type=int, choices=(0, 1), default=0,
                     help="1: replicas see the center one step late (row f4; co-located SGD)")
     ap.add_argument("--exchange", choices=("nccl", "p2p"), default="nccl",
@@ -168,9 +168,10 @@ def kernel_name(variant, optimizer, n, staleness=0):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
     if staleness:
         return "colocated_wide<stale>"
-    if n > 8 or (optimizer != "sgd" and n > 6 and variant == "auto"):
+    two_state = optimizer in ("adam", "adamw")
+    if n > 8 or (two_state and n > 6 and variant == "auto"):
         name = "colocated_wide"
-    elif optimizer != "sgd":
+    elif two_state:
         if variant == "auto":
             variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else "bulkpipe")
         name = "colocated_" + variant
@@ -183,25 +184,26 @@ def kernel_name(variant, optimizer, n, staleness=0):
 
 
 def colocated_launches(n, k, args, batched):
-    """Our kernels per co-located step: the fused kernel(s) plus, for Adam, the
-    step-counter kernel that precedes each launch."""
-    adam = args.optimizer != "sgd"
-    per_stage = n > 8 or not batched or (adam and n > 6 and args.variant == "auto") or args.staleness
+    """Our kernels per co-located step: the fused kernel(s) plus, for Adam(W) and
+    ASGD, the step-counter kernel that precedes each launch."""
+    coef = args.optimizer != "sgd"
+    two_state = args.optimizer in ("adam", "adamw")
+    per_stage = n > 8 or not batched or (two_state and n > 6 and args.variant == "auto") or args.staleness
     launches = k if per_stage else (k + 7) // 8
-    return launches * (2 if adam else 1)
+    return launches * (2 if coef else 1)
 
 
 def bytes_colocated(n, p, optimizer="sgd"):
     """Algorithmic HBM bytes of one co-located launch (fp32): read x~ and, per
     replica, x_i, g_i and the optimizer state; write x_i, the state and x~.
-    SGD-momentum (one state vector): (20 N + 8) P; Adam(W) (two): (28 N + 8) P."""
-    return ((20 if optimizer == "sgd" else 28) * n + 8) * p
+    SGD-momentum / ASGD (one state vector): (20 N + 8) P; Adam(W) (two): (28 N + 8) P."""
+    return ((28 if optimizer in ("adam", "adamw") else 20) * n + 8) * p
 
 
 def bytes_spread_local(p, optimizer="sgd"):
     """HBM bytes of the spread local kernel: read x, g, state, x~; write x, state, r:
     28 P (SGD) / 36 P (Adam)."""
-    return (28 if optimizer == "sgd" else 36) * p
+    return (36 if optimizer in ("adam", "adamw") else 28) * p
 
 
 def run_ours(args, rank, world, local):
@@ -224,7 +226,7 @@ def run_ours(args, rank, world, local):
     n = (args.n or cfg.n_pipelines) if not spread else world
     sizes = cfg.stage_sizes
     a, b, r = synth.mode_coeffs(MODE, n)
-    lr = synth.LR if args.optimizer == "sgd" else 1e-3
+    lr = synth.LR if args.optimizer in ("sgd", "asgd") else 1e-3
     stream = torch.cuda.current_stream(dev)
     if spread:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")

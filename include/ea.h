@@ -18,6 +18,11 @@
  *                       m <- b1 m + (1-b1) g';  v <- b2 v + (1-b2) g'^2;
  *                       Delta_i = -(lr/(1-b1^t)) m / (sqrt(v)/sqrt(1-b2^t) + eps)
  *                       (Adam: g' = g + lambda x;  AdamW: g' = g, Delta -= lr lambda x)
+ *                     ASGD (averaged SGD, the AWD-LSTM run's optimizer; torch.optim.ASGD;
+ *                     DESIGN.md c29; t = the stage's step count):
+ *                       eta_t = lr / (1 + l*lr*(t-1))^a;  mu_t = 1 / max(1, t-1-t0)
+ *                       Delta_i = -eta_t * (g + lambda x + l x)      (l = asgd_lambd decay term)
+ *                       ax_i <- mu_t == 1 ? x_i + Delta_i : ax_i + mu_t*(x_i + Delta_i - ax_i)
  *     Step 2  dilution in the ratio (1-alpha):alpha plus the local update:
  *                       x_i <- (1-alpha)*x_i + alpha*x~ + Delta_i
  *     Step 3/4  send and accumulate the contribution
@@ -64,7 +69,7 @@ extern "C" {
 #define EA_API
 #endif
 
-#define EA_ABI_VERSION 3
+#define EA_ABI_VERSION 4
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
@@ -81,8 +86,10 @@ typedef enum {
 typedef enum { EA_COLOCATED = 0, EA_SPREAD = 1 } ea_layout;
 
 /* Local optimizer of Step 1 ("a user-specified optimizer"; the paper
- * trains with Adam and SGD). */
-typedef enum { EA_OPT_SGD = 0, EA_OPT_ADAM = 1, EA_OPT_ADAMW = 2 } ea_optimizer;
+ * trains GNMT/BERT with Adam and AWD with SGD/ASGD).  State slots
+ * (ea_get_state): SGD 1 (momentum), Adam/AdamW 2 (m, v), ASGD 1 (the
+ * average ax). */
+typedef enum { EA_OPT_SGD = 0, EA_OPT_ADAM = 1, EA_OPT_ADAMW = 2, EA_OPT_ASGD = 3 } ea_optimizer;
 
 /* How EA_SPREAD exchanges contributions and the center (rows a6/a7). */
 typedef enum {
@@ -122,7 +129,11 @@ typedef struct {
   int32_t staleness;            /* 0: synchronous center (c3); 1: the replicas see the center one step
                                    late, x~_{t-1}, as with the paper's asynchronous queues (
                                    reading c28, row f4).  1 needs EA_COLOCATED (any optimizer); the
-                                   library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step). */
+                                   library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step).
+                                   SGD, Adam and AdamW only. */
+  double asgd_lambd;            /* ASGD: decay term l >= 0 (torch default 1e-4) */
+  double asgd_alpha;            /* ASGD: power a of the eta schedule (torch default 0.75) */
+  double asgd_t0;               /* ASGD: step after which averaging starts, >= 0 (torch default 1e6) */
 } ea_config;
 
 typedef struct ea_ctx* ea_handle;

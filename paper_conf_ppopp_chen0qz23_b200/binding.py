@@ -21,10 +21,10 @@ EA_COLOCATED, EA_SPREAD = 0, 1
 STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA_ESTATE", 5: "EA_ENOMEM"}
 LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
 VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3}
-OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2}
+OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2, "asgd": 3}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
-ABI_VERSION = 3
+ABI_VERSION = 4
 
 
 class LibraryNotBuilt(RuntimeError):
@@ -60,6 +60,9 @@ class EAConfig(ctypes.Structure):
         ("eps", ctypes.c_float),
         ("exchange", ctypes.c_int32),
         ("staleness", ctypes.c_int32),
+        ("asgd_lambd", ctypes.c_double),
+        ("asgd_alpha", ctypes.c_double),
+        ("asgd_t0", ctypes.c_double),
     ]
 
 
@@ -279,7 +282,8 @@ class ElasticAveraging:
                  weight_decay: float = 0.0, nesterov: bool = False, layout: str = "colocated", rank: int = 0,
                  world: int = 1, device: Optional[int] = None, kernel_variant: str = "auto",
                  nccl_id: Optional[bytes] = None, optimizer: str = "sgd", betas=(0.9, 0.999), eps: float = 1e-8,
-                 exchange: str = "nccl", staleness: int = 0):
+                 exchange: str = "nccl", staleness: int = 0, asgd_lambd: float = 1e-4, asgd_alpha: float = 0.75,
+                 asgd_t0: float = 1e6):
         import torch
         self._lib = load_library()
         self.n = int(n_pipelines)
@@ -294,7 +298,8 @@ class ElasticAveraging:
                        1.0 / self.n if alpha is None else float(alpha), float(beta), float(rho), float(lr),
                        float(momentum), float(weight_decay), int(bool(nesterov)), LAYOUTS[layout], int(rank),
                        int(world), self.device, VARIANTS[kernel_variant], OPTIMIZERS[optimizer],
-                       float(betas[0]), float(betas[1]), float(eps), EXCHANGES[exchange], int(staleness))
+                       float(betas[0]), float(betas[1]), float(eps), EXCHANGES[exchange], int(staleness),
+                       float(asgd_lambd), float(asgd_alpha), float(asgd_t0))
         self._cfg = cfg
         self.rank, self.world = int(rank), int(world)
         idbuf = None
@@ -405,7 +410,7 @@ class ElasticAveraging:
     # -- optimizer state
     def state(self, stage: int, replica: int, slot: int = 0):
         """Zero-copy torch view of library-owned optimizer state: slot 0 = SGD
-        momentum / Adam first moment, slot 1 = Adam second moment."""
+        momentum / Adam first moment / ASGD average ax, slot 1 = Adam second moment."""
         ptr = ctypes.c_void_p()
         _check(self._lib.ea_get_state(self._h, stage, replica, slot, ctypes.byref(ptr)), self._h)
         return _device_view(ptr.value, self.stage_params[stage], self.device)
@@ -430,11 +435,11 @@ class ElasticAveraging:
 
     def set_hyper(self, **kw):
         """Change hyper-parameters (alpha, beta, rho, lr, momentum, weight_decay,
-        nesterov, beta1, beta2, eps) for the steps enqueued afterwards."""
+        nesterov, beta1, beta2, eps, asgd_lambd, asgd_alpha, asgd_t0) for the steps enqueued afterwards."""
         cfg = EAConfig.from_buffer_copy(self._cfg)
         for k, v in kw.items():
             if k not in ("alpha", "beta", "rho", "lr", "momentum", "weight_decay", "nesterov", "beta1", "beta2",
-                         "eps"):
+                         "eps", "asgd_lambd", "asgd_alpha", "asgd_t0"):
                 raise KeyError(k)
             setattr(cfg, k, int(bool(v)) if k == "nesterov" else float(v))
         _check(self._lib.ea_set_hyper(self._h, ctypes.byref(cfg)), self._h)

@@ -141,6 +141,13 @@ ea_status check_hyper(ea_ctx* h, const ea_config& c) {
       return EA_EINVAL;
     }
     if (!(c.eps > 0.f) || !finite(c.eps)) { set_err(h, "Adam eps must be finite and > 0"); return EA_EINVAL; }
+  } else if (c.optimizer == EA_OPT_ASGD) {
+    if (!(c.asgd_lambd >= 0.0 && c.asgd_lambd < 1e30) || !(c.asgd_alpha >= 0.0 && c.asgd_alpha < 1e30) ||
+        !(c.asgd_t0 >= 0.0 && c.asgd_t0 < 1e300)) {
+      set_err(h, "ASGD lambd, alpha, t0 must be finite and >= 0, got %g, %g, %g", c.asgd_lambd, c.asgd_alpha,
+              c.asgd_t0);
+      return EA_EINVAL;
+    }
   } else {
     set_err(h, "unknown optimizer %d", c.optimizer);
     return EA_EINVAL;
@@ -157,13 +164,14 @@ ea::Hyper make_hyper(const ea_config& c) {
   hp.beta2 = static_cast<float>(c.beta2); hp.one_minus_beta2 = static_cast<float>(1.0 - c.beta2);
   hp.eps = c.eps;
   hp.lr_wd = static_cast<float>((double)c.lr * (double)c.weight_decay);
+  hp.asgd_lambd = static_cast<float>(c.asgd_lambd);
   return hp;
 }
 
-int state_slots(const ea_ctx* h) { return h->cfg.optimizer == EA_OPT_SGD ? 1 : 2; }
+int state_slots(const ea_ctx* h) { return ea::two_state(h->cfg.optimizer) ? 2 : 1; }
 
 // Device step counters are needed when a kernel consumes the step count:
-// Adam's bias correction and the peer-memory exchange's epoch.
+// Adam's bias correction, ASGD's eta_t / mu_t and the peer-memory exchange's epoch.
 bool device_steps(const ea_ctx* h) {
   return h->cfg.optimizer != EA_OPT_SGD || (h->cfg.layout == EA_SPREAD && h->cfg.exchange == EA_XCHG_P2P);
 }
@@ -187,7 +195,11 @@ ea_status advance(ea_ctx* h, const int32_t* stages, int count, cudaStream_t s) {
     ea::StageList l;
     l.count = 0;
     for (int j = j0; j < count && j < j0 + 8; ++j) l.idx[l.count++] = stages[j];
-    cudaError_t e = ea::launch_advance_steps(h->d_steps, h->d_coef, l, h->cfg.beta1, h->cfg.beta2, (double)h->cfg.lr, s);
+    ea::CoefParams cp;
+    cp.opt = h->cfg.optimizer;
+    cp.beta1 = h->cfg.beta1; cp.beta2 = h->cfg.beta2; cp.lr = (double)h->cfg.lr;
+    cp.lambd = h->cfg.asgd_lambd; cp.asgd_alpha = h->cfg.asgd_alpha; cp.t0 = h->cfg.asgd_t0;
+    cudaError_t e = ea::launch_advance_steps(h->d_steps, h->d_coef, l, cp, s);
     if (e != cudaSuccess) return cuda_fail(h, e, "step-counter kernel launch");
   }
   return EA_OK;
@@ -268,7 +280,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   }();
   // Adam with N > 6: the replica-loop kernel measured fastest (0.919 of peak at N = 8 vs 0.75 bulk-copy
   // pipeline and 0.73 lane kernel, profiles/r01_adam_nsweep.jsonl)
-  const bool adam_wide = opt != EA_OPT_SGD && n > 6 && h->variant == 0;
+  const bool adam_wide = ea::two_state(opt) && n > 6 && h->variant == 0;
   const bool stale = h->cfg.staleness == 1;
   if (n > ea::kMaxFusedN || force_wide || adam_wide || stale) {  // replica loop: one launch per stage
     for (int j = 0; j < count; ++j) {
@@ -569,6 +581,10 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     set_err(nullptr, "staleness 1 is supported for EA_COLOCATED");
     return EA_EINVAL;
   }
+  if (c.staleness == 1 && c.optimizer == EA_OPT_ASGD) {
+    set_err(nullptr, "staleness 1 supports SGD, Adam and AdamW");
+    return EA_EINVAL;
+  }
   if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {
     set_err(nullptr, "peer-memory exchange supports world <= %d", ea::kMaxWorld);
     return EA_EINVAL;
@@ -808,7 +824,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
       if ((e = cudaEventRecord(h->ev_h2d[b], h->h2d)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
       if ((e = cudaStreamWaitEvent(s, h->ev_h2d[b], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
       // the fused step on [off, off+len) of the stage (elementwise: any chunk is a valid sub-problem)
-      if (n > ea::kMaxFusedN || (opt != EA_OPT_SGD && n > 6 && h->variant == 0)) {
+      if (n > ea::kMaxFusedN || (ea::two_state(opt) && n > 6 && h->variant == 0)) {
         ea::ReplicaTable t;
         for (int i = 0; i < n; ++i) {
           t.x[i] = replica_ptrs[(size_t)j * n + i] + off;
@@ -1038,6 +1054,7 @@ ea_status ea_set_hyper(ea_handle h, const ea_config* cfg) {
   c.alpha = cfg->alpha; c.beta = cfg->beta; c.rho = cfg->rho; c.lr = cfg->lr;
   c.momentum = cfg->momentum; c.weight_decay = cfg->weight_decay; c.nesterov = cfg->nesterov;
   c.beta1 = cfg->beta1; c.beta2 = cfg->beta2; c.eps = cfg->eps;
+  c.asgd_lambd = cfg->asgd_lambd; c.asgd_alpha = cfg->asgd_alpha; c.asgd_t0 = cfg->asgd_t0;
   h->cfg = c;
   h->hp = make_hyper(c);
   return EA_OK;

@@ -7,8 +7,14 @@
 
 namespace ea {
 
-// Local optimizer of Step 1 (DESIGN.md c7 SGD-momentum, c21 Adam/AdamW).
-enum Opt : int { kOptSGD = 0, kOptAdam = 1, kOptAdamW = 2 };
+// Local optimizer of Step 1 (DESIGN.md c7 SGD-momentum, c21 Adam/AdamW, c29 ASGD).
+enum Opt : int { kOptSGD = 0, kOptAdam = 1, kOptAdamW = 2, kOptASGD = 3 };
+
+// Adam(W) keep two state vectors (m, v); SGD-momentum and ASGD one (momentum / the average ax), so they
+// move the same bytes and share the kernels' 3-stream geometry.
+constexpr bool two_state(int opt) { return opt == kOptAdam || opt == kOptAdamW; }
+// Optimizers with per-step coefficients (StepCoef): Adam(W)'s bias corrections, ASGD's eta_t and mu_t.
+constexpr bool has_coef(int opt) { return opt != kOptSGD; }
 
 // Hyper-parameters in the form the kernels consume (fp32).
 struct Hyper {
@@ -24,6 +30,7 @@ struct Hyper {
   float beta2, one_minus_beta2;
   float eps;
   float lr_wd;     // lr * wd (AdamW decoupled decay)
+  float asgd_lambd;  // ASGD decay term l (Delta = -eta_t (g + wd x + l x))
 };
 
 // Per-stage Adam bias corrections for the step being taken (t = the stage's
@@ -31,8 +38,15 @@ struct Hyper {
 // stream right before the step's kernel, so a captured CUDA graph advances t
 // on every replay.
 struct StepCoef {
-  float step_size;     // lr / (1 - beta1^t)
-  float inv_sqrt_bc2;  // 1 / sqrt(1 - beta2^t)
+  float step_size;     // Adam: lr / (1 - beta1^t);     ASGD: eta_t = lr / (1 + l lr (t-1))^a
+  float inv_sqrt_bc2;  // Adam: 1 / sqrt(1 - beta2^t);  ASGD: mu_t = 1 / max(1, t-1-t0)
+};
+
+// What advance_steps needs to compute StepCoef for the handle's optimizer.
+struct CoefParams {
+  int opt;
+  double beta1, beta2, lr;          // Adam(W)
+  double lambd, asgd_alpha, t0;     // ASGD
 };
 
 // Stage list of one advance_steps launch.
@@ -42,8 +56,8 @@ struct StageList {
 };
 
 // On `s`: for every listed stage, ++steps[stage] and recompute coef[stage] (double precision).
-cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, double beta1, double beta2,
-                                 double lr, cudaStream_t s);
+cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, const CoefParams& cp,
+                                 cudaStream_t s);
 
 constexpr int kMaxReplicas = 64;      // EA_MAX_REPLICAS
 constexpr int kMaxFusedN = 8;         // replicas handled by the compile-time-N kernels

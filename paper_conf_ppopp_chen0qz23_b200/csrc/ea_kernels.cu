@@ -74,7 +74,7 @@ struct Mem {
 
 // ---------------------------------------------------------------- the math
 // One (replica, element) update; returns the replica's contribution r_i.
-// m: SGD momentum / Adam first moment; v: Adam second moment (SGD: untouched).
+// m: SGD momentum / Adam first moment / ASGD average; v: Adam second moment (SGD, ASGD: untouched).
 template <int OPT>
 __device__ __forceinline__ float ea_elem(float& x, float g, float& m, float& v, float c, const Hyper& hp,
                                          const StepCoef& sc) {
@@ -85,6 +85,13 @@ __device__ __forceinline__ float ea_elem(float& x, float g, float& m, float& v, 
     const float d = hp.nesterov ? fmaf(hp.momentum, mn, gg) : mn;
     delta = -hp.lr * d;                             // local update Delta_i (Step 1)
     m = mn;
+  } else if constexpr (OPT == kOptASGD) {
+    // torch.optim.ASGD (reading c29): x_local = x (1 - l eta_t) - eta_t g', so Delta = -eta_t (g' + l x);
+    // the average tracks the optimizer's own iterate x + Delta (mu_t == 1: a copy, as torch does)
+    const float gg = fmaf(hp.wd, x, g);
+    delta = -sc.step_size * fmaf(hp.asgd_lambd, x, gg);
+    const float xl = x + delta;
+    m = sc.inv_sqrt_bc2 == 1.f ? xl : fmaf(sc.inv_sqrt_bc2, xl - m, m);
   } else {
     const float gg = OPT == kOptAdam ? fmaf(hp.wd, x, g) : g;
     const float mn = fmaf(hp.beta1, m, hp.one_minus_beta1 * gg);
@@ -138,11 +145,11 @@ __device__ void stage_tail(const StageRefs& st, const Hyper& hp) {
     float acc = 0.f;
 #pragma unroll
     for (int i = 0; i < N; ++i) {
-      float x = st.x[i][j], m = st.m[i][j], v = OPT == kOptSGD ? 0.f : st.v[i][j];
+      float x = st.x[i][j], m = st.m[i][j], v = two_state(OPT) ? st.v[i][j] : 0.f;
       acc += ea_elem<OPT>(x, st.g[i][j], m, v, c, hp, sc);
       st.x[i][j] = x;
       st.m[i][j] = m;
-      if (OPT != kOptSGD) st.v[i][j] = v;
+      if (two_state(OPT)) st.v[i][j] = v;
     }
     st.c[j] = fmaf(acc, hp.inv_n, c);
   }
@@ -208,7 +215,7 @@ __device__ __forceinline__ bool wave_item(const StageBatch& b, int64_t C, WaveCu
 template <int N, int U, int HINT, int OPT>
 __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, int64_t ve, const Hyper& hp,
                                               const Mem<HINT>& mem, const StepCoef& sc) {
-  constexpr bool kTwo = OPT != kOptSGD;  // Adam(W): second moment v
+  constexpr bool kTwo = two_state(OPT);  // Adam(W): second moment v
   for (int64_t base = va + threadIdx.x; base < ve; base += (int64_t)kThreads * U) {
     float4 c[U], x[N][U], g[N][U], m[N][U], w[kTwo ? N : 1][U];
     bool ok[U];
@@ -256,7 +263,7 @@ __device__ __forceinline__ void regloop_range(const StageRefs& st, int64_t va, i
 // spill 120 B).
 template <int N, int OPT>
 constexpr int regloop_min_blocks() {
-  return (OPT != kOptSGD && N == 5) ? 2 : 0;  // 0: no minimum (ptxas default heuristics)
+  return (two_state(OPT) && N == 5) ? 2 : 0;  // 0: no minimum (ptxas default heuristics)
 }
 
 template <int N, int U, int HINT, int OPT>
@@ -264,7 +271,7 @@ __global__ void __launch_bounds__(kThreads, regloop_min_blocks<N, OPT>()) coloca
                                                                                             const Hyper hp) {
   const Mem<HINT> mem;
   __shared__ StepCoef s_coef[kMaxLaunchStages];
-  if (OPT != kOptSGD) {
+  if (has_coef(OPT)) {
     if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
     __syncthreads();
   }
@@ -272,7 +279,7 @@ __global__ void __launch_bounds__(kThreads, regloop_min_blocks<N, OPT>()) coloca
   int s;
   int64_t v0, nv;
   while (wave_item(b, (int64_t)kThreads * U, cur, s, v0, nv))
-    regloop_range<N, U, HINT, OPT>(b.st[s], v0, v0 + nv, hp, mem, OPT == kOptSGD ? StepCoef{0.f, 0.f} : s_coef[s]);
+    regloop_range<N, U, HINT, OPT>(b.st[s], v0, v0 + nv, hp, mem, has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f});
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
@@ -292,7 +299,7 @@ __device__ __forceinline__ void wide_load(const ReplicaTable& t, int i, int64_t 
       r.x[u] = mem.ld(t.x[i] + 4 * v);
       r.g[u] = mem.ld_ro(t.g[i] + 4 * v);
       r.m[u] = mem.ld(t.m[i] + 4 * v);
-      if (OPT != kOptSGD) r.w[u] = mem.ld(t.v[i] + 4 * v);
+      if (two_state(OPT)) r.w[u] = mem.ld(t.v[i] + 4 * v);
     }
   }
 }
@@ -308,7 +315,7 @@ __device__ __forceinline__ void wide_proc(const ReplicaTable& t, int i, int64_t 
     add4(acc[u], ea_vec<OPT>(r.x[u], r.g[u], r.m[u], r.w[u], cu[u], hp, sc));
     mem.st(t.x[i] + 4 * v, r.x[u]);
     mem.st(t.m[i] + 4 * v, r.m[u]);
-    if (OPT != kOptSGD) mem.st(t.v[i] + 4 * v, r.w[u]);
+    if (two_state(OPT)) mem.st(t.v[i] + 4 * v, r.w[u]);
   }
 }
 
@@ -369,11 +376,11 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
       const float cused = stale ? prev[j] : c;
       float acc = 0.f;
       for (int i = 0; i < n; ++i) {
-        float x = t.x[i][j], m = t.m[i][j], v = OPT == kOptSGD ? 0.f : t.v[i][j];
+        float x = t.x[i][j], m = t.m[i][j], v = two_state(OPT) ? t.v[i][j] : 0.f;
         acc += ea_elem<OPT>(x, t.g[i][j], m, v, cused, hp, sc);
         t.x[i][j] = x;
         t.m[i][j] = m;
-        if (OPT != kOptSGD) t.v[i][j] = v;
+        if (two_state(OPT)) t.v[i][j] = v;
       }
       center[j] = fmaf(acc, hp.inv_n, c);
       if (stale) prev[j] = c;
@@ -449,7 +456,7 @@ template <int N, int HINT, int OPT, int PASSES = kLanePasses, int MINB = 1>
 __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const StageBatch b, const Hyper hp) {
   using G = LaneGeom<N, PASSES>;
   constexpr int CH = G::CH, kPasses = PASSES, kVecPerWarp = G::kVecPerWarp, kTileVec = G::kTileVec;
-  constexpr bool kTwoState = OPT != kOptSGD;
+  constexpr bool kTwoState = two_state(OPT);
   __shared__ __align__(128) float4 s_center[2][kTileVec];
   __shared__ __align__(8) uint64_t s_bar[2];
   const Mem<HINT> mem;
@@ -464,7 +471,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
     mbar_init(&s_bar[1], 1);
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (kTwoState && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+  if (has_coef(OPT) && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
   __syncthreads();
 
   auto issue = [&](int s, int64_t v0, int64_t nv, int buf) {
@@ -488,7 +495,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       issue(s_next, v0_next, nv_next, buf ^ 1);
     }
     const StageRefs& st = b.st[s];
-    const StepCoef sc = kTwoState ? s_coef[s] : StepCoef{0.f, 0.f};
+    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
     float* xi = nullptr;
     const float* gi = nullptr;
     float* mi = nullptr;
@@ -593,11 +600,11 @@ template <int OPT>
 __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
   const StepCoef sc = load_coef<OPT>(st.scp);
   for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
-    float x = st.x[0][j], m = st.m[0][j], v = OPT == kOptSGD ? 0.f : st.v[0][j];
+    float x = st.x[0][j], m = st.m[0][j], v = two_state(OPT) ? st.v[0][j] : 0.f;
     contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
     st.x[0][j] = x;
     st.m[0][j] = m;
-    if (OPT != kOptSGD) st.v[0][j] = v;
+    if (two_state(OPT)) st.v[0][j] = v;
   }
   for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
 }
@@ -607,7 +614,7 @@ __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, 
 template <int N, int HINT, int OPT, int TILE, bool SPREAD>
 __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& hp, float* __restrict__ contrib,
                                               int64_t p_pad, int issue_lanes) {
-  constexpr int A = OPT == kOptSGD ? 3 : 4;
+  constexpr int A = two_state(OPT) ? 4 : 3;
   using G = BulkGeom<N, TILE, A>;
   constexpr int T = G::kTile, S = G::kStages;
   extern __shared__ __align__(128) float4 smem[];
@@ -624,7 +631,7 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
-  if (OPT != kOptSGD && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+  if (has_coef(OPT) && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
   __syncthreads();
 
   if (warp == kBulkConsumerWarps) {
@@ -664,7 +671,7 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
       mbar_wait(&full[slot], (k / S) & 1);
       const float4* base = smem + slot * G::kSlotVec;
       const StageRefs& st = b.st[s];
-      const StepCoef sc = OPT == kOptSGD ? StepCoef{0.f, 0.f} : s_coef[s];
+      const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
       for (int lv = threadIdx.x; lv < nv; lv += 32 * kBulkConsumerWarps) {
         const float4 c = base[lv];
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -739,7 +746,7 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
           xv[u] = mem.ld(x + 4 * v);
           gv[u] = mem.ld_ro(g + 4 * v);
           mv[u] = mem.ld(m + 4 * v);
-          if (OPT != kOptSGD) wv[u] = mem.ld(vs + 4 * v);
+          if (two_state(OPT)) wv[u] = mem.ld(vs + 4 * v);
           cv[u] = mem.ld_ro(center + 4 * v);
         }
       }
@@ -750,7 +757,7 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
           const float4 r = ea_vec<OPT>(xv[u], gv[u], mv[u], wv[u], cv[u], hp, sc);
           mem.st(x + 4 * v, xv[u]);
           mem.st(m + 4 * v, mv[u]);
-          if (OPT != kOptSGD) mem.st(vs + 4 * v, wv[u]);
+          if (two_state(OPT)) mem.st(vs + 4 * v, wv[u]);
           mem.st(contrib + 4 * v, r);
         }
       }
@@ -761,11 +768,11 @@ __global__ void __launch_bounds__(kThreads) spread_local(float* __restrict__ x, 
   const int64_t gsz = (int64_t)gridDim.x * kThreads;
   for (int64_t j = 4 * nvec + gtid; j < p_pad; j += gsz) {
     if (j < p) {
-      float xs = x[j], ms = m[j], ws = OPT == kOptSGD ? 0.f : vs[j];
+      float xs = x[j], ms = m[j], ws = two_state(OPT) ? vs[j] : 0.f;
       contrib[j] = ea_elem<OPT>(xs, g[j], ms, ws, center[j], hp, sc);
       x[j] = xs;
       m[j] = ms;
-      if (OPT != kOptSGD) vs[j] = ws;
+      if (two_state(OPT)) vs[j] = ws;
     } else {
       contrib[j] = 0.f;
     }
@@ -842,11 +849,11 @@ int regloop_u1() {
   return v;
 }
 
-template <int N, int HINT>
+template <int N, int HINT, int OPT = kOptSGD>
 cudaError_t launch_regloop(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   constexpr int U = N <= 2 ? 4 : (N <= 4 ? 2 : 1);
-  if (U > 1 && regloop_u1()) return launch_regloop_u<N, HINT, 1>(b, hp, num_sms, s);
-  return launch_regloop_u<N, HINT, U>(b, hp, num_sms, s);
+  if (U > 1 && regloop_u1()) return launch_regloop_u<N, HINT, 1, OPT>(b, hp, num_sms, s);
+  return launch_regloop_u<N, HINT, U, OPT>(b, hp, num_sms, s);
 }
 
 // Tuning knob for measurement: AVGPIPE_EA_LANE_TUNE=<passes><minblocks>: "23", "24", "81" (N=4,
@@ -900,7 +907,7 @@ int bulk_issue_lanes() {
 
 template <int N, int HINT, int OPT, int TILE>
 cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using G = BulkGeom<N, TILE, OPT == kOptSGD ? 3 : 4>;
+  using G = BulkGeom<N, TILE, two_state(OPT) ? 4 : 3>;
   auto k = colocated_bulkpipe<N, HINT, OPT, TILE>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
   if (e != cudaSuccess) return e;
@@ -922,7 +929,7 @@ int bulk_tile() {
 
 template <int N, int HINT, int OPT>
 cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  constexpr int A = OPT == kOptSGD ? 3 : 4;
+  constexpr int A = two_state(OPT) ? 4 : 3;
   if constexpr (HINT == 0) {
     switch (bulk_tile()) {
       case 64: return launch_bulkpipe_t<N, HINT, OPT, 64>(b, hp, num_sms, s);
@@ -941,6 +948,11 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
 
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (opt == kOptASGD) {  // SGD's streams and geometry (one state vector), no L2-hint variants
+    if (variant == kVariantBulkPipe) return launch_bulkpipe<N, 0, kOptASGD>(b, hp, num_sms, s);
+    if (variant == kVariantRegLoop) return launch_regloop<N, 0, kOptASGD>(b, hp, num_sms, s);
+    return launch_laneshfl<N, 0, kOptASGD>(b, hp, num_sms, s);
+  }
   if (opt != kOptSGD && variant == kVariantRegLoop)
     return opt == kOptAdam ? launch_regloop_u<N, 0, 1, kOptAdam>(b, hp, num_sms, s)
                            : launch_regloop_u<N, 0, 1, kOptAdamW>(b, hp, num_sms, s);
@@ -982,7 +994,7 @@ template <int OPT>
 cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
                                int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
                                cudaStream_t s) {
-  constexpr int A = OPT == kOptSGD ? 3 : 4;
+  constexpr int A = two_state(OPT) ? 4 : 3;
   constexpr int TILE = default_bulk_tile<1, A>();
   using G = BulkGeom<1, TILE, A>;
   auto k = spread_bulkpipe<OPT, TILE>;
@@ -1012,7 +1024,7 @@ cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v
                                     float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
   if (!spread_reg()) return launch_spread_bulk<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
-  constexpr int U = OPT == kOptSGD ? 4 : 2;
+  constexpr int U = two_state(OPT) ? 2 : 4;
   const int64_t nvec = p / 4;
   auto k = spread_local<U, OPT>;
   int64_t units = (nvec + kThreads * U - 1) / (kThreads * U);
@@ -1021,25 +1033,32 @@ cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v
   return cudaGetLastError();
 }
 
-// Step counter + Adam bias corrections, on the stream (graph-capturable).
-__global__ void advance_steps(int64_t* steps, StepCoef* coef, const StageList list, double beta1, double beta2,
-                              double lr) {
+// Step counter + the step's coefficients, on the stream (graph-capturable): Adam(W) bias corrections, or
+// ASGD's eta_t and mu_t (torch.optim.ASGD's state after t-1 steps: eta = lr / (1 + l lr (t-1))^a,
+// mu = 1 / max(1, t-1-t0); eta_1 = lr, mu_1 = 1).
+__global__ void advance_steps(int64_t* steps, StepCoef* coef, const StageList list, const CoefParams cp) {
   const int i = threadIdx.x;
   if (i >= list.count) return;
   const int s = list.idx[i];
   const int64_t t = ++steps[s];
-  const double bc1 = 1.0 - pow(beta1, (double)t);
-  const double bc2 = 1.0 - pow(beta2, (double)t);
-  coef[s].step_size = bc1 > 0.0 ? static_cast<float>(lr / bc1) : 0.f;
+  if (cp.opt == kOptASGD) {
+    const double k = (double)(t - 1);
+    coef[s].step_size = static_cast<float>(cp.lr / pow(1.0 + cp.lambd * cp.lr * k, cp.asgd_alpha));
+    coef[s].inv_sqrt_bc2 = static_cast<float>(1.0 / fmax(1.0, k - cp.t0));
+    return;
+  }
+  const double bc1 = 1.0 - pow(cp.beta1, (double)t);
+  const double bc2 = 1.0 - pow(cp.beta2, (double)t);
+  coef[s].step_size = bc1 > 0.0 ? static_cast<float>(cp.lr / bc1) : 0.f;
   coef[s].inv_sqrt_bc2 = bc2 > 0.0 ? static_cast<float>(1.0 / sqrt(bc2)) : 0.f;
 }
 
 }  // namespace
 
-cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, double beta1, double beta2,
-                                 double lr, cudaStream_t s) {
+cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, const CoefParams& cp,
+                                 cudaStream_t s) {
   if (list.count <= 0) return cudaSuccess;
-  advance_steps<<<1, 32, 0, s>>>(steps, coef, list, beta1, beta2, lr);
+  advance_steps<<<1, 32, 0, s>>>(steps, coef, list, cp);
   return cudaGetLastError();
 }
 
@@ -1052,7 +1071,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // N = 8 (0.98-0.99).  Adam(W): the lane kernel for N = 1 (0.915), the register loop for N = 2, 3 (0.96 /
   // 0.95; bulk pipeline 0.88 / 0.90), the bulk-copy pipeline for N = 4..6 (0.97 / 0.95 / 0.93); N > 6 goes to
   // the replica-loop kernel (ea_api.cu)
-  if (variant == kVariantAuto && opt != kOptSGD)
+  if (variant == kVariantAuto && two_state(opt))
     variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : kVariantBulkPipe);
   if (variant == kVariantAuto)
     variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
@@ -1074,6 +1093,7 @@ cudaError_t launch_colocated_wide(const ReplicaTable& t, int n, float* center, f
   if (p <= 0) return cudaSuccess;
   if (opt == kOptAdam) return launch_wide_opt<kOptAdam>(t, n, center, prev, p, hp, sc, num_sms, s);
   if (opt == kOptAdamW) return launch_wide_opt<kOptAdamW>(t, n, center, prev, p, hp, sc, num_sms, s);
+  if (opt == kOptASGD) return launch_wide_opt<kOptASGD>(t, n, center, prev, p, hp, sc, num_sms, s);
   return launch_wide_opt<kOptSGD>(t, n, center, prev, p, hp, sc, num_sms, s);
 }
 
@@ -1085,6 +1105,8 @@ cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, co
     return launch_spread_local_opt<kOptAdam>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   if (opt == kOptAdamW)
     return launch_spread_local_opt<kOptAdamW>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+  if (opt == kOptASGD)
+    return launch_spread_local_opt<kOptASGD>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   return launch_spread_local_opt<kOptSGD>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
 }
 

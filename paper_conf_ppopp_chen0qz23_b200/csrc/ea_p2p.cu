@@ -68,6 +68,11 @@ __device__ __forceinline__ float p2p_elem(float& x, float g, float& m, float& v,
     const float d = hp.nesterov ? fmaf(hp.momentum, mn, gg) : mn;
     delta = -hp.lr * d;
     m = mn;
+  } else if constexpr (OPT == kOptASGD) {  // reading c29, as ea_elem
+    const float gg = fmaf(hp.wd, x, g);
+    delta = -sc.step_size * fmaf(hp.asgd_lambd, x, gg);
+    const float xl = x + delta;
+    m = sc.inv_sqrt_bc2 == 1.f ? xl : fmaf(sc.inv_sqrt_bc2, xl - m, m);
   } else {
     const float gg = OPT == kOptAdam ? fmaf(hp.wd, x, g) : g;
     const float mn = fmaf(hp.beta1, m, hp.one_minus_beta1 * gg);
@@ -104,7 +109,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
   const int N = a.world, r = a.rank;
   const float inv_n = a.hp.inv_n;
   const uint32_t epoch = static_cast<uint32_t>(*a.stepp);
-  const StepCoef sc = OPT == kOptSGD ? StepCoef{0.f, 0.f} : *a.scp;
+  const StepCoef sc = has_coef(OPT) ? *a.scp : StepCoef{0.f, 0.f};
 
   // ---------------- Phase A: local update, push contributions to the owners
   for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
@@ -118,25 +123,25 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
       float4 rv;
       if (j + 3 < a.p) {
         float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
-        float4 w = OPT == kOptSGD ? make_float4(0.f, 0.f, 0.f, 0.f) : ld4(a.v + j);
+        float4 w = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
         rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
         rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
         rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
         rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
         st4(a.x + j, x);
         st4(a.m + j, m);
-        if (OPT != kOptSGD) st4(a.v + j, w);
+        if (two_state(OPT)) st4(a.v + j, w);
       } else {  // the ragged end of the replica and the zero padding of the center
         float rr[4];
         for (int q = 0; q < 4; ++q) {
           const int64_t jj = j + q;
           rr[q] = 0.f;
           if (jj < a.p) {
-            float x = a.x[jj], m = a.m[jj], w = OPT == kOptSGD ? 0.f : a.v[jj];
+            float x = a.x[jj], m = a.m[jj], w = two_state(OPT) ? a.v[jj] : 0.f;
             rr[q] = p2p_elem<OPT>(x, a.g[jj], m, w, a.center[jj], a.hp, sc);
             a.x[jj] = x;
             a.m[jj] = m;
-            if (OPT != kOptSGD) a.v[jj] = w;
+            if (two_state(OPT)) a.v[jj] = w;
           }
         }
         rv = make_float4(rr[0], rr[1], rr[2], rr[3]);
@@ -205,6 +210,7 @@ cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int m
   if (grid < 1) grid = 1;
   if (opt == kOptAdam) spread_p2p<kOptAdam><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
   else if (opt == kOptAdamW) spread_p2p<kOptAdamW><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
+  else if (opt == kOptASGD) spread_p2p<kOptASGD><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
   else spread_p2p<kOptSGD><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
   return cudaGetLastError();
 }
@@ -222,6 +228,7 @@ int blocks_per_sm_t() {
 // exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
 int p2p_blocks_per_sm(int opt) {
   if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD>();
+  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD>();
   return opt == kOptAdam ? blocks_per_sm_t<kOptAdam>() : blocks_per_sm_t<kOptAdamW>();
 }
 

@@ -12,7 +12,7 @@ from __future__ import annotations
 
 import numpy as np
 
-from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_adam_stale, ea_step_stale
+from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_adam_stale, ea_step_asgd, ea_step_stale
 from paper_conf_ppopp_chen0qz23_b200 import synth
 
 TOL = 1e-5
@@ -37,21 +37,30 @@ def f32(v: float) -> float:
     return float(np.float32(v))
 
 
+ASGD_TEST = dict(asgd_lambd=1e-2, asgd_alpha=0.75, asgd_t0=5.0)   # averaging starts within a short test
+
+
 def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nesterov=False, betas=(0.9, 0.999),
-          eps=1e-8):
+          eps=1e-8, asgd=ASGD_TEST):
     """Oracle hyper-parameters equal to what the ABI carries (reading c12: the
     oracle consumes the same fp32 values upcast): alpha, beta, rho, lr,
     momentum, weight_decay, eps are float32 fields; beta1/beta2 are double.
     (Adam's Delta = -lr m/(sqrt(v)+eps) has slope ~lr/eps where the gradient
     is near 0, so the 2e-10 relative gap between 0.01 and float32(0.01) alone
-    moves such an element by ~1e-5 of rms(x).)"""
+    moves such an element by ~1e-5 of rms(x).)  The ASGD fields are double."""
     a, b, r = synth.mode_coeffs(mode, n, alpha)
     return Hyper(alpha=f32(a), beta=f32(b), rho=f32(r), lr=f32(lr), momentum=f32(momentum), weight_decay=f32(wd),
-                 nesterov=nesterov, beta1=betas[0], beta2=betas[1], eps=f32(eps))
+                 nesterov=nesterov, beta1=betas[0], beta2=betas[1], eps=f32(eps), **asgd)
+
+
+def asgd_kw(hp):
+    """ElasticAveraging keyword arguments carrying hp's ASGD fields."""
+    return dict(asgd_lambd=hp.asgd_lambd, asgd_alpha=hp.asgd_alpha, asgd_t0=hp.asgd_t0)
 
 
 class OracleStage:
-    """float64 oracle state of one stage (optimizer 'sgd' | 'adam' | 'adamw')."""
+    """float64 oracle state of one stage (optimizer 'sgd' | 'adam' | 'adamw' | 'asgd'; ms holds the
+    momentum / first moment / ASGD average)."""
 
     def __init__(self, reps, center, optimizer="sgd", staleness=0):
         self.xs = [np.asarray(x, dtype=np.float64) for x in reps]
@@ -72,6 +81,8 @@ class OracleStage:
                 self.xs, self.ms, self.vs, self.c, self.c_prev, grads, hp, self.t, decoupled=self.opt == "adamw")
         elif self.opt == "sgd":
             self.xs, self.ms, self.c = ea_step(self.xs, self.ms, self.c, grads, hp)
+        elif self.opt == "asgd":
+            self.xs, self.ms, self.c = ea_step_asgd(self.xs, self.ms, self.c, grads, hp, self.t)
         else:
             self.xs, self.ms, self.vs, self.c = ea_step_adam(self.xs, self.ms, self.vs, self.c, grads, hp, self.t,
                                                              decoupled=self.opt == "adamw")

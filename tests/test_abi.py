@@ -51,20 +51,36 @@ def test_abi_version(lib):
     assert lib.ea_abi_version() == binding.ABI_VERSION
 
 
-def test_config_struct_layout_matches_header():
-    # ea_config: 2 x int32, pointer, 6 floats, 7 int32, [pad], 2 doubles, float, 2 int32, [pad] (x86-64)
-    assert ctypes.sizeof(binding.EAConfig) == 104
-    assert binding.EAConfig.beta1.offset == 72 and binding.EAConfig.eps.offset == 88
-    assert binding.EAConfig.exchange.offset == 92 and binding.EAConfig.staleness.offset == 96
-    assert binding.EAConfig.stage_params.offset == 8
-    assert ctypes.sizeof(binding.EAOp) == 8
+def test_config_struct_layout_matches_header(tmp_path):
+    """ctypes' ea_config / ea_op layout == what the C compiler makes of include/ea.h (sizeof and the
+    offset of every field)."""
+    import shutil
+    import subprocess
+    if shutil.which("gcc") is None:
+        pytest.skip("gcc not available")
+    fields = [f for f, _ in binding.EAConfig._fields_]
+    src = ['#include <stddef.h>', '#include <stdio.h>', '#include "ea.h"', "int main(void) {",
+           '  printf("size %zu\\n", sizeof(ea_config));', '  printf("op %zu\\n", sizeof(ea_op));']
+    src += [f'  printf("{f} %zu\\n", offsetof(ea_config, {f}));' for f in fields]
+    src += ["  return 0;", "}"]
+    (tmp_path / "layout.c").write_text("\n".join(src) + "\n")
+    exe = tmp_path / "layout"
+    subprocess.run(["gcc", "-std=c99", "-I", os.path.join(ROOT, "include"), str(tmp_path / "layout.c"), "-o",
+                    str(exe)], check=True)
+    got = dict(line.split() for line in subprocess.run([str(exe)], capture_output=True, text=True,
+                                                       check=True).stdout.splitlines())
+    assert int(got["size"]) == ctypes.sizeof(binding.EAConfig)
+    assert int(got["op"]) == ctypes.sizeof(binding.EAOp)
+    for f in fields:
+        assert int(got[f]) == getattr(binding.EAConfig, f).offset, f
 
 
 def _cfg(**kw):
     sp = (ctypes.c_int64 * 2)(1000, 1001)
     base = dict(n_pipelines=2, n_stages=2, stage_params=sp, alpha=0.5, beta=0.0, rho=1.0, lr=0.05, momentum=0.9,
                 weight_decay=0.0, nesterov=0, layout=0, rank=0, world=1, device=0, kernel_variant=0, optimizer=0,
-                beta1=0.9, beta2=0.999, eps=1e-8, exchange=0, staleness=0)
+                beta1=0.9, beta2=0.999, eps=1e-8, exchange=0, staleness=0, asgd_lambd=1e-4, asgd_alpha=0.75,
+                asgd_t0=1e6)
     base.update(kw)
     c = binding.EAConfig(**base)
     c._keep = sp
@@ -86,7 +102,11 @@ def _cfg(**kw):
     (dict(kernel_variant=9), "kernel_variant"),
     (dict(n_pipelines=65), "N must be"),
     (dict(lr=float("nan")), "finite"),
-    (dict(optimizer=3), "optimizer"),
+    (dict(optimizer=4), "optimizer"),
+    (dict(optimizer=3, asgd_lambd=-1.0), "ASGD"),
+    (dict(optimizer=3, asgd_t0=float("nan")), "ASGD"),
+    (dict(optimizer=3, asgd_alpha=float("inf")), "ASGD"),
+    (dict(optimizer=3, staleness=1), "staleness 1 supports"),
     (dict(exchange=5), "exchange"),
     (dict(staleness=2), "staleness"),
     (dict(staleness=1, layout=1, world=2, rank=0), "staleness 1"),

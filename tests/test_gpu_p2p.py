@@ -16,19 +16,19 @@ import torch
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import EAError, ElasticAveraging
 from paper_conf_ppopp_chen0qz23_b200.parallel import replica_of
-from tests._parity import TOL, OracleStage, hyper, rel_err, to_np
+from tests._parity import TOL, OracleStage, asgd_kw, hyper, rel_err, to_np
 
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
 def _run(n, sizes, steps, mode, optimizer="sgd", stage_order=None):
-    lr = synth.LR if optimizer == "sgd" else 1e-3
+    lr = synth.LR if optimizer in ("sgd", "asgd") else 1e-3
     hp = hyper(n, mode, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     hs = [ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
                            weight_decay=hp.weight_decay, layout="spread", rank=r, world=n, optimizer=optimizer,
-                           exchange="p2p") for r in range(n)]
+                           exchange="p2p", **asgd_kw(hp)) for r in range(n)]
     if n > 1:
         ElasticAveraging.p2p_connect(hs)
     streams = [torch.cuda.Stream() for _ in range(n)]
@@ -78,7 +78,7 @@ def test_p2p_exchange_matches_oracle(n, mode):
     _run(n, [200_003, 64, 1_000_000], 10, mode)
 
 
-@pytest.mark.parametrize("n,optimizer", [(2, "adam"), (4, "adamw")])
+@pytest.mark.parametrize("n,optimizer", [(2, "adam"), (4, "adamw"), (3, "asgd")])
 def test_p2p_exchange_adam(n, optimizer):
     _run(n, [300_001, 17], 12, "combined", optimizer)
 

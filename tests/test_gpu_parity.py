@@ -17,7 +17,7 @@ import torch
 
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import EAError, ElasticAveraging, get_unique_id
-from tests._parity import TOL, OracleStage, hyper, rel_err, to_np
+from tests._parity import TOL, OracleStage, asgd_kw, hyper, rel_err, to_np
 
 pytestmark = pytest.mark.gpu
 
@@ -41,7 +41,7 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
         handles[v] = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr,
                                       momentum=hp.momentum, weight_decay=hp.weight_decay, nesterov=hp.nesterov,
                                       kernel_variant=v, optimizer=optimizer, betas=(hp.beta1, hp.beta2), eps=hp.eps,
-                                      staleness=staleness)
+                                      staleness=staleness, **asgd_kw(hp))
     gbuf = [[torch.empty(p, device=dev) for _ in range(n)] for p in sizes]
     order = list(reversed(range(len(sizes))))
     for t in range(steps):
@@ -68,7 +68,7 @@ def _run_colocated(n, sizes, steps, mode, variants=VARIANTS, alpha=None, nestero
             for i in range(n):
                 errs.append(rel_err(to_np(reps[i]), o.xs[i]))
                 errs.append(rel_err(to_np(handles[v].momentum(s, i)), o.ms[i]))
-                if optimizer != "sgd":
+                if optimizer in ("adam", "adamw"):
                     errs.append(rel_err(to_np(handles[v].state(s, i, 1)), o.vs[i]))
             if optimizer != "sgd":
                 assert handles[v].get_step(s) == steps
@@ -147,6 +147,22 @@ def test_adam_register_loop(optimizer, n):
     _run_colocated(n, sizes[:1], 8, "paper", optimizer=optimizer, lr=1e-3, variants=("regloop",))
 
 
+# ------------------------------------------------------------------ ASGD (row f1, reading c29)
+@pytest.mark.parametrize("mode", synth.MODES)
+def test_asgd_c1_100_steps(mode):
+    """C1 + tail stage, 100 steps, ASGD as the local optimizer (averaging from step t0 + 2 = 7 on): the
+    iterate, the average ax and the center, every kernel variant, all stages in one launch."""
+    _run_colocated(2, [1_000_000, 1_000_003], 100, mode, optimizer="asgd", wd=1e-3, many=True,
+                   variants=("auto", "regloop", "laneshfl", "bulkpipe"))
+
+
+@pytest.mark.parametrize("n", [1, 3, 4, 5, 8, 12])
+def test_asgd_replica_counts_and_sizes(n):
+    sizes = [100_003, 7, 4096, 33]
+    _run_colocated(n, sizes, 20, "combined", optimizer="asgd", many=True)
+    _run_colocated(n, sizes[:2], 12, "paper", optimizer="asgd", variants=("auto",))
+
+
 # ------------------------------------------------------------------ stale center (row f4)
 @pytest.mark.parametrize("n", [1, 2, 4, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
@@ -209,16 +225,18 @@ def _placement(rank, stage, n):
     return replica_of(rank, stage, n)
 
 
-@pytest.mark.parametrize("n,optimizer", [(2, "sgd"), (3, "sgd"), (4, "sgd"), (8, "sgd"), (2, "adam"), (4, "adamw")])
+@pytest.mark.parametrize("n,optimizer", [(2, "sgd"), (3, "sgd"), (4, "sgd"), (8, "sgd"), (2, "adam"), (4, "adamw"),
+                                         (3, "asgd")])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 64), steps=20):
     """N ranks on one GPU, external-collective mode: the real local and shard
     kernels, with the reduce-scatter / all-gather done by the test."""
     sizes = list(sizes)
-    hp = hyper(n, mode, lr=synth.LR if optimizer == "sgd" else 1e-3, wd=0.0 if optimizer == "sgd" else 1e-2)
+    hp = hyper(n, mode, lr=synth.LR if optimizer in ("sgd", "asgd") else 1e-3, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     hs = [ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
-                           weight_decay=hp.weight_decay, layout="spread", rank=r, world=n, optimizer=optimizer)
+                           weight_decay=hp.weight_decay, layout="spread", rank=r, world=n, optimizer=optimizer,
+                           **asgd_kw(hp))
           for r in range(n)]
     oracle, gstreams, xs, centers = [], [], [], []
     for s, p in enumerate(sizes):
@@ -262,7 +280,7 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 
             i = _placement(r, s, n)
             assert rel_err(to_np(xs[s][r]), o.xs[i]) <= TOL
             assert rel_err(to_np(hs[r].momentum(s, 0)), o.ms[i]) <= TOL
-            if optimizer != "sgd":
+            if optimizer in ("adam", "adamw"):
                 assert rel_err(to_np(hs[r].state(s, 0, 1)), o.vs[i]) <= TOL
             assert rel_err(to_np(centers[s][r][:p]), o.c) <= TOL
             assert torch.all(centers[s][r][p:] == 0), "center padding must stay zero"
@@ -420,18 +438,18 @@ def test_bad_pointers_rejected_before_enqueue():
 
 
 # ------------------------------------------------------------------ host-buffer path
-@pytest.mark.parametrize("optimizer,n", [("sgd", 2), ("sgd", 4), ("adamw", 3), ("sgd", 12)])
+@pytest.mark.parametrize("optimizer,n", [("sgd", 2), ("sgd", 4), ("adamw", 3), ("sgd", 12), ("asgd", 4)])
 def test_step_many_host_pipelined(optimizer, n):
     """ea_step_many_host: gradients from pinned host memory in 4 Mi-element
     chunks (a 9,000,003-element stage spans 3 ragged chunks), centers copied
     back to host; must equal the oracle and the device-resident center."""
     sizes = [9_000_003, 1_000, 5] if n <= 4 else [4_500_001, 77]
     steps = 3
-    lr = synth.LR if optimizer == "sgd" else 1e-3
+    lr = synth.LR if optimizer in ("sgd", "asgd") else 1e-3
     hp = hyper(n, "combined", lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
-                         weight_decay=hp.weight_decay, optimizer=optimizer)
+                         weight_decay=hp.weight_decay, optimizer=optimizer, **asgd_kw(hp))
     oracle, gstreams, xs, cs, host_out = [], [], [], [], []
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
@@ -466,18 +484,18 @@ def test_step_many_host_pipelined(optimizer, n):
 
 
 # ------------------------------------------------------------------ CUDA graphs
-@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw"])
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
 def test_step_many_captured_in_a_cuda_graph(optimizer):
     """ea_step_many is stream-ordered work only -- including Adam's step
     counter and bias corrections, which live on the device -- so a whole EA
     step can be captured once and replayed.  Replays must equal the oracle run
     step by step, and the step counter must count replays."""
     n, sizes, steps = 3, [100_003, 4096, 7], 6
-    lr = synth.LR if optimizer == "sgd" else 1e-3
+    lr = synth.LR if optimizer in ("sgd", "asgd") else 1e-3
     hp = hyper(n, "combined", lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
     dev = torch.device("cuda:0")
     h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
-                         weight_decay=hp.weight_decay, optimizer=optimizer)
+                         weight_decay=hp.weight_decay, optimizer=optimizer, **asgd_kw(hp))
     oracle, gstreams, xs, cs, gb = [], [], [], [], []
     for s, p in enumerate(sizes):
         reps, c = synth.host_state(n, p, seed=synth.WEIGHT_SEED + s)
@@ -506,7 +524,8 @@ def test_step_many_captured_in_a_cuda_graph(optimizer):
         assert rel_err(to_np(cs[s]), oracle[s].c) <= TOL
         for i in range(n):
             assert rel_err(to_np(xs[s][i]), oracle[s].xs[i]) <= TOL
-            if optimizer != "sgd":
+            assert rel_err(to_np(h.state(s, i, 0)), oracle[s].ms[i]) <= TOL
+            if optimizer in ("adam", "adamw"):
                 assert rel_err(to_np(h.state(s, i, 1)), oracle[s].vs[i]) <= TOL
         if optimizer != "sgd":
             assert h.get_step(s) == steps          # device counter: replays, not the one capture
