@@ -535,6 +535,17 @@ def _oracle_sample(n, p_sample, seed=0):
     return reps, [np.zeros(p_sample, dtype=np.float32) for _ in range(n)], c, gs
 
 
+def cpu_model():
+    """The host CPU's model name (/proc/cpuinfo), reported beside the oracle timings."""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return None
+
+
 def cpu_baseline(cfg, n, seconds=10.0):
     """The float64 oracle, as it stands (single-threaded numpy), on a bounded
     sample: one full stage of the workload, repeated until `seconds` pass."""
@@ -553,7 +564,7 @@ def cpu_baseline(cfg, n, seconds=10.0):
             break
     out = {"value": n * p * steps / el, "unit": UNIT, "cores": 1, "kind": "oracle",
            "sample": f"{steps} oracle steps of one {p}-element stage x N={n} (float64 numpy, 1 thread), "
-                     f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0))}
+                     f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0)), "cpu_model": cpu_model()}
     out["all_cores"] = cpu_baseline_all_cores(xs, ms, c, g, hp, seconds=seconds / 2)
     return out
 
@@ -611,7 +622,8 @@ def run_reference(args, rank, world):
            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
            "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
            "config": {"workload": cfg.name, "n_pipelines": n, "params_per_step_sample": p_sample, "mode": MODE},
-           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
+                            "cpu_model": cpu_model()},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
            "gpu_launches": 0}
     emit(out)
