@@ -384,6 +384,8 @@ def run_ours(args, rank, world, local):
                      "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
         if world == 1 and local is not None:
             out["roofline"] = local     # no NVLink traffic at world 1: the local kernel is the bound
+            local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
+                             "(NCCL copy + shard update) shares HBM on the side stream")
         else:
             out["roofline"] = nvlink
             if local is not None:

@@ -12,9 +12,9 @@ enum Opt : int { kOptSGD = 0, kOptAdam = 1, kOptAdamW = 2, kOptASGD = 3 };
 
 // Adam(W) keep two state vectors (m, v); SGD-momentum and ASGD one (momentum / the average ax), so they
 // move the same bytes and share the kernels' 3-stream geometry.
-constexpr bool two_state(int opt) { return opt == kOptAdam || opt == kOptAdamW; }
+__host__ __device__ constexpr bool two_state(int opt) { return opt == kOptAdam || opt == kOptAdamW; }
 // Optimizers with per-step coefficients (StepCoef): Adam(W)'s bias corrections, ASGD's eta_t and mu_t.
-constexpr bool has_coef(int opt) { return opt != kOptSGD; }
+__host__ __device__ constexpr bool has_coef(int opt) { return opt != kOptSGD; }
 
 // Hyper-parameters in the form the kernels consume (fp32).
 struct Hyper {

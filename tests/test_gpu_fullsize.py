@@ -95,3 +95,84 @@ def test_beyond_int32_elements(n, p):
         pytest.skip(f"needs {need / 1e9:.0f} GB")
     _run_sampled(n, [p], 1, "auto", k=100_000)
     torch.cuda.empty_cache()
+
+
+def _run_spread_sampled(n, sizes, steps, exchange, optimizer="sgd", k=200_000):
+    """Spread layout at full stage sizes, in bench.py's launch configuration (ea_step per stage in the global
+    order K-1..0, ea_sync per step): world 1 over NCCL, or N virtual ranks on this GPU with the fused P2P
+    kernel.  Sampled elements of every rank's replica, optimizer state and center against the oracle."""
+    from paper_conf_ppopp_chen0qz23_b200.binding import get_unique_id
+    from paper_conf_ppopp_chen0qz23_b200.parallel import replica_of, stage_order
+    dev = torch.device("cuda:0")
+    lr = synth.LR if optimizer == "sgd" else 1e-3
+    hp = hyper(n, "combined", lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+    kw = dict(alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+              weight_decay=hp.weight_decay, layout="spread", world=n, optimizer=optimizer, exchange=exchange)
+    if n == 1:
+        hs = [ElasticAveraging(sizes, 1, rank=0, nccl_id=get_unique_id() if exchange == "nccl" else None, **kw)]
+    else:
+        hs = [ElasticAveraging(sizes, n, rank=r, **kw) for r in range(n)]
+        ElasticAveraging.p2p_connect(hs)
+    streams = [torch.cuda.Stream() for _ in range(n)]
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(11)
+    rng = np.random.default_rng(1)
+    state = []
+    for s, p in enumerate(sizes):
+        reps, c, grads = synth.device_state(n, p, dev, seed=100 + s)
+        cap = hs[0].center_capacity(s)
+        centers = []
+        for r in range(n):
+            cc = torch.zeros(cap, device=dev)
+            cc[:p] = c
+            centers.append(cc)
+        del c
+        # rank r hosts replica replica_of(r, s, n): keep the replicas indexed by rank
+        xs = [reps[replica_of(r, s, n)] for r in range(n)]
+        gs = [grads[replica_of(r, s, n)] for r in range(n)]
+        state.append((xs, gs, centers, _sample_idx(p, k, rng).to(dev)))
+    order = stage_order(len(sizes))
+    f64 = lambda t, idx: t[idx].double().cpu().numpy()
+    for t in range(steps):
+        before = []
+        for s, (xs, gs, centers, idx) in enumerate(state):
+            for g in gs:
+                g.normal_(0.0, synth.GRAD_STD, generator=gen)
+            vs = [f64(hs[r].state(s, 0, 1), idx) for r in range(n)] if optimizer != "sgd" else None
+            before.append(([f64(x, idx) for x in xs], [f64(hs[r].momentum(s, 0), idx) for r in range(n)],
+                           f64(centers[0], idx), [f64(g, idx) for g in gs], vs))
+        torch.cuda.synchronize()
+        for s in order:
+            xs, gs, centers, _ = state[s]
+            for r in range(n):
+                hs[r].step(s, [xs[r]], [gs[r]], centers[r], stream=streams[r])
+        for r in range(n):
+            hs[r].sync(streams[r])
+        torch.cuda.synchronize()
+        for s, (xs, gs, centers, idx) in enumerate(state):
+            bx, bm, bc, bg, bv = before[s]
+            if optimizer == "sgd":
+                ox, om, oc = ea_step(bx, bm, bc, bg, hp)
+            else:
+                ox, om, ov, oc = ea_step_adam(bx, bm, bv, bc, bg, hp, t + 1, decoupled=optimizer == "adamw")
+            for r in range(n):
+                assert rel_err(f64(centers[r], idx), oc) <= TOL, (s, t, r)
+                assert rel_err(f64(xs[r], idx), ox[r]) <= TOL, (s, t, r)
+                assert rel_err(f64(hs[r].momentum(s, 0), idx), om[r]) <= TOL, (s, t, r)
+                if optimizer != "sgd":
+                    assert rel_err(f64(hs[r].state(s, 0, 1), idx), ov[r]) <= TOL, (s, t, r)
+    for h in hs:
+        h.close()
+
+
+@pytest.mark.parametrize("optimizer", ["sgd", "adamw"])
+def test_c4_stages_spread_nccl_world1_sampled(optimizer):
+    """Two C4-sized stages (44,375,000 elements each) through the NCCL spread path at world 1."""
+    cfg = synth.CONFIGS["C4"]
+    _run_spread_sampled(1, cfg.stage_sizes[:2], 2, "nccl", optimizer)
+
+
+def test_c4_stage_p2p_8_virtual_ranks_sampled():
+    """One C4-sized stage, 8 virtual ranks, the fused P2P exchange (the bench's N=8 kernel at full size)."""
+    cfg = synth.CONFIGS["C4"]
+    _run_spread_sampled(8, cfg.stage_sizes[:1], 2, "p2p")
