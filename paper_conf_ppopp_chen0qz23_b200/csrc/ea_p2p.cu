@@ -26,6 +26,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <cstdlib>
+
 #include "ea_internal.h"
 
 namespace ea {
@@ -102,8 +104,97 @@ __device__ bool wait_at_least(const uint32_t* flag, uint32_t target, uint64_t ti
   return true;
 }
 
+// Phase A on one chunk [e0, e0 + 4 nv4): each thread hoists the loads of UA float4 of every input stream
+// (x, g, state(s), x~) before any arithmetic (UA = 1: one float4 at a time), then updates, stores x and the
+// state locally and the contribution into the owner's inbox (a peer store).
 template <int OPT>
-__global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const P2PView view) {
+__device__ __forceinline__ float4 ragged4(const P2PArgs& a, int64_t j, const StepCoef& sc) {
+  float rr[4];
+  for (int q = 0; q < 4; ++q) {
+    const int64_t jj = j + q;
+    rr[q] = 0.f;
+    if (jj < a.p) {
+      float xs = a.x[jj], ms = a.m[jj], ws = two_state(OPT) ? a.v[jj] : 0.f;
+      rr[q] = p2p_elem<OPT>(xs, a.g[jj], ms, ws, a.center[jj], a.hp, sc);
+      a.x[jj] = xs;
+      a.m[jj] = ms;
+      if (two_state(OPT)) a.v[jj] = ws;
+    }
+  }
+  return make_float4(rr[0], rr[1], rr[2], rr[3]);
+}
+
+template <int OPT, int UA>
+__device__ __forceinline__ void phase_a_chunk(const P2PArgs& a, int64_t e0, int64_t nv4, float* dst,
+                                              const StepCoef& sc) {
+  if constexpr (UA == 1) {  // one float4 per stream at a time (32 registers for SGD: 8 CTAs/SM)
+    for (int64_t lv = threadIdx.x; lv < nv4; lv += kP2PThreads) {
+      const int64_t j = e0 + 4 * lv;
+      float4 rv;
+      if (j + 3 < a.p) {
+        float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
+        float4 w = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
+        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
+        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
+        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
+        st4(a.x + j, x);
+        st4(a.m + j, m);
+        if (two_state(OPT)) st4(a.v + j, w);
+      } else {  // the ragged end of the replica and the zero padding of the center
+        rv = ragged4<OPT>(a, j, sc);
+      }
+      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
+    }
+    return;
+  }
+  for (int64_t lb = threadIdx.x; lb < nv4; lb += (int64_t)kP2PThreads * UA) {
+    float4 x[UA], g[UA], m[UA], c4[UA], w[UA];
+    bool full[UA];
+#pragma unroll
+    for (int u = 0; u < UA; ++u) {
+      const int64_t lv = lb + (int64_t)u * kP2PThreads;
+      const int64_t j = e0 + 4 * lv;
+      full[u] = lv < nv4 && j + 3 < a.p;
+      if (full[u]) {
+        x[u] = ld4(a.x + j);
+        g[u] = ld4(a.g + j);
+        m[u] = ld4(a.m + j);
+        c4[u] = ld4(a.center + j);
+        w[u] = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < UA; ++u) {
+      const int64_t lv = lb + (int64_t)u * kP2PThreads;
+      if (lv >= nv4) continue;
+      const int64_t j = e0 + 4 * lv;
+      float4 rv;
+      if (full[u]) {
+        rv.x = p2p_elem<OPT>(x[u].x, g[u].x, m[u].x, w[u].x, c4[u].x, a.hp, sc);
+        rv.y = p2p_elem<OPT>(x[u].y, g[u].y, m[u].y, w[u].y, c4[u].y, a.hp, sc);
+        rv.z = p2p_elem<OPT>(x[u].z, g[u].z, m[u].z, w[u].z, c4[u].z, a.hp, sc);
+        rv.w = p2p_elem<OPT>(x[u].w, g[u].w, m[u].w, w[u].w, c4[u].w, a.hp, sc);
+        st4(a.x + j, x[u]);
+        st4(a.m + j, m[u]);
+        if (two_state(OPT)) st4(a.v + j, w[u]);
+      } else {
+        rv = ragged4<OPT>(a, j, sc);
+      }
+      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
+    }
+  }
+}
+
+// Resident CTAs asked of ptxas: UA = 1 keeps the register counts of the plain loop (SGD/ASGD 32: 8 CTAs/SM,
+// Adam(W) 48: 5); the hoisted variants trade CTAs for bytes in flight per thread.
+__host__ __device__ constexpr int p2p_min_blocks(int opt, int ua) {
+  return ua == 1 ? (two_state(opt) ? 5 : 8) : (ua == 2 ? 4 : 2);
+}
+
+template <int OPT, int UA>
+__global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p2p(const P2PArgs a,
+                                                                                  const P2PView view) {
   const int tid = threadIdx.x;
   const int64_t Q = a.chunk, nch = a.nchunks, slots = a.slots;
   const int N = a.world, r = a.rank;
@@ -118,36 +209,7 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
     float* dst = view.inbox[o] + ((int64_t)r * slots + slot) * Q;
-    for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) {
-      const int64_t j = e0 + 4 * lv;
-      float4 rv;
-      if (j + 3 < a.p) {
-        float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
-        float4 w = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
-        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
-        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
-        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
-        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
-        st4(a.x + j, x);
-        st4(a.m + j, m);
-        if (two_state(OPT)) st4(a.v + j, w);
-      } else {  // the ragged end of the replica and the zero padding of the center
-        float rr[4];
-        for (int q = 0; q < 4; ++q) {
-          const int64_t jj = j + q;
-          rr[q] = 0.f;
-          if (jj < a.p) {
-            float x = a.x[jj], m = a.m[jj], w = two_state(OPT) ? a.v[jj] : 0.f;
-            rr[q] = p2p_elem<OPT>(x, a.g[jj], m, w, a.center[jj], a.hp, sc);
-            a.x[jj] = x;
-            a.m[jj] = m;
-            if (two_state(OPT)) a.v[jj] = w;
-          }
-        }
-        rv = make_float4(rr[0], rr[1], rr[2], rr[3]);
-      }
-      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
-    }
+    phase_a_chunk<OPT, UA>(a, e0, len / 4, dst, sc);
     __syncthreads();
     if (tid == 0) {
       __threadfence_system();
@@ -201,6 +263,40 @@ __global__ void __launch_bounds__(kP2PThreads) spread_p2p(const P2PArgs a, const
   }
 }
 
+// Phase-A unroll knob for measurement: AVGPIPE_EA_P2P_UNROLL = 1 | 2 | 4 (default 1).
+int p2p_unroll() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_P2P_UNROLL");
+    const int k = e ? std::atoi(e) : 1;
+    return (k == 2 || k == 4) ? k : 1;
+  }();
+  return v;
+}
+
+template <int UA>
+void launch_ua(const P2PArgs& a, const P2PView& v, int opt, int grid, cudaStream_t s) {
+  if (opt == kOptAdam) spread_p2p<kOptAdam, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
+  else if (opt == kOptAdamW) spread_p2p<kOptAdamW, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
+  else if (opt == kOptASGD) spread_p2p<kOptASGD, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
+  else spread_p2p<kOptSGD, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
+}
+
+template <int OPT, int UA>
+int blocks_per_sm_t() {
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT, UA>, kP2PThreads, 0) != cudaSuccess ||
+      per_sm < 1)
+    per_sm = 1;
+  return per_sm;
+}
+
+template <int UA>
+int blocks_per_sm_ua(int opt) {
+  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD, UA>();
+  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD, UA>();
+  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam, UA>() : blocks_per_sm_t<kOptAdamW, UA>();
+}
+
 }  // namespace
 
 cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s) {
@@ -208,28 +304,18 @@ cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int m
   int64_t grid = max_ctas;
   if (grid > a.nchunks) grid = a.nchunks;
   if (grid < 1) grid = 1;
-  if (opt == kOptAdam) spread_p2p<kOptAdam><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
-  else if (opt == kOptAdamW) spread_p2p<kOptAdamW><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
-  else if (opt == kOptASGD) spread_p2p<kOptASGD><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
-  else spread_p2p<kOptSGD><<<static_cast<int>(grid), kP2PThreads, 0, s>>>(a, v);
+  const int ua = p2p_unroll();
+  if (ua == 4) launch_ua<4>(a, v, opt, static_cast<int>(grid), s);
+  else if (ua == 2) launch_ua<2>(a, v, opt, static_cast<int>(grid), s);
+  else launch_ua<1>(a, v, opt, static_cast<int>(grid), s);
   return cudaGetLastError();
 }
 
-template <int OPT>
-int blocks_per_sm_t() {
-  int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT>, kP2PThreads, 0) != cudaSuccess ||
-      per_sm < 1)
-    per_sm = 1;
-  return per_sm;
-}
-
-// Resident CTAs per SM of the instance that will run (SGD 32 registers: 8; Adam(W) 48: 5).  The grid never
-// exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
+// Resident CTAs per SM of the instance that will run (UA = 1: SGD 32 registers: 8; Adam(W) 48: 5).  The grid
+// never exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
 int p2p_blocks_per_sm(int opt) {
-  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD>();
-  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD>();
-  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam>() : blocks_per_sm_t<kOptAdamW>();
+  const int ua = p2p_unroll();
+  return ua == 4 ? blocks_per_sm_ua<4>(opt) : ua == 2 ? blocks_per_sm_ua<2>(opt) : blocks_per_sm_ua<1>(opt);
 }
 
 }  // namespace ea
