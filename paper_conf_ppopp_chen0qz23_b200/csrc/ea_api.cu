@@ -387,6 +387,16 @@ uint64_t p2p_timeout_ns() {
   return static_cast<uint64_t>(ms > 0 ? ms : 30000) * 1000000ull;
 }
 
+// Measurement knob AVGPIPE_EA_P2P_FENCE=0: no fence.sc.sys before the release operations that publish a
+// chunk (bar.sync orders the CTA's stores before thread 0's release, which is cumulative at system scope).
+int p2p_sc_fence() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_P2P_FENCE");
+    return (e && e[0] == '0') ? 0 : 1;
+  }();
+  return v;
+}
+
 // Lay out and allocate this rank's exchange buffer (per stage: inbox, outbox, counters).
 ea_status p2p_alloc(ea_ctx* h) {
   const int n = h->cfg.n_pipelines;
@@ -507,6 +517,7 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   a.hp = h->hp;
   a.err = h->err_dev;
   a.timeout_ns = p2p_timeout_ns();
+  a.sc_fence = p2p_sc_fence();
   // all ranks' kernels must be resident together: ranks sharing this device share its SMs
   int max_ctas = h->num_sms * ea::p2p_blocks_per_sm(h->cfg.optimizer) / h->same_device_ranks;
   if (max_ctas < 1) max_ctas = 1;

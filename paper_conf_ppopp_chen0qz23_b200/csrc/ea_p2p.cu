@@ -212,7 +212,7 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
     phase_a_chunk<OPT, UA>(a, e0, len / 4, dst, sc);
     __syncthreads();
     if (tid == 0) {
-      __threadfence_system();
+      if (a.sc_fence) __threadfence_system();  // fence.sc; the release below is cumulative on its own
       red_add_release_sys(view.arrive[o] + slot, 1u);
     }
   }
@@ -242,7 +242,7 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
     }
     __syncthreads();
     if (tid == 0) {
-      __threadfence_system();
+      if (a.sc_fence) __threadfence_system();
       st_release_sys(view.ready[r] + slot, epoch);
     }
     (void)s_ok;
