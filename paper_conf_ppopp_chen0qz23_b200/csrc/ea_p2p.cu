@@ -104,9 +104,7 @@ __device__ bool wait_at_least(const uint32_t* flag, uint32_t target, uint64_t ti
   return true;
 }
 
-// Phase A on one chunk [e0, e0 + 4 nv4): each thread hoists the loads of UA float4 of every input stream
-// (x, g, state(s), x~) before any arithmetic (UA = 1: one float4 at a time), then updates, stores x and the
-// state locally and the contribution into the owner's inbox (a peer store).
+// Scalar path for the ragged end of the replica and the zero padding of the center (4 elements from j).
 template <int OPT>
 __device__ __forceinline__ float4 ragged4(const P2PArgs& a, int64_t j, const StepCoef& sc) {
   float rr[4];
@@ -124,77 +122,77 @@ __device__ __forceinline__ float4 ragged4(const P2PArgs& a, int64_t j, const Ste
   return make_float4(rr[0], rr[1], rr[2], rr[3]);
 }
 
-template <int OPT, int UA>
+// Phase A on one chunk [e0, e0 + 4 nv4) by the kP2PThreads compute threads: update, store x and the state
+// locally and the contribution into the owner's inbox (a peer store).  (Hoisting 2 or 4 float4 per stream per
+// thread measured 6-25% slower: fewer resident CTAs, profiles/r01_s3_p2p_unroll_occupancy.jsonl.)
+template <int OPT>
 __device__ __forceinline__ void phase_a_chunk(const P2PArgs& a, int64_t e0, int64_t nv4, float* dst,
                                               const StepCoef& sc) {
-  if constexpr (UA == 1) {  // one float4 per stream at a time (32 registers for SGD: 8 CTAs/SM)
-    for (int64_t lv = threadIdx.x; lv < nv4; lv += kP2PThreads) {
-      const int64_t j = e0 + 4 * lv;
-      float4 rv;
-      if (j + 3 < a.p) {
-        float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
-        float4 w = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
-        rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
-        rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
-        rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
-        rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
-        st4(a.x + j, x);
-        st4(a.m + j, m);
-        if (two_state(OPT)) st4(a.v + j, w);
-      } else {  // the ragged end of the replica and the zero padding of the center
-        rv = ragged4<OPT>(a, j, sc);
-      }
-      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
+  for (int64_t lv = threadIdx.x; lv < nv4; lv += kP2PThreads) {
+    const int64_t j = e0 + 4 * lv;
+    float4 rv;
+    if (j + 3 < a.p) {
+      float4 x = ld4(a.x + j), g = ld4(a.g + j), m = ld4(a.m + j), c4 = ld4(a.center + j);
+      float4 w = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+      rv.x = p2p_elem<OPT>(x.x, g.x, m.x, w.x, c4.x, a.hp, sc);
+      rv.y = p2p_elem<OPT>(x.y, g.y, m.y, w.y, c4.y, a.hp, sc);
+      rv.z = p2p_elem<OPT>(x.z, g.z, m.z, w.z, c4.z, a.hp, sc);
+      rv.w = p2p_elem<OPT>(x.w, g.w, m.w, w.w, c4.w, a.hp, sc);
+      st4(a.x + j, x);
+      st4(a.m + j, m);
+      if (two_state(OPT)) st4(a.v + j, w);
+    } else {  // the ragged end of the replica and the zero padding of the center
+      rv = ragged4<OPT>(a, j, sc);
     }
-    return;
-  }
-  for (int64_t lb = threadIdx.x; lb < nv4; lb += (int64_t)kP2PThreads * UA) {
-    float4 x[UA], g[UA], m[UA], c4[UA], w[UA];
-    bool full[UA];
-#pragma unroll
-    for (int u = 0; u < UA; ++u) {
-      const int64_t lv = lb + (int64_t)u * kP2PThreads;
-      const int64_t j = e0 + 4 * lv;
-      full[u] = lv < nv4 && j + 3 < a.p;
-      if (full[u]) {
-        x[u] = ld4(a.x + j);
-        g[u] = ld4(a.g + j);
-        m[u] = ld4(a.m + j);
-        c4[u] = ld4(a.center + j);
-        w[u] = two_state(OPT) ? ld4(a.v + j) : make_float4(0.f, 0.f, 0.f, 0.f);
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < UA; ++u) {
-      const int64_t lv = lb + (int64_t)u * kP2PThreads;
-      if (lv >= nv4) continue;
-      const int64_t j = e0 + 4 * lv;
-      float4 rv;
-      if (full[u]) {
-        rv.x = p2p_elem<OPT>(x[u].x, g[u].x, m[u].x, w[u].x, c4[u].x, a.hp, sc);
-        rv.y = p2p_elem<OPT>(x[u].y, g[u].y, m[u].y, w[u].y, c4[u].y, a.hp, sc);
-        rv.z = p2p_elem<OPT>(x[u].z, g[u].z, m[u].z, w[u].z, c4[u].z, a.hp, sc);
-        rv.w = p2p_elem<OPT>(x[u].w, g[u].w, m[u].w, w[u].w, c4[u].w, a.hp, sc);
-        st4(a.x + j, x[u]);
-        st4(a.m + j, m[u]);
-        if (two_state(OPT)) st4(a.v + j, w[u]);
-      } else {
-        rv = ragged4<OPT>(a, j, sc);
-      }
-      st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
-    }
+    st4(dst + 4 * lv, rv);  // peer store into the owner's inbox
   }
 }
 
-// Resident CTAs asked of ptxas: UA = 1 keeps the register counts of the plain loop (SGD/ASGD 32: 8 CTAs/SM,
-// Adam(W) 48: 5); the hoisted variants trade CTAs for bytes in flight per thread.
-__host__ __device__ constexpr int p2p_min_blocks(int opt, int ua) {
-  return ua == 1 ? (two_state(opt) ? 5 : 8) : (ua == 2 ? 4 : 2);
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(b)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {  // release at CTA scope
+  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_addr(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {  // acquire at CTA scope
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 P1, [%0], %1;\n"
+      "@!P1 bra WAIT_%=;\n"
+      "}\n" ::"r"(smem_addr(b)),
+      "r"(parity)
+      : "memory");
+}
+// Barrier of the compute warps only (named barrier 1): the signal warp never joins phases B and C.
+template <int SW>
+__device__ __forceinline__ void compute_sync() {
+  if constexpr (SW) asm volatile("bar.sync 1, %0;" ::"n"(kP2PThreads) : "memory");
+  else __syncthreads();
 }
 
-template <int OPT, int UA>
-__global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p2p(const P2PArgs a,
-                                                                                  const P2PView view) {
+constexpr int kSigDepth = 4;  // chunks the compute warps may run ahead of the signal warp
+
+// SW = 0: after each chunk the CTA's threads meet at a block barrier and thread 0 publishes the chunk (a
+// system-scope release-add on the owner's arrival counter) -- every compute warp waits for the slowest one and
+// for the release.  SW = 1: a ninth "signal" warp publishes instead: each compute warp arrives (release, CTA
+// scope) on the chunk's smem mbarrier as soon as its own stores are issued and goes on to the next chunk; the
+// signal warp waits for the eight arrivals (acquire, CTA scope) and issues the system-scope release-add, which
+// is cumulative, so the peers that acquire the counter see every compute warp's stores.
+template <int SW>
+constexpr int p2p_threads() { return kP2PThreads + (SW ? 32 : 0); }
+// Resident CTAs asked of ptxas (the plain loop's own register counts: SGD/ASGD 32, Adam(W) 48).
+__host__ __device__ constexpr int p2p_min_blocks(int opt, int sw) {
+  return sw ? (two_state(opt) ? 4 : 5) : (two_state(opt) ? 5 : 8);
+}
+
+template <int OPT, int SW>
+__global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) spread_p2p(const P2PArgs a,
+                                                                                       const P2PView view) {
   const int tid = threadIdx.x;
   const int64_t Q = a.chunk, nch = a.nchunks, slots = a.slots;
   const int N = a.world, r = a.rank;
@@ -202,18 +200,56 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
   const uint32_t epoch = static_cast<uint32_t>(*a.stepp);
   const StepCoef sc = has_coef(OPT) ? *a.scp : StepCoef{0.f, 0.f};
 
-  // ---------------- Phase A: local update, push contributions to the owners
-  for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
-    const int o = static_cast<int>(c % N);
-    const int64_t slot = c / N;
-    const int64_t e0 = c * Q;
-    const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-    float* dst = view.inbox[o] + ((int64_t)r * slots + slot) * Q;
-    phase_a_chunk<OPT, UA>(a, e0, len / 4, dst, sc);
-    __syncthreads();
+  if constexpr (SW) {
+    __shared__ __align__(8) uint64_t full[kSigDepth], empty[kSigDepth];
     if (tid == 0) {
-      if (a.sc_fence) __threadfence_system();  // fence.sc; the release below is cumulative on its own
-      red_add_release_sys(view.arrive[o] + slot, 1u);
+      for (int i = 0; i < kSigDepth; ++i) {
+        mbar_init(&full[i], kP2PThreads / 32);
+        mbar_init(&empty[i], 1);
+      }
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    if (tid >= kP2PThreads) {  // ---- the signal warp: publish chunks in order, then leave
+      int k = 0;
+      for (int64_t c = blockIdx.x; c < nch; c += gridDim.x, ++k) {
+        const int sl = k % kSigDepth;
+        mbar_wait(&full[sl], (k / kSigDepth) & 1);
+        if (tid == kP2PThreads) {
+          if (a.sc_fence) __threadfence_system();
+          red_add_release_sys(view.arrive[static_cast<int>(c % N)] + c / N, 1u);
+          mbar_arrive(&empty[sl]);
+        }
+        __syncwarp();
+      }
+      return;
+    }
+    // ---- compute warps, phase A
+    int k = 0;
+    for (int64_t c = blockIdx.x; c < nch; c += gridDim.x, ++k) {
+      const int sl = k % kSigDepth;
+      if (k >= kSigDepth) mbar_wait(&empty[sl], ((k / kSigDepth) - 1) & 1);   // the signal warp took chunk k-D
+      const int o = static_cast<int>(c % N);
+      const int64_t slot = c / N;
+      const int64_t e0 = c * Q;
+      const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
+      phase_a_chunk<OPT>(a, e0, len / 4, view.inbox[o] + ((int64_t)r * slots + slot) * Q, sc);
+      __syncwarp();
+      if ((tid & 31) == 0) mbar_arrive(&full[sl]);
+    }
+  } else {
+    // ---------------- Phase A: local update, push contributions to the owners
+    for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
+      const int o = static_cast<int>(c % N);
+      const int64_t slot = c / N;
+      const int64_t e0 = c * Q;
+      const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
+      phase_a_chunk<OPT>(a, e0, len / 4, view.inbox[o] + ((int64_t)r * slots + slot) * Q, sc);
+      __syncthreads();
+      if (tid == 0) {
+        if (a.sc_fence) __threadfence_system();  // fence.sc; the release below is cumulative on its own
+        red_add_release_sys(view.arrive[o] + slot, 1u);
+      }
     }
   }
 
@@ -225,7 +261,7 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
     if (tid == 0) s_ok = wait_at_least(view.arrive[r] + slot, (uint32_t)N * epoch, a.timeout_ns, a.err);
-    __syncthreads();
+    compute_sync<SW>();
     const float* in = view.inbox[r] + slot * Q;
     float* out = view.outbox[r] + slot * Q;
     for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) {
@@ -240,7 +276,7 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
       st4(a.center + e0 + 4 * lv, cv);
       st4(out + 4 * lv, cv);
     }
-    __syncthreads();
+    compute_sync<SW>();
     if (tid == 0) {
       if (a.sc_fence) __threadfence_system();
       st_release_sys(view.ready[r] + slot, epoch);
@@ -256,45 +292,46 @@ __global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT, UA)) spread_p
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
     if (tid == 0) s_ok = wait_at_least(view.ready[o] + slot, epoch, a.timeout_ns, a.err);
-    __syncthreads();
+    compute_sync<SW>();
     const float* src = view.outbox[o] + slot * Q;
     for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) st4(a.center + e0 + 4 * lv, ld_cg(src + 4 * lv));
-    __syncthreads();
+    compute_sync<SW>();
   }
 }
 
-// Phase-A unroll knob for measurement: AVGPIPE_EA_P2P_UNROLL = 1 | 2 | 4 (default 1).
-int p2p_unroll() {
+// Signal-warp knob (measurement): AVGPIPE_EA_P2P_SIGWARP = 1 selects SW = 1.
+int p2p_sigwarp() {
   static const int v = [] {
-    const char* e = std::getenv("AVGPIPE_EA_P2P_UNROLL");
-    const int k = e ? std::atoi(e) : 1;
-    return (k == 2 || k == 4) ? k : 1;
+    const char* e = std::getenv("AVGPIPE_EA_P2P_SIGWARP");
+    return (e && e[0] == '1') ? 1 : 0;
   }();
   return v;
 }
 
-template <int UA>
-void launch_ua(const P2PArgs& a, const P2PView& v, int opt, int grid, cudaStream_t s) {
-  if (opt == kOptAdam) spread_p2p<kOptAdam, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
-  else if (opt == kOptAdamW) spread_p2p<kOptAdamW, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
-  else if (opt == kOptASGD) spread_p2p<kOptASGD, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
-  else spread_p2p<kOptSGD, UA><<<grid, kP2PThreads, 0, s>>>(a, v);
+template <int SW>
+void launch_sw(const P2PArgs& a, const P2PView& v, int opt, int grid, cudaStream_t s) {
+  constexpr int T = p2p_threads<SW>();
+  if (opt == kOptAdam) spread_p2p<kOptAdam, SW><<<grid, T, 0, s>>>(a, v);
+  else if (opt == kOptAdamW) spread_p2p<kOptAdamW, SW><<<grid, T, 0, s>>>(a, v);
+  else if (opt == kOptASGD) spread_p2p<kOptASGD, SW><<<grid, T, 0, s>>>(a, v);
+  else spread_p2p<kOptSGD, SW><<<grid, T, 0, s>>>(a, v);
 }
 
-template <int OPT, int UA>
+template <int OPT, int SW>
 int blocks_per_sm_t() {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT, UA>, kP2PThreads, 0) != cudaSuccess ||
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT, SW>, p2p_threads<SW>(), 0) !=
+          cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   return per_sm;
 }
 
-template <int UA>
-int blocks_per_sm_ua(int opt) {
-  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD, UA>();
-  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD, UA>();
-  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam, UA>() : blocks_per_sm_t<kOptAdamW, UA>();
+template <int SW>
+int blocks_per_sm_sw(int opt) {
+  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD, SW>();
+  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD, SW>();
+  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam, SW>() : blocks_per_sm_t<kOptAdamW, SW>();
 }
 
 }  // namespace
@@ -304,18 +341,13 @@ cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int m
   int64_t grid = max_ctas;
   if (grid > a.nchunks) grid = a.nchunks;
   if (grid < 1) grid = 1;
-  const int ua = p2p_unroll();
-  if (ua == 4) launch_ua<4>(a, v, opt, static_cast<int>(grid), s);
-  else if (ua == 2) launch_ua<2>(a, v, opt, static_cast<int>(grid), s);
-  else launch_ua<1>(a, v, opt, static_cast<int>(grid), s);
+  if (p2p_sigwarp()) launch_sw<1>(a, v, opt, static_cast<int>(grid), s);
+  else launch_sw<0>(a, v, opt, static_cast<int>(grid), s);
   return cudaGetLastError();
 }
 
-// Resident CTAs per SM of the instance that will run (UA = 1: SGD 32 registers: 8; Adam(W) 48: 5).  The grid
-// never exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
-int p2p_blocks_per_sm(int opt) {
-  const int ua = p2p_unroll();
-  return ua == 4 ? blocks_per_sm_ua<4>(opt) : ua == 2 ? blocks_per_sm_ua<2>(opt) : blocks_per_sm_ua<1>(opt);
-}
+// Resident CTAs per SM of the instance that will run (SW = 0: SGD/ASGD 32 registers -> 8, Adam(W) 48 -> 5).
+// The grid never exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
+int p2p_blocks_per_sm(int opt) { return p2p_sigwarp() ? blocks_per_sm_sw<1>(opt) : blocks_per_sm_sw<0>(opt); }
 
 }  // namespace ea
