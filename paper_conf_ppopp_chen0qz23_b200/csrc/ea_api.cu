@@ -387,12 +387,13 @@ uint64_t p2p_timeout_ns() {
   return static_cast<uint64_t>(ms > 0 ? ms : 30000) * 1000000ull;
 }
 
-// Measurement knob AVGPIPE_EA_P2P_FENCE=0: no fence.sc.sys before the release operations that publish a
-// chunk (bar.sync orders the CTA's stores before thread 0's release, which is cumulative at system scope).
+// Measurement knob AVGPIPE_EA_P2P_FENCE=1: a fence.sc.sys before the release operations that publish a chunk.
+// Default off: bar.sync orders the CTA's stores before thread 0's release, which is cumulative at system
+// scope (PTX memory model); the fence measured 1.5-2.5% slower (profiles/r01_s3_p2p_fence.jsonl).
 int p2p_sc_fence() {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_P2P_FENCE");
-    return (e && e[0] == '0') ? 0 : 1;
+    return (e && e[0] == '1') ? 1 : 0;
   }();
   return v;
 }

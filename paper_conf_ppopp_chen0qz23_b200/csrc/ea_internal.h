@@ -141,7 +141,7 @@ struct P2PArgs {
   const StepCoef* scp;   // device: Adam coefficients
   uint32_t* err;       // host-mapped error flag (timeouts)
   uint64_t timeout_ns;
-  int sc_fence;        // 1: fence.sc.sys before each release (knob AVGPIPE_EA_P2P_FENCE=0 drops it)
+  int sc_fence;        // 1: fence.sc.sys before each release (knob AVGPIPE_EA_P2P_FENCE=1; default 0)
 };
 
 cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);

@@ -148,51 +148,13 @@ __device__ __forceinline__ void phase_a_chunk(const P2PArgs& a, int64_t e0, int6
   }
 }
 
-__device__ __forceinline__ uint32_t smem_addr(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_addr(b)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* b) {  // release at CTA scope
-  asm volatile("mbarrier.arrive.release.cta.shared::cta.b64 _, [%0];" ::"r"(smem_addr(b)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {  // acquire at CTA scope
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.acquire.cta.shared::cta.b64 P1, [%0], %1;\n"
-      "@!P1 bra WAIT_%=;\n"
-      "}\n" ::"r"(smem_addr(b)),
-      "r"(parity)
-      : "memory");
-}
-// Barrier of the compute warps only (named barrier 1): the signal warp never joins phases B and C.
-template <int SW>
-__device__ __forceinline__ void compute_sync() {
-  if constexpr (SW) asm volatile("bar.sync 1, %0;" ::"n"(kP2PThreads) : "memory");
-  else __syncthreads();
-}
+// Resident CTAs asked of ptxas (the plain loop's own register counts: SGD/ASGD 32 -> 8 CTAs/SM, Adam(W) 48 -> 5).
+// (A dedicated signal warp that publishes chunks while the compute warps move on measured slower on one rank,
+// 0.82-0.86 vs 0.86-0.90 of HBM peak: profiles/r01_s3_p2p_sigwarp.jsonl.)
+__host__ __device__ constexpr int p2p_min_blocks(int opt) { return two_state(opt) ? 5 : 8; }
 
-constexpr int kSigDepth = 4;  // chunks the compute warps may run ahead of the signal warp
-
-// SW = 0: after each chunk the CTA's threads meet at a block barrier and thread 0 publishes the chunk (a
-// system-scope release-add on the owner's arrival counter) -- every compute warp waits for the slowest one and
-// for the release.  SW = 1: a ninth "signal" warp publishes instead: each compute warp arrives (release, CTA
-// scope) on the chunk's smem mbarrier as soon as its own stores are issued and goes on to the next chunk; the
-// signal warp waits for the eight arrivals (acquire, CTA scope) and issues the system-scope release-add, which
-// is cumulative, so the peers that acquire the counter see every compute warp's stores.
-template <int SW>
-constexpr int p2p_threads() { return kP2PThreads + (SW ? 32 : 0); }
-// Resident CTAs asked of ptxas (the plain loop's own register counts: SGD/ASGD 32, Adam(W) 48).
-__host__ __device__ constexpr int p2p_min_blocks(int opt, int sw) {
-  return sw ? (two_state(opt) ? 4 : 5) : (two_state(opt) ? 5 : 8);
-}
-
-template <int OPT, int SW>
-__global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) spread_p2p(const P2PArgs a,
-                                                                                       const P2PView view) {
+template <int OPT>
+__global__ void __launch_bounds__(kP2PThreads, p2p_min_blocks(OPT)) spread_p2p(const P2PArgs a, const P2PView view) {
   const int tid = threadIdx.x;
   const int64_t Q = a.chunk, nch = a.nchunks, slots = a.slots;
   const int N = a.world, r = a.rank;
@@ -200,56 +162,20 @@ __global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) sp
   const uint32_t epoch = static_cast<uint32_t>(*a.stepp);
   const StepCoef sc = has_coef(OPT) ? *a.scp : StepCoef{0.f, 0.f};
 
-  if constexpr (SW) {
-    __shared__ __align__(8) uint64_t full[kSigDepth], empty[kSigDepth];
-    if (tid == 0) {
-      for (int i = 0; i < kSigDepth; ++i) {
-        mbar_init(&full[i], kP2PThreads / 32);
-        mbar_init(&empty[i], 1);
-      }
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
+  // ---------------- Phase A: local update, push contributions to the owners
+  for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
+    const int o = static_cast<int>(c % N);
+    const int64_t slot = c / N;
+    const int64_t e0 = c * Q;
+    const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
+    phase_a_chunk<OPT>(a, e0, len / 4, view.inbox[o] + ((int64_t)r * slots + slot) * Q, sc);
+    // the block barrier orders every thread's stores before thread 0's system-scope release, which is
+    // cumulative: a peer that acquires the counter sees them all (an extra fence.sc.sys measured 1.5-2.5%
+    // slower and is only a knob now, AVGPIPE_EA_P2P_FENCE=1)
     __syncthreads();
-    if (tid >= kP2PThreads) {  // ---- the signal warp: publish chunks in order, then leave
-      int k = 0;
-      for (int64_t c = blockIdx.x; c < nch; c += gridDim.x, ++k) {
-        const int sl = k % kSigDepth;
-        mbar_wait(&full[sl], (k / kSigDepth) & 1);
-        if (tid == kP2PThreads) {
-          if (a.sc_fence) __threadfence_system();
-          red_add_release_sys(view.arrive[static_cast<int>(c % N)] + c / N, 1u);
-          mbar_arrive(&empty[sl]);
-        }
-        __syncwarp();
-      }
-      return;
-    }
-    // ---- compute warps, phase A
-    int k = 0;
-    for (int64_t c = blockIdx.x; c < nch; c += gridDim.x, ++k) {
-      const int sl = k % kSigDepth;
-      if (k >= kSigDepth) mbar_wait(&empty[sl], ((k / kSigDepth) - 1) & 1);   // the signal warp took chunk k-D
-      const int o = static_cast<int>(c % N);
-      const int64_t slot = c / N;
-      const int64_t e0 = c * Q;
-      const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-      phase_a_chunk<OPT>(a, e0, len / 4, view.inbox[o] + ((int64_t)r * slots + slot) * Q, sc);
-      __syncwarp();
-      if ((tid & 31) == 0) mbar_arrive(&full[sl]);
-    }
-  } else {
-    // ---------------- Phase A: local update, push contributions to the owners
-    for (int64_t c = blockIdx.x; c < nch; c += gridDim.x) {
-      const int o = static_cast<int>(c % N);
-      const int64_t slot = c / N;
-      const int64_t e0 = c * Q;
-      const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
-      phase_a_chunk<OPT>(a, e0, len / 4, view.inbox[o] + ((int64_t)r * slots + slot) * Q, sc);
-      __syncthreads();
-      if (tid == 0) {
-        if (a.sc_fence) __threadfence_system();  // fence.sc; the release below is cumulative on its own
-        red_add_release_sys(view.arrive[o] + slot, 1u);
-      }
+    if (tid == 0) {
+      if (a.sc_fence) __threadfence_system();
+      red_add_release_sys(view.arrive[o] + slot, 1u);
     }
   }
 
@@ -261,7 +187,7 @@ __global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) sp
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
     if (tid == 0) s_ok = wait_at_least(view.arrive[r] + slot, (uint32_t)N * epoch, a.timeout_ns, a.err);
-    compute_sync<SW>();
+    __syncthreads();
     const float* in = view.inbox[r] + slot * Q;
     float* out = view.outbox[r] + slot * Q;
     for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) {
@@ -276,7 +202,7 @@ __global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) sp
       st4(a.center + e0 + 4 * lv, cv);
       st4(out + 4 * lv, cv);
     }
-    compute_sync<SW>();
+    __syncthreads();
     if (tid == 0) {
       if (a.sc_fence) __threadfence_system();
       st_release_sys(view.ready[r] + slot, epoch);
@@ -292,46 +218,20 @@ __global__ void __launch_bounds__(p2p_threads<SW>(), p2p_min_blocks(OPT, SW)) sp
     const int64_t e0 = c * Q;
     const int64_t len = (a.p_pad - e0) < Q ? (a.p_pad - e0) : Q;
     if (tid == 0) s_ok = wait_at_least(view.ready[o] + slot, epoch, a.timeout_ns, a.err);
-    compute_sync<SW>();
+    __syncthreads();
     const float* src = view.outbox[o] + slot * Q;
     for (int64_t lv = tid; lv < len / 4; lv += kP2PThreads) st4(a.center + e0 + 4 * lv, ld_cg(src + 4 * lv));
-    compute_sync<SW>();
+    __syncthreads();
   }
 }
 
-// Signal-warp knob (measurement): AVGPIPE_EA_P2P_SIGWARP = 1 selects SW = 1.
-int p2p_sigwarp() {
-  static const int v = [] {
-    const char* e = std::getenv("AVGPIPE_EA_P2P_SIGWARP");
-    return (e && e[0] == '1') ? 1 : 0;
-  }();
-  return v;
-}
-
-template <int SW>
-void launch_sw(const P2PArgs& a, const P2PView& v, int opt, int grid, cudaStream_t s) {
-  constexpr int T = p2p_threads<SW>();
-  if (opt == kOptAdam) spread_p2p<kOptAdam, SW><<<grid, T, 0, s>>>(a, v);
-  else if (opt == kOptAdamW) spread_p2p<kOptAdamW, SW><<<grid, T, 0, s>>>(a, v);
-  else if (opt == kOptASGD) spread_p2p<kOptASGD, SW><<<grid, T, 0, s>>>(a, v);
-  else spread_p2p<kOptSGD, SW><<<grid, T, 0, s>>>(a, v);
-}
-
-template <int OPT, int SW>
+template <int OPT>
 int blocks_per_sm_t() {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT, SW>, p2p_threads<SW>(), 0) !=
-          cudaSuccess ||
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, spread_p2p<OPT>, kP2PThreads, 0) != cudaSuccess ||
       per_sm < 1)
     per_sm = 1;
   return per_sm;
-}
-
-template <int SW>
-int blocks_per_sm_sw(int opt) {
-  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD, SW>();
-  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD, SW>();
-  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam, SW>() : blocks_per_sm_t<kOptAdamW, SW>();
 }
 
 }  // namespace
@@ -341,13 +241,20 @@ cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int m
   int64_t grid = max_ctas;
   if (grid > a.nchunks) grid = a.nchunks;
   if (grid < 1) grid = 1;
-  if (p2p_sigwarp()) launch_sw<1>(a, v, opt, static_cast<int>(grid), s);
-  else launch_sw<0>(a, v, opt, static_cast<int>(grid), s);
+  const int g = static_cast<int>(grid);
+  if (opt == kOptAdam) spread_p2p<kOptAdam><<<g, kP2PThreads, 0, s>>>(a, v);
+  else if (opt == kOptAdamW) spread_p2p<kOptAdamW><<<g, kP2PThreads, 0, s>>>(a, v);
+  else if (opt == kOptASGD) spread_p2p<kOptASGD><<<g, kP2PThreads, 0, s>>>(a, v);
+  else spread_p2p<kOptSGD><<<g, kP2PThreads, 0, s>>>(a, v);
   return cudaGetLastError();
 }
 
-// Resident CTAs per SM of the instance that will run (SW = 0: SGD/ASGD 32 registers -> 8, Adam(W) 48 -> 5).
-// The grid never exceeds what is resident: the phase-B/C waits rely on every CTA of every rank being on an SM.
-int p2p_blocks_per_sm(int opt) { return p2p_sigwarp() ? blocks_per_sm_sw<1>(opt) : blocks_per_sm_sw<0>(opt); }
+// Resident CTAs per SM of the instance that will run.  The grid never exceeds what is resident: the phase-B/C
+// waits rely on every CTA of every rank being on an SM.
+int p2p_blocks_per_sm(int opt) {
+  if (opt == kOptSGD) return blocks_per_sm_t<kOptSGD>();
+  if (opt == kOptASGD) return blocks_per_sm_t<kOptASGD>();
+  return opt == kOptAdam ? blocks_per_sm_t<kOptAdam>() : blocks_per_sm_t<kOptAdamW>();
+}
 
 }  // namespace ea
