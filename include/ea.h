@@ -260,8 +260,8 @@ EA_API ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard
 
 /* *state_dev = device pointer to optimizer-state slot `slot` of (stage,
  * replica): P_s floats, owned by the library, valid until ea_destroy.
- * slot 0 = SGD momentum / Adam first moment, slot 1 = Adam second moment
- * (EA_EINVAL for SGD).  EA_SPREAD: replica must be 0. */
+ * slot 0 = SGD momentum / Adam first moment / ASGD average, slot 1 = Adam second moment
+ * (EA_EINVAL for SGD and ASGD).  EA_SPREAD: replica must be 0. */
 EA_API ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, float** state_dev);
 
 /* Copy P_s floats from device pointer src into state slot `slot` of (stage,
