@@ -382,10 +382,22 @@ def run_ours(args, rank, world, local):
                                                                      "<" + args.optimizer + ">"),
                      "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
                      "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
+        if args.exchange == "p2p":
+            # the fused kernel's own HBM bytes per rank and element: phase A 28 (SGD/ASGD; Adam 36,
+            # r included), phase B 4 + 12/N, phase C 8 (N-1)/N -- 40 + 4/N for SGD
+            a_bytes = 28 if args.optimizer not in ("adam", "adamw") else 36
+            hbm_bytes = sum((a_bytes + 4 + 12 / n + 8 * (n - 1) / n) * h.center_capacity(s) for s in range(len(sizes)))
+            hbm_gbs = hbm_bytes / (ms * 1e-3) / 1e9
+            local = {"bound": "hbm", "achieved": hbm_gbs, "peak": peak, "unit": "GB/s", "frac": hbm_gbs / peak,
+                     "traffic": None, "kernel": "spread_p2p" + ("" if args.optimizer == "sgd" else
+                                                                "<" + args.optimizer + ">"),
+                     "bytes_per_step": hbm_bytes, "peak_source": peak_src,
+                     "note": "whole step (one fused kernel per stage): the kernel's HBM bytes / step time"}
         if world == 1 and local is not None:
             out["roofline"] = local     # no NVLink traffic at world 1: the local kernel is the bound
-            local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
-                             "(NCCL copy + shard update) shares HBM on the side stream")
+            if args.exchange == "nccl":
+                local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
+                                 "(NCCL copy + shard update) shares HBM on the side stream")
         else:
             out["roofline"] = nvlink
             if local is not None:
