@@ -114,10 +114,12 @@ class PipelineStage:
                         y.backward(gy)
                     if self.prev is not None:
                         pending.append(self._send(x.grad, self.prev, self._tag(i, j, True)))
+        if self.ea is not None:
+            # this stage's last backward is done: the averaging step goes onto the stream now, so it overlaps
+            # the activation-gradient sends still in flight (they never read the parameters; "not block")
+            self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center)
         for w in pending:
             w.wait()
-        if self.ea is not None:
-            self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center)
         if torch.cuda.is_available() and str(device).startswith("cuda"):
             torch.cuda.synchronize()
         dt = time.perf_counter() - t0
