@@ -275,10 +275,12 @@ EA_API ea_status ea_get_step(ea_handle h, int32_t stage, int64_t* step);
 EA_API ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step);
 
 /* Replace the hyper-parameters (alpha, beta, rho, lr, momentum, weight_decay,
- * nesterov, beta1, beta2, eps) from cfg, e.g. for a learning-rate schedule;
- * same validation as ea_init; optimizer, n_pipelines and layout must equal
- * the handle's (other fields are ignored).  Takes effect for steps enqueued
- * afterwards. */
+ * nesterov, beta1, beta2, eps, asgd_lambd, asgd_alpha, asgd_t0) from cfg,
+ * e.g. for a learning-rate schedule; same validation as ea_init; optimizer,
+ * n_pipelines and layout must equal the handle's (other fields are ignored).
+ * Takes effect for steps enqueued afterwards (ASGD: eta_t of the next step is
+ * computed from the new lr; torch.optim.ASGD would use the eta it computed
+ * at the end of the previous step with the old lr). */
 EA_API ea_status ea_set_hyper(ea_handle h, const ea_config* cfg);
 
 /* Wait for outstanding work, free everything the library owns, destroy the
