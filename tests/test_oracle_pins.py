@@ -531,3 +531,70 @@ def test_p3_asgd_center_stays_the_average():
     for t, g in enumerate(_grads(rng, n, p, 20)):
         xs, axs, c = ea_step_asgd(xs, axs, c, g, hp, t + 1)
         np.testing.assert_allclose(c, np.mean(xs, axis=0), rtol=0, atol=1e-15)
+
+
+# ---------------------------------------------------------------- stale center with ASGD (rows f1 x f4)
+def test_asgd_stale_with_equal_centers_is_the_synchronous_asgd_step():
+    from oracle.ea_oracle import ea_step_asgd, ea_step_asgd_stale
+    rng = np.random.default_rng(36)
+    n, p = 3, 100
+    xs, _, c = _rand_state(rng, n, p)
+    axs = [x + rng.normal(0, 1e-4, p) for x in xs]
+    g = [rng.normal(0, 1e-2, p) for _ in range(n)]
+    hp = Hyper(alpha=0.3, beta=0.9, rho=1.0, lr=0.2, weight_decay=1e-3, asgd_lambd=1e-2, asgd_t0=1.0)
+    a = ea_step_asgd(xs, axs, c, g, hp, 5)
+    b = ea_step_asgd_stale(xs, axs, c, c, g, hp, 5)
+    for i in range(n):
+        np.testing.assert_array_equal(a[0][i], b[0][i])
+        np.testing.assert_array_equal(a[1][i], b[1][i])
+    np.testing.assert_array_equal(a[2], b[2])
+    np.testing.assert_array_equal(b[3], c)
+
+
+def test_asgd_stale_alpha0_is_independent_torch_asgd():
+    """alpha = 0: the (stale) center never feeds back, so each replica is torch.optim.ASGD (float64)."""
+    from oracle.ea_oracle import ea_step_asgd_stale
+    rng = np.random.default_rng(37)
+    n, p, steps, lr = 2, 120, 10, 0.3
+    xs, _, c = _rand_state(rng, n, p)
+    gs = _grads(rng, n, p, steps)
+    hp = Hyper(alpha=0.0, beta=1.0, rho=1.0, lr=lr, weight_decay=1e-3, asgd_lambd=5e-2, asgd_t0=2.0)
+    ox, oa, oc, op = [x.copy() for x in xs], [np.zeros(p) for _ in range(n)], c.copy(), c.copy()
+    for t in range(steps):
+        ox, oa, oc, op = ea_step_asgd_stale(ox, oa, oc, op, gs[t], hp, t + 1)
+    prev = torch.get_default_dtype()
+    torch.set_default_dtype(torch.float64)
+    try:
+        for i in range(n):
+            w = torch.nn.Parameter(torch.tensor(xs[i], dtype=torch.float64))
+            opt = torch.optim.ASGD([w], lr=lr, lambd=5e-2, alpha=0.75, t0=2.0, weight_decay=1e-3)
+            for t in range(steps):
+                w.grad = torch.tensor(gs[t][i], dtype=torch.float64)
+                opt.step()
+            np.testing.assert_allclose(ox[i], w.detach().numpy(), rtol=1e-13, atol=1e-16)
+            np.testing.assert_allclose(oa[i], opt.state[w]["ax"].numpy(), rtol=1e-13, atol=1e-16)
+    finally:
+        torch.set_default_dtype(prev)
+
+
+@pytest.mark.parametrize("n,alpha,rho", [(2, 0.5, 1.0), (4, 0.25, 0.0), (3, 0.1, 1.0)])
+def test_asgd_stale_zero_gradient_state_space_closed_form(n, alpha, rho):
+    """Zero gradients and no decay term (lambd = 0) give Delta = 0, so the stale state-space closed form
+    (mean x, x~_t, x~_{t-1}) = A^t s_0 with A = [[1-a, 0, a], [b, 1, -b], [0, 1, 0]] holds with ASGD too."""
+    from oracle.ea_oracle import ea_step_asgd_stale
+    rng = np.random.default_rng(38)
+    p, steps = 50, 10
+    beta = n * alpha
+    xs, _, c = _rand_state(rng, n, p)
+    c = c + rng.normal(0, 1e-3, p)
+    hp = Hyper(alpha=alpha, beta=beta, rho=rho, lr=0.1, asgd_lambd=0.0, asgd_t0=0.0)
+    A = np.array([[1 - alpha, 0.0, alpha], [beta, 1.0, -beta], [0.0, 1.0, 0.0]])
+    s0 = np.stack([np.mean(xs, axis=0), c, c])
+    z = [np.zeros(p)] * n
+    cur_x, cur_a, cur_c, prev_c = xs, z, c, c
+    for t in range(1, steps + 1):
+        cur_x, cur_a, cur_c, prev_c = ea_step_asgd_stale(cur_x, cur_a, cur_c, prev_c, z, hp, t)
+        st = np.linalg.matrix_power(A, t) @ s0
+        np.testing.assert_allclose(np.mean(cur_x, axis=0), st[0], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(cur_c, st[1], rtol=1e-12, atol=1e-15)
+        np.testing.assert_allclose(prev_c, st[2], rtol=1e-12, atol=1e-15)
