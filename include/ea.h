@@ -130,7 +130,7 @@ typedef struct {
                                    late, x~_{t-1}, as with the paper's asynchronous queues (
                                    reading c28, row f4).  1 needs EA_COLOCATED (any optimizer); the
                                    library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step).
-                                   SGD, Adam and AdamW only. */
+                                   Any optimizer. */
   double asgd_lambd;            /* ASGD: decay term l >= 0 (torch default 1e-4) */
   double asgd_alpha;            /* ASGD: power a of the eta schedule (torch default 0.75) */
   double asgd_t0;               /* ASGD: step after which averaging starts, >= 0 (torch default 1e6) */

@@ -593,10 +593,6 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     set_err(nullptr, "staleness 1 is supported for EA_COLOCATED");
     return EA_EINVAL;
   }
-  if (c.staleness == 1 && c.optimizer == EA_OPT_ASGD) {
-    set_err(nullptr, "staleness 1 supports SGD, Adam and AdamW");
-    return EA_EINVAL;
-  }
   if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {
     set_err(nullptr, "peer-memory exchange supports world <= %d", ea::kMaxWorld);
     return EA_EINVAL;

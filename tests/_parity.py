@@ -12,7 +12,8 @@ from __future__ import annotations
 
 import numpy as np
 
-from oracle.ea_oracle import Hyper, ea_step, ea_step_adam, ea_step_adam_stale, ea_step_asgd, ea_step_stale
+from oracle.ea_oracle import (Hyper, ea_step, ea_step_adam, ea_step_adam_stale, ea_step_asgd, ea_step_asgd_stale,
+                               ea_step_stale)
 from paper_conf_ppopp_chen0qz23_b200 import synth
 
 TOL = 1e-5
@@ -76,6 +77,9 @@ class OracleStage:
         self.t += 1
         if self.staleness == 1 and self.opt == "sgd":
             self.xs, self.ms, self.c, self.c_prev = ea_step_stale(self.xs, self.ms, self.c, self.c_prev, grads, hp)
+        elif self.staleness == 1 and self.opt == "asgd":
+            self.xs, self.ms, self.c, self.c_prev = ea_step_asgd_stale(self.xs, self.ms, self.c, self.c_prev, grads,
+                                                                       hp, self.t)
         elif self.staleness == 1:
             self.xs, self.ms, self.vs, self.c, self.c_prev = ea_step_adam_stale(
                 self.xs, self.ms, self.vs, self.c, self.c_prev, grads, hp, self.t, decoupled=self.opt == "adamw")

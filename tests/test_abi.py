@@ -106,7 +106,6 @@ def _cfg(**kw):
     (dict(optimizer=3, asgd_lambd=-1.0), "ASGD"),
     (dict(optimizer=3, asgd_t0=float("nan")), "ASGD"),
     (dict(optimizer=3, asgd_alpha=float("inf")), "ASGD"),
-    (dict(optimizer=3, staleness=1), "staleness 1 supports"),
     (dict(exchange=5), "exchange"),
     (dict(staleness=2), "staleness"),
     (dict(staleness=1, layout=1, world=2, rank=0), "staleness 1"),

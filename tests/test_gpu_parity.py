@@ -181,6 +181,14 @@ def test_stale_center_adam(optimizer, n):
     _run_colocated(n, [65_537], 15, "paper", variants=("auto",), staleness=1, optimizer=optimizer, lr=1e-3)
 
 
+@pytest.mark.parametrize("n", [1, 2, 8, 12])
+def test_stale_center_asgd(n):
+    """staleness 1 with ASGD as the local optimizer (readings c28 + c29; averaging from step 7 on)."""
+    _run_colocated(n, [100_003, 7, 4096], 30, "combined", variants=("auto",), staleness=1, many=True,
+                   optimizer="asgd", wd=1e-3)
+    _run_colocated(n, [65_537], 15, "paper", variants=("auto",), staleness=1, optimizer="asgd")
+
+
 def test_stale_center_c1_100_steps():
     _run_colocated(2, [1_000_000, 1_000_003], 100, "combined", variants=("auto",), staleness=1, many=True)
 
