@@ -167,6 +167,8 @@ def workload_key(gpus: int, override):
 def kernel_name(variant, optimizer, n, staleness=0):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
     if staleness:
+        if 2 <= n <= 4 and variant == "auto":   # ea_api.cu: the lane kernel with x~_{t-1} staged beside x~_t
+            return "colocated_laneshfl<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"
     two_state = optimizer in ("adam", "adamw")
     if n > 8 or (two_state and n > 6 and variant == "auto"):
@@ -188,7 +190,9 @@ def colocated_launches(n, k, args, batched):
     ASGD, the step-counter kernel that precedes each launch."""
     coef = args.optimizer != "sgd"
     two_state = args.optimizer in ("adam", "adamw")
-    per_stage = n > 8 or not batched or (two_state and n > 6 and args.variant == "auto") or args.staleness
+    stale_lane = args.staleness and 2 <= n <= 4 and args.variant == "auto"
+    per_stage = (n > 8 or not batched or (two_state and n > 6 and args.variant == "auto")
+                 or (args.staleness and not stale_lane))
     launches = k if per_stage else (k + 7) // 8
     return launches * (2 if coef else 1)
 

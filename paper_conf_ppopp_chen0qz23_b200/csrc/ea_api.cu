@@ -282,6 +282,46 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // pipeline and 0.73 lane kernel, profiles/r01_adam_nsweep.jsonl)
   const bool adam_wide = ea::two_state(opt) && n > 6 && h->variant == 0;
   const bool stale = h->cfg.staleness == 1;
+  // stale center: the lane kernel with x~_{t-1} staged beside x~_t for 2 <= N <= 4 under the default variant, else
+  // the replica loop (AVGPIPE_EA_FORCE_WIDE=1 selects the replica loop for A/B measurement)
+  const bool stale_lane = stale && n >= 2 && n <= ea::kMaxStaleLaneN && h->variant == 0 && !force_wide;
+  auto stale_prev = [&](int st, const float* center) -> float* {
+    float* prev = h->prev[st];
+    if (!h->prev_init[st]) {  // x~_{-1} := x~_0 (c28)
+      e = cudaMemcpyAsync(prev, center, sizeof(float) * h->p[st], cudaMemcpyDeviceToDevice, s);
+      if (e != cudaSuccess) return nullptr;
+      h->prev_init[st] = 1;
+    }
+    return prev;
+  };
+  if (stale_lane) {
+    for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
+      const int cnt = count - j0 < ea::kMaxLaunchStages ? count - j0 : ea::kMaxLaunchStages;
+      ea_status st2 = advance(h, stages + j0, cnt, s);
+      if (st2 != EA_OK) return st2;
+      ea::StageBatch b;
+      b.nstages = 0;
+      for (int j = j0; j < j0 + cnt; ++j) {
+        const int st = stages[j];
+        ea::StageRefs& r = b.st[b.nstages++];
+        for (int i = 0; i < ea::kMaxFusedN; ++i) {
+          const bool on = i < n;
+          r.x[i] = on ? replica_ptrs[j * n + i] : nullptr;
+          r.g[i] = on ? grad_ptrs[j * n + i] : nullptr;
+          r.m[i] = on ? state_ptr(h, 0, st, i) : nullptr;
+          r.v[i] = (on && two) ? state_ptr(h, 1, st, i) : nullptr;
+        }
+        r.c = center_ptrs[j];
+        r.p = h->p[st];
+        r.scp = h->d_coef + st;
+        r.prev = stale_prev(st, center_ptrs[j]);
+        if (!r.prev) return cuda_fail(h, e, "stale-center init");
+      }
+      e = ea::launch_colocated_batch_stale(b, n, h->hp, opt, h->num_sms, s);
+      if (e != cudaSuccess) return cuda_fail(h, e, "co-located stale kernel launch");
+    }
+    return EA_OK;
+  }
   if (n > ea::kMaxFusedN || force_wide || adam_wide || stale) {  // replica loop: one launch per stage
     for (int j = 0; j < count; ++j) {
       const int st = stages[j];
@@ -296,12 +336,8 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
       if (st2 != EA_OK) return st2;
       float* prev = nullptr;
       if (stale) {
-        prev = h->prev[st];
-        if (!h->prev_init[st]) {  // x~_{-1} := x~_0 (c28)
-          e = cudaMemcpyAsync(prev, center_ptrs[j], sizeof(float) * h->p[st], cudaMemcpyDeviceToDevice, s);
-          if (e != cudaSuccess) return cuda_fail(h, e, "stale-center init");
-          h->prev_init[st] = 1;
-        }
+        prev = stale_prev(st, center_ptrs[j]);
+        if (!prev) return cuda_fail(h, e, "stale-center init");
       }
       e = ea::launch_colocated_wide(t, n, center_ptrs[j], prev, h->p[st], h->hp, opt, h->d_coef + st, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");

@@ -72,6 +72,7 @@ struct StageRefs {
   float* c;
   int64_t p;             // elements
   const StepCoef* scp;   // device: this stage's Adam coefficients (unused by SGD)
+  float* prev = nullptr; // staleness 1 (row f4): x~_{t-1}, read by the replicas, then set to x~_t
 };
 
 // Up to kMaxLaunchStages stages updated by ONE launch (same N).
@@ -102,6 +103,13 @@ enum KernelVariant : int {
 // place, one launch.  Adam/AdamW always use the lane kernel.
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s);
+
+// Stale center (row f4) for a batch of stages with 2 <= N <= kMaxStaleLaneN (N = 1's two 16 KB tiles
+// double-buffered exceed static shared memory), every st[].prev set: the lane kernel
+// with x~_{t-1} staged beside x~_t (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
+constexpr int kMaxStaleLaneN = 4;
+cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int num_sms,
+                                         cudaStream_t s);
 
 // Co-located step for one stage with any N <= kMaxReplicas (replica loop).  prev != nullptr: stale
 // center (row f4): replicas use prev (x~_{t-1}), center is updated from x~_t, prev <- x~_t.

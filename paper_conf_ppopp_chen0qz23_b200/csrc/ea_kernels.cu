@@ -137,21 +137,24 @@ __device__ __forceinline__ StepCoef load_coef(const StepCoef* scp) {
 }
 
 // Scalar tail of one stage: elements [4*(p/4), p) (fewer than 4), one thread.
-template <int N, int OPT>
+// STALE: the replicas see st.prev[j] (x~_{t-1}) and st.prev[j] becomes x~_t (row f4).
+template <int N, int OPT, bool STALE = false>
 __device__ void stage_tail(const StageRefs& st, const Hyper& hp) {
   const StepCoef sc = load_coef<OPT>(st.scp);
   for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
     const float c = st.c[j];
+    const float cu = STALE ? st.prev[j] : c;
     float acc = 0.f;
 #pragma unroll
     for (int i = 0; i < N; ++i) {
       float x = st.x[i][j], m = st.m[i][j], v = two_state(OPT) ? st.v[i][j] : 0.f;
-      acc += ea_elem<OPT>(x, st.g[i][j], m, v, c, hp, sc);
+      acc += ea_elem<OPT>(x, st.g[i][j], m, v, cu, hp, sc);
       st.x[i][j] = x;
       st.m[i][j] = m;
       if (two_state(OPT)) st.v[i][j] = v;
     }
     st.c[j] = fmaf(acc, hp.inv_n, c);
+    if (STALE) st.prev[j] = c;
   }
 }
 
@@ -452,12 +455,16 @@ struct LaneGeom {
   static constexpr int kTileVec = (kThreads / 32) * kVecPerWarp;  // float4 of center per tile
 };
 
-template <int N, int HINT, int OPT, int PASSES = kLanePasses, int MINB = 1>
+// STALE (row f4, reading c28): every stage's x~_{t-1} tile (st.prev) is staged beside x~_t by a second bulk
+// copy on the same mbarrier; the replicas dilute with and measure their gap to x~_{t-1}, replica-0 lanes write
+// x~_{t+1} = x~_t + R/N and copy x~_t into prev.
+template <int N, int HINT, int OPT, int PASSES = kLanePasses, int MINB = 1, bool STALE = false>
 __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const StageBatch b, const Hyper hp) {
   using G = LaneGeom<N, PASSES>;
   constexpr int CH = G::CH, kPasses = PASSES, kVecPerWarp = G::kVecPerWarp, kTileVec = G::kTileVec;
   constexpr bool kTwoState = two_state(OPT);
   __shared__ __align__(128) float4 s_center[2][kTileVec];
+  __shared__ __align__(128) float4 s_prev[2][STALE ? kTileVec : 1];
   __shared__ __align__(8) uint64_t s_bar[2];
   const Mem<HINT> mem;
 
@@ -476,8 +483,9 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
 
   auto issue = [&](int s, int64_t v0, int64_t nv, int buf) {
     const uint32_t bytes = static_cast<uint32_t>(nv * 16);
-    mbar_expect_tx(&s_bar[buf], bytes);
+    mbar_expect_tx(&s_bar[buf], STALE ? 2 * bytes : bytes);
     bulk_g2s(&s_center[buf][0], b.st[s].c + 4 * v0, bytes, &s_bar[buf]);
+    if (STALE) bulk_g2s(&s_prev[buf][0], b.st[s].prev + 4 * v0, bytes, &s_bar[buf]);
   };
 
   WaveCursor cur{0, 0};
@@ -529,9 +537,10 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
       const int lv = warp * kVecPerWarp + k * CH + chunk;
       const bool in = lv < nv;  // uniform across the NP lanes of a chunk
       const float4 c = in ? s_center[buf][lv] : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float4 cu = (STALE && in) ? s_prev[buf][lv] : c;  // the center the replicas see
       float4 r = make_float4(0.f, 0.f, 0.f, 0.f);
       if (active && in) {
-        r = ea_vec<OPT>(x[k], g[k], m[k], w[k], c, hp, sc);
+        r = ea_vec<OPT>(x[k], g[k], m[k], w[k], cu, hp, sc);
         const int64_t v = v0 + lv;
         mem.st(xi + 4 * v, x[k]);
         mem.st(mi + 4 * v, m[k]);
@@ -544,7 +553,10 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
         r.z += __shfl_xor_sync(0xffffffffu, r.z, off);
         r.w += __shfl_xor_sync(0xffffffffu, r.w, off);
       }
-      if (rep == 0 && in) mem.st(st.c + 4 * (v0 + lv), center_apply(c, r, hp.inv_n));
+      if (rep == 0 && in) {
+        mem.st(st.c + 4 * (v0 + lv), center_apply(c, r, hp.inv_n));
+        if (STALE) mem.st(st.prev + 4 * (v0 + lv), c);
+      }
     }
     __syncthreads();  // everyone done reading s_center[buf] before it is refilled
     buf ^= 1;
@@ -554,7 +566,7 @@ __global__ void __launch_bounds__(kThreads, MINB) colocated_laneshfl(const Stage
     nv = nv_next;
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
 // ============================================================================
@@ -866,9 +878,9 @@ int lane_tune() {
   return v;
 }
 
-template <int N, int HINT, int OPT, int PASSES, int MINB>
+template <int N, int HINT, int OPT, int PASSES, int MINB, bool STALE = false>
 cudaError_t launch_laneshfl_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  auto k = colocated_laneshfl<N, HINT, OPT, PASSES, MINB>;
+  auto k = colocated_laneshfl<N, HINT, OPT, PASSES, MINB, STALE>;
   k<<<persistent_grid(k, units_of(b, LaneGeom<N, PASSES>::kTileVec), num_sms), kThreads, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
@@ -1084,6 +1096,29 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
     case 6: return launch_n<6>(b, hp, opt, variant, num_sms, s);
     case 7: return launch_n<7>(b, hp, opt, variant, num_sms, s);
     case 8: return launch_n<8>(b, hp, opt, variant, num_sms, s);
+    default: return cudaErrorInvalidValue;
+  }
+}
+
+template <int N>
+cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
+  switch (opt) {
+    case kOptAdam: return launch_laneshfl_t<N, 0, kOptAdam, kLanePasses, 2, true>(b, hp, num_sms, s);
+    case kOptAdamW: return launch_laneshfl_t<N, 0, kOptAdamW, kLanePasses, 2, true>(b, hp, num_sms, s);
+    case kOptASGD: return launch_laneshfl_t<N, 0, kOptASGD, kLanePasses, 2, true>(b, hp, num_sms, s);
+    default: return launch_laneshfl_t<N, 0, kOptSGD, kLanePasses, 2, true>(b, hp, num_sms, s);
+  }
+}
+
+cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int num_sms,
+                                         cudaStream_t s) {
+  if (b.nstages <= 0) return cudaSuccess;
+  for (int t = 0; t < b.nstages; ++t)
+    if (!b.st[t].prev) return cudaErrorInvalidValue;
+  switch (n) {
+    case 2: return launch_stale_n<2>(b, hp, opt, num_sms, s);
+    case 3: return launch_stale_n<3>(b, hp, opt, num_sms, s);
+    case 4: return launch_stale_n<4>(b, hp, opt, num_sms, s);
     default: return cudaErrorInvalidValue;
   }
 }
