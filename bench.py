@@ -166,6 +166,9 @@ def workload_key(gpus: int, override):
 # ----------------------------------------------------------------------------- our arm
 def kernel_name(variant, optimizer, n, staleness=0):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
+    force_wide = os.environ.get("AVGPIPE_EA_FORCE_WIDE", "")[:1] == "1"   # ea_api.cu measurement knob
+    if force_wide:
+        return "colocated_wide" + ("<stale>" if staleness else "")
     if staleness:
         if 2 <= n <= 4 and variant == "auto":   # ea_api.cu: the lane kernel with x~_{t-1} staged beside x~_t
             return "colocated_laneshfl<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
@@ -191,8 +194,9 @@ def colocated_launches(n, k, args, batched):
     coef = args.optimizer != "sgd"
     two_state = args.optimizer in ("adam", "adamw")
     stale_lane = args.staleness and 2 <= n <= 4 and args.variant == "auto"
+    force_wide = os.environ.get("AVGPIPE_EA_FORCE_WIDE", "")[:1] == "1"   # ea_api.cu measurement knob
     per_stage = (n > 8 or not batched or (two_state and n > 6 and args.variant == "auto")
-                 or (args.staleness and not stale_lane))
+                 or (args.staleness and not stale_lane) or force_wide)
     launches = k if per_stage else (k + 7) // 8
     return launches * (2 if coef else 1)
 
