@@ -45,7 +45,9 @@ def _worker(rank, K, N, M, extra, dynamic, port, q):
                 m.zero_grad()
             st.run_iteration(inputs=xs if rank == 0 else None, targets=ys if rank == K - 1 else None,
                              loss_fn=loss_fn, act_shape=(B, D), act_dtype=torch.float32)
-        grads = [[p.grad.clone() for p in m.parameters()] for m in stage_mods]
+        # numpy copies are pickled by value: tensors would travel as shared-memory file descriptors, which fail
+        # (FileNotFoundError) when this process exits before the parent has received them
+        grads = [[p.grad.detach().numpy().copy() for p in m.parameters()] for m in stage_mods]
         q.put((rank, "ok", grads, st.history))
     except Exception as e:  # pragma: no cover
         import traceback
@@ -72,7 +74,7 @@ def _run(K, N, M, extra, dynamic=False):
     for _ in range(K):
         r, status, grads, hist = q.get(timeout=300)
         assert status == "ok", status
-        out[r] = (grads, hist)
+        out[r] = ([[torch.from_numpy(a) for a in gm] for gm in grads], hist)
     for p in procs:
         p.join(timeout=60)
     return out
