@@ -101,7 +101,42 @@ def measured_peaks():
     return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-NVLINK_PEAK_GBS = 770.0   # measured peer copy per direction (B200_PROFILING.md)
+NVLINK_PEAK_GBS = 770.0   # B200_PROFILING.md: measured peer copy per direction per GPU (900 GB/s nominal)
+NVLINK_PEAK_SOURCE = ("measured reference in /opt/skills/guides/B200_PROFILING.md: peer copy 770 GB/s per direction "
+                      "per GPU (8-rank all-reduce busBW 725 GB/s at 1 GiB; 900 GB/s nominal NVLink 5)")
+
+
+def nccl_debug_setup(rank):
+    """NCCL_DEBUG=INFO into a per-rank file (unless the caller set NCCL_DEBUG), so the line can report the
+    algorithm / protocol / NVLS NCCL chose for the library's communicator."""
+    if "NCCL_DEBUG" in os.environ:
+        return os.environ.get("NCCL_DEBUG_FILE")
+    import tempfile
+    path = os.path.join(tempfile.gettempdir(), f"avgpipe_nccl_{os.getpid()}_{rank}.log")
+    os.environ["NCCL_DEBUG"] = "INFO"
+    os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT,TUNING,NVLS")
+    os.environ["NCCL_DEBUG_FILE"] = path
+    return path
+
+
+def nccl_debug_summary(path, limit=12):
+    """Distinct NCCL INFO lines that name the algorithm / protocol / NVLS / channels of the communicators."""
+    if not path or not os.path.exists(path):
+        return None
+    import re
+    keep, seen = [], set()
+    pat = re.compile(r"(algo|Algo|proto|Proto|NVLS|nvls|CollNet|Channel \d+/|channels|Ring|Tree|comm 0x.*nRanks)")
+    for line in open(path, errors="replace"):
+        if "NCCL INFO" not in line or not pat.search(line):
+            continue
+        msg = re.sub(r"^.*NCCL INFO ", "", line.strip())
+        msg = re.sub(r"0x[0-9a-f]+", "0x..", msg)
+        if msg not in seen:
+            seen.add(msg)
+            keep.append(msg)
+        if len(keep) >= limit:
+            break
+    return keep
 
 
 class ClockSampler:
@@ -222,6 +257,7 @@ def run_ours(args, rank, world, local):
     from paper_conf_ppopp_chen0qz23_b200 import parallel
 
     shared = shared_gpu_test_mode()
+    nccl_log = None
     if shared:
         local = 0
     torch.cuda.set_device(local)
@@ -247,11 +283,12 @@ def run_ours(args, rank, world, local):
             dist.init_process_group("gloo")
             uid = None
         else:
+            nccl_log = nccl_debug_setup(rank)
             dist.init_process_group("nccl", device_id=dev)
             uid = parallel.broadcast_unique_id()
         h = ElasticAveraging(sizes, n, alpha=a, beta=b, rho=r, lr=lr, momentum=synth.MOMENTUM,
                              layout="spread", rank=rank, world=world, device=local, nccl_id=uid,
-                             optimizer=args.optimizer, exchange=args.exchange)
+                             optimizer=args.optimizer, exchange=args.exchange, staleness=args.staleness)
         if shared and world > 1:
             parallel.connect_p2p(h)      # IPC handles over the gloo group
         state = []
@@ -316,10 +353,9 @@ def run_ours(args, rank, world, local):
     if spread:
         dist.barrier()
     # per-launch events for the dominant kernel (co-located: every ea_step is one kernel)
-    ev = None
-    if not spread or args.exchange == "nccl":   # spread + NCCL: events bracket each stage's local kernel
-        ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-               for _ in (range(1) if batched else sizes)] for _ in range(args.steps)]
+    # spread: events bracket each stage's local kernel (the exchange is on the library's side stream)
+    ev = [[(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+           for _ in (range(1) if batched else sizes)] for _ in range(args.steps)]
     t0, t1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         torch.cuda.synchronize()
@@ -374,44 +410,40 @@ def run_ours(args, rank, world, local):
         out["gbps"] = step_bytes / (ms * 1e-3) / 1e9
         nv_gbs = nv_bytes / (ms * 1e-3) / 1e9
         nvlink = {"bound": "nvlink", "achieved": nv_gbs, "peak": NVLINK_PEAK_GBS, "unit": "GB/s",
-                  "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None,
-                  "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / "
-                          "step time; peak = measured peer copy per direction"}
-        local = None
-        if ev is not None:
-            # the local kernel (rows a1-a4) runs on the caller's stream between each stage's events;
-            # the exchange runs on the library's side stream, outside them
-            kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(len(sizes))]
-            avg_ms = sum(kern_ms) / len(kern_ms)
-            per_launch_bytes = step_bytes / len(sizes)
-            achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
-            local = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
-                     "traffic": None, "kernel": "spread_bulkpipe" + ("" if args.optimizer == "sgd" else
-                                                                     "<" + args.optimizer + ">"),
-                     "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
-                     "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
-        if args.exchange == "p2p":
-            # the fused kernel's own HBM bytes per rank and element: phase A 28 (SGD/ASGD; Adam 36,
-            # r included), phase B 4 + 12/N, phase C 8 (N-1)/N -- 40 + 4/N for SGD
-            a_bytes = 28 if args.optimizer not in ("adam", "adamw") else 36
-            hbm_bytes = sum((a_bytes + 4 + 12 / n + 8 * (n - 1) / n) * h.center_capacity(s) for s in range(len(sizes)))
-            hbm_gbs = hbm_bytes / (ms * 1e-3) / 1e9
-            local = {"bound": "hbm", "achieved": hbm_gbs, "peak": peak, "unit": "GB/s", "frac": hbm_gbs / peak,
-                     "traffic": None, "kernel": "spread_p2p" + ("" if args.optimizer == "sgd" else
-                                                                "<" + args.optimizer + ">"),
-                     "bytes_per_step": hbm_bytes, "peak_source": peak_src,
-                     "note": "whole step (one fused kernel per stage): the kernel's HBM bytes / step time"}
-        if world == 1 and local is not None:
+                  "frac": nv_gbs / NVLINK_PEAK_GBS, "traffic": None, "peak_source": NVLINK_PEAK_SOURCE,
+                  "traffic_note": "ncu has no NVLink byte counter on a one-GPU capture; the bytes are the "
+                                  "algorithmic (ring busBW) volume",
+                  "bytes_per_step": nv_bytes,
+                  "note": "whole step: per-GPU NVLink bytes 2(N-1)/N*4*P_pad (ring busBW convention) / step time"}
+        # the local kernel (rows a1-a4; p2p: + the pushes into the owners' inboxes) runs on the caller's stream
+        # between each stage's events; the exchange runs on the library's side stream, outside them
+        kern = ("p2p_push" if args.exchange == "p2p" else "spread_bulkpipe") + \
+            ("" if args.optimizer == "sgd" else "<" + args.optimizer + ">")
+        kern_ms = [ev[k][j][0].elapsed_time(ev[k][j][1]) for k in range(args.steps) for j in range(len(sizes))]
+        avg_ms = sum(kern_ms) / len(kern_ms)
+        if args.exchange == "p2p":   # the push kernel reads/writes the padded vectors (28 / 36 B per element)
+            launch_bytes = [bytes_spread_local(h.center_capacity(s), args.optimizer) for s in range(len(sizes))]
+        else:
+            launch_bytes = [bytes_spread_local(p, args.optimizer) for p in sizes]
+        per_launch_bytes = sum(launch_bytes) / len(sizes)
+        achieved = per_launch_bytes / (avg_ms * 1e-3) / 1e9
+        local = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+                 "traffic": traffic_from_profiles(cfg.name, kern), "kernel": kern,
+                 "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
+                 "share_of_step": sum(kern_ms) / args.steps / ms, "peak_source": peak_src}
+        if world == 1:
             out["roofline"] = local     # no NVLink traffic at world 1: the local kernel is the bound
-            if args.exchange == "nccl":
-                local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
-                                 "(NCCL copy + shard update) shares HBM on the side stream")
+            local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
+                             "(side stream) shares HBM")
         else:
             out["roofline"] = nvlink
-            if local is not None:
-                out["local_kernel_roofline"] = local
-        per_stage = 2 if args.exchange == "p2p" else (2 if args.optimizer == "sgd" else 3)
-        out["gpu_launches"] = args.steps * per_stage * len(sizes)   # ours only (NCCL kernels excluded)
+            out["local_kernel_roofline"] = local
+        if args.exchange == "nccl":
+            out["config"]["nccl"] = nccl_debug_summary(nccl_log)
+        # ours per stage: the local kernel + the shard update (NCCL) or the exchange kernel (p2p), and the
+        # step-counter kernel when something on the device consumes the step count (Adam/ASGD, the p2p epoch)
+        per_stage = 2 + (1 if (args.optimizer != "sgd" or args.exchange == "p2p") else 0)
+        out["gpu_launches"] = args.steps * per_stage * len(sizes)   # NCCL's own kernels excluded
     out["clocks"] = clk.summary()
     if not spread:
         out["copy_gbs_same_box"] = same_box_copy_gbs(dev)
@@ -419,9 +451,10 @@ def run_ours(args, rank, world, local):
         out["e2e"] = e2e_colocated(h, state, sizes, n, args, stream, dev, order)
     elif spread and not args.no_e2e:
         out["e2e"] = e2e_spread(h, state, sizes, args, stream, dev, order, rank, world)
-    if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        out["cpu_baseline"] = cpu_baseline(cfg, n, seconds=args.cpu_seconds)
     h.close()
+    if rank == 0 and not args.no_cpu_baseline:
+        # N > 1: one stage-shard (P_s/N elements x N replicas) on rank 0, per-element rate extrapolated
+        out["cpu_baseline"] = cpu_baseline(cfg, n, seconds=args.cpu_seconds, shard=world > 1)
     if rank == 0:
         emit(out)
     if spread:
@@ -568,12 +601,14 @@ def cpu_model():
     return None
 
 
-def cpu_baseline(cfg, n, seconds=10.0):
+def cpu_baseline(cfg, n, seconds=10.0, shard=False):
     """The float64 oracle, as it stands (single-threaded numpy), on a bounded
-    sample: one full stage of the workload, repeated until `seconds` pass."""
+    sample: one full stage of the workload (shard=True, the N>1 lines: one
+    stage-shard of P_s/N elements x N replicas, SURVEY §8(d) -- the full C3-C5
+    float64 state exceeds host RAM), repeated until `seconds` pass."""
     from oracle.ea_oracle import Hyper, ea_step
     from paper_conf_ppopp_chen0qz23_b200 import synth
-    p = cfg.stage_sizes[0]
+    p = cfg.stage_sizes[0] // (n if shard else 1)
     a, b, r = synth.mode_coeffs(MODE, n)
     hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
     xs, ms, c, g = _oracle_sample(n, p)
@@ -584,9 +619,13 @@ def cpu_baseline(cfg, n, seconds=10.0):
         el = time.perf_counter() - t0
         if el >= seconds:
             break
+    what = f"stage-shard (P_s/N of {cfg.stage_sizes[0]})" if shard else "stage"
     out = {"value": n * p * steps / el, "unit": UNIT, "cores": 1, "kind": "oracle",
-           "sample": f"{steps} oracle steps of one {p}-element stage x N={n} (float64 numpy, 1 thread), "
+           "sample": f"{steps} oracle steps of one {p}-element {what} x N={n} (float64 numpy, 1 thread), "
                      f"{el:.1f} s", "host_cores_available": len(os.sched_getaffinity(0)), "cpu_model": cpu_model()}
+    if shard:
+        out["extrapolated"] = ("per-element rate of one stage-shard; the whole job's state does not fit host RAM "
+                               "in float64 (SURVEY §8(d))")
     out["all_cores"] = cpu_baseline_all_cores(xs, ms, c, g, hp, seconds=seconds / 2)
     return out
 
@@ -618,10 +657,19 @@ def cpu_baseline_all_cores(xs, ms, c, g, hp, seconds=5.0):
                       f"on {cores} threads (float64 numpy), {el:.1f} s"}
 
 
+REFERENCE_BUDGET_S = 150.0   # the reference arm's timed steps + warm-up stay within a few minutes
+
+
 def run_reference(args, rank, world):
-    """--impl reference: the float64 oracle on host cores; rank 0 only."""
+    """--impl reference: the float64 oracle, as it stands, on host cores; rank 0 only.
+
+    N = 1: the WHOLE workload (every stage, every replica, full size) per step when K + W steps fit
+    REFERENCE_BUDGET_S (C2: ~2.3 s per step on one core), else the same leading fraction of every stage.
+    N > 1: one stage-shard (P_s/N elements x N replicas) per step, per-element rate extrapolated to the job
+    (the full C3-C5 float64 state does not fit host RAM)."""
     if rank != 0:
         return
+    import numpy as np
     from oracle.ea_oracle import Hyper, ea_step
     from paper_conf_ppopp_chen0qz23_b200 import synth
     key = workload_key(world, args.config)
@@ -629,25 +677,63 @@ def run_reference(args, rank, world):
     n = cfg.n_pipelines if world == 1 else world
     a, b, r = synth.mode_coeffs(MODE, n)
     hp = Hyper(alpha=a, beta=b, rho=r, lr=synth.LR, momentum=synth.MOMENTUM)
-    p_sample = 1 << 16      # per-step bounded sample: 65,536 elements x N replicas
-    xs, ms, c, g = _oracle_sample(n, p_sample)
-    for _ in range(args.warmup):
-        xs, ms, c = ea_step(xs, ms, c, g, hp)
+    if world == 1:
+        parts = list(cfg.stage_sizes)
+    else:
+        parts = [cfg.stage_sizes[0] // n]
+    states = [_oracle_sample(n, p, seed=s) for s, p in enumerate(parts)]
+
+    def one_step(states, frac=1.0):
+        out = []
+        for xs, ms, c, g in states:
+            if frac < 1.0:
+                k = max(1, int(len(c) * frac))
+                xk, mk, ck = ea_step([x[:k] for x in xs], [m[:k] for m in ms], c[:k], [gi[:k] for gi in g], hp)
+                for x, v in zip(xs, xk):
+                    x[:k] = v
+                for m, v in zip(ms, mk):
+                    m[:k] = v
+                c[:k] = ck
+                out.append((xs, ms, c, g))
+            else:
+                xs2, ms2, c2 = ea_step(xs, ms, c, g, hp)
+                out.append((xs2, ms2, c2, g))
+        return out
+
+    t0 = time.perf_counter()
+    states = one_step(states)                # calibration (counts as one warm-up step)
+    t_full = time.perf_counter() - t0
+    frac = min(1.0, REFERENCE_BUDGET_S / max(t_full * (args.steps + max(args.warmup - 1, 0)), 1e-9))
+    for _ in range(max(args.warmup - 1, 0)):
+        states = one_step(states, frac)
     t0 = time.perf_counter()
     for _ in range(args.steps):
-        xs, ms, c = ea_step(xs, ms, c, g, hp)
+        states = one_step(states, frac)
     el = time.perf_counter() - t0
+    elems = sum(max(1, int(p * frac)) if frac < 1.0 else p for p in parts)
     ms_step = el / args.steps * 1e3
-    value = n * p_sample / (el / args.steps)
-    sample = f"each step: {p_sample} elements x N={n} replicas of {cfg.name} (float64 numpy, 1 thread)"
+    value = n * elems / (el / args.steps)
+    if world == 1 and frac >= 1.0:
+        sample = f"the whole workload each step: {len(parts)} stages x {parts[0]} elements x N={n} replicas"
+    elif world == 1:
+        sample = (f"each step: the leading {frac:.3f} of every stage ({elems} of {sum(parts)} elements) x N={n} "
+                  f"replicas (K + W steps of the whole workload exceed {REFERENCE_BUDGET_S:.0f} s)")
+    else:
+        sample = f"each step: one stage-shard, {parts[0]} elements (P_s/N) x N={n} replicas; rate extrapolated"
+    same = world == 1 and frac >= 1.0
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "weak",
-           "vs_baseline": None, "dtype": "f64", "data": "synthetic", "impl": "reference",
-           "config": {"workload": cfg.name, "n_pipelines": n, "params_per_step_sample": p_sample, "mode": MODE},
-           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle", "sample": sample,
-                            "cpu_model": cpu_model()},
+           "vs_baseline": None, "dtype": "f64", "data": "synthetic (seeded numpy PCG64, synth.host_state)",
+           "impl": "reference",
+           "config": {"workload": cfg.name, "n_pipelines": n, "params_per_step_sample": elems, "mode": MODE,
+                      "same_config": same},
+           "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
+                            "sample": sample + " (float64 numpy, 1 thread)", "cpu_model": cpu_model(),
+                            "host_cores_available": len(os.sched_getaffinity(0))},
            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
            "gpu_launches": 0}
+    if not same:
+        out["cpu_baseline"]["extrapolated"] = "per-element rate of the sample"
     emit(out)
 
 

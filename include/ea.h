@@ -73,6 +73,7 @@ extern "C" {
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
+#define EA_SLOT_CENTER_PREV 2  /* ea_get_state / ea_set_state slot of the stale center x~_{t-1} (staleness 1) */
 
 typedef enum {
   EA_OK = 0,
@@ -94,9 +95,10 @@ typedef enum { EA_OPT_SGD = 0, EA_OPT_ADAM = 1, EA_OPT_ADAMW = 2, EA_OPT_ASGD = 
 /* How EA_SPREAD exchanges contributions and the center (rows a6/a7). */
 typedef enum {
   EA_XCHG_NCCL = 0,  /* ncclReduceScatter -> shard update kernel -> in-place ncclAllGather on a side stream */
-  EA_XCHG_P2P = 1    /* ONE fused kernel per stage: local update, contributions pushed into the owners'
-                        inboxes over NVLink peer memory (CUDA IPC), owner reduction + center update,
-                        center chunks pulled back -- overlapped chunk by chunk (see ea_p2p.cu) */
+  EA_XCHG_P2P = 1    /* the library's own peer-memory kernels (CUDA IPC mappings over NVLink): p2p_push
+                        on the caller's stream (local update, contributions stored straight into the
+                        owners' inboxes), p2p_exchange on the side stream (owner reduction + center
+                        update, center chunks pulled back), see ea_p2p.cu */
 } ea_exchange;
 
 typedef struct {
@@ -128,9 +130,13 @@ typedef struct {
   int32_t exchange;             /* EA_SPREAD: ea_exchange (ignored for EA_COLOCATED) */
   int32_t staleness;            /* 0: synchronous center (c3); 1: the replicas see the center one step
                                    late, x~_{t-1}, as with the paper's asynchronous queues (
-                                   reading c28, row f4).  1 needs EA_COLOCATED (any optimizer); the
-                                   library keeps x~_{t-1} (P_s floats per stage, 8 B/element/step).
-                                   Any optimizer. */
+                                   reading c28, row f4).  Any optimizer; EA_COLOCATED, or EA_SPREAD with
+                                   EA_XCHG_NCCL (there the local step of iteration t waits only for the
+                                   snapshot of x~_t taken at the start of exchange t-1, so that exchange
+                                   overlaps the whole iteration t).  The library keeps x~_{t-1} (P_s
+                                   floats per stage, slot EA_SLOT_CENTER_PREV); x~_{-1} := x~_0 at the
+                                   stage's first step, which must not be taken while the stream is
+                                   capturing a CUDA graph (EA_ESTATE) unless the slot was set. */
   double asgd_lambd;            /* ASGD: decay term l >= 0 (torch default 1e-4) */
   double asgd_alpha;            /* ASGD: power a of the eta schedule (torch default 0.75) */
   double asgd_t0;               /* ASGD: step after which averaging starts, >= 0 (torch default 1e6) */
@@ -187,8 +193,10 @@ EA_API int64_t ea_shard_elems(ea_handle h, int32_t stage);
  * shard update -> all-gather) runs on the library's side stream and `stream`
  * does NOT wait for it -- the next forward and the other stages' local steps
  * proceed while the center is exchanged (never block the
- * pipelines).  EA_XCHG_P2P: one fused kernel on `stream` (local update and
- * exchange).  Call ea_sync before reading x~ on any stream.  All ranks must
+ * pipelines).  EA_XCHG_P2P: the same split -- the push kernel (local update,
+ * contributions pushed to the owners over peer memory) on `stream`, the
+ * owner reduction and the pull of the other shards on the side stream.  Call
+ * ea_sync before reading x~ on any stream.  All ranks must
  * call ea_step for the same stages in the same order (collective ordering).
  * Pointers must stay valid until the work completes. */
 EA_API ea_status ea_step(ea_handle h, int32_t stage, float* const* replica_ptrs,
@@ -261,16 +269,22 @@ EA_API ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard
 /* *state_dev = device pointer to optimizer-state slot `slot` of (stage,
  * replica): P_s floats, owned by the library, valid until ea_destroy.
  * slot 0 = SGD momentum / Adam first moment / ASGD average, slot 1 = Adam second moment
- * (EA_EINVAL for SGD and ASGD).  EA_SPREAD: replica must be 0. */
+ * (EA_EINVAL for SGD and ASGD), slot EA_SLOT_CENTER_PREV = the stale center
+ * x~_{t-1} of a staleness-1 handle (replica 0; defined after the stage's first
+ * step or an ea_set_state of the slot).  EA_SPREAD: replica must be 0. */
 EA_API ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, float** state_dev);
 
 /* Copy P_s floats from device pointer src into state slot `slot` of (stage,
- * replica), ordered on `stream` (after pending EA_SPREAD side-stream work). */
+ * replica), ordered on `stream` (after pending EA_SPREAD side-stream work).
+ * Setting EA_SLOT_CENTER_PREV marks x~_{t-1} as given (checkpoint resume; no
+ * x~_{-1} := x~_0 initialisation at the next step). */
 EA_API ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, const float* src,
                               void* stream);
 
 /* Step count t of `stage` (number of ea_step / ea_spread_local calls so far;
- * Adam's bias correction uses t+1 for the next step). */
+ * Adam's bias correction uses t+1 for the next step).  ea_set_step changes
+ * only the optimizer's t (resume); the peer-memory exchange keeps its own
+ * epoch counter, which every rank advances once per ea_step. */
 EA_API ea_status ea_get_step(ea_handle h, int32_t stage, int64_t* step);
 EA_API ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step);
 
@@ -284,7 +298,11 @@ EA_API ea_status ea_set_step(ea_handle h, int32_t stage, int64_t step);
 EA_API ea_status ea_set_hyper(ea_handle h, const ea_config* cfg);
 
 /* Wait for outstanding work, free everything the library owns, destroy the
- * communicator.  NULL is a no-op. */
+ * communicator.  EA_XCHG_P2P with an NCCL communicator: a barrier over the
+ * communicator precedes freeing the IPC-exported exchange buffer, so every
+ * rank must call ea_destroy (collective); handles wired with ea_p2p_open /
+ * ea_p2p_connect must be destroyed after a caller-side barrier of all ranks.
+ * NULL is a no-op. */
 EA_API ea_status ea_destroy(ea_handle h);
 
 /* Message of the last failing call on h (h == NULL: this thread's last

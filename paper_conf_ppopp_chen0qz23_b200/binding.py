@@ -25,6 +25,7 @@ OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2, "asgd": 3}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
 ABI_VERSION = 4
+SLOT_CENTER_PREV = 2   # EA_SLOT_CENTER_PREV: the stale center x~_{t-1} (staleness 1)
 
 
 class LibraryNotBuilt(RuntimeError):
@@ -263,6 +264,12 @@ def _ptr(t, what: str) -> int:
     return t.data_ptr()
 
 
+def _numel(t, want: int, what: str):
+    """The C ABI takes bare pointers: a tensor of the wrong size would be read or written past its end."""
+    if t.numel() != want:
+        raise ValueError(f"{what} has {t.numel()} elements, the library expects {want}")
+
+
 def _host_ptr(t, what: str) -> int:
     import torch
     if not isinstance(t, torch.Tensor) or t.dtype != torch.float32 or t.is_cuda or not t.is_contiguous():
@@ -325,14 +332,28 @@ class ElasticAveraging:
         return v
 
     # -- the step
+    def _p(self, stage: int) -> int:
+        if not 0 <= int(stage) < len(self.stage_params):
+            raise EAError(EA_EINVAL, f"stage {stage} out of range")
+        return self.stage_params[int(stage)]
+
+    def _check_stage_tensors(self, stage, reps, gs, center):
+        want = self.n if self.layout == "colocated" else 1
+        if len(reps) != want or len(gs) != want:
+            raise ValueError(f"stage {stage}: need {want} replica and gradient tensors, got {len(reps)}/{len(gs)}")
+        p = self._p(stage)
+        for t in reps:
+            _numel(t, p, f"stage {stage} replica")
+        for t in gs:
+            _numel(t, p, f"stage {stage} gradient")
+        _numel(center, self.center_capacity(stage), f"stage {stage} center (ea_center_capacity)")
+
     def step(self, stage: int, replicas, grads, center, stream=None):
         reps = list(replicas)
         gs = list(grads)
         rp = (ctypes.c_void_p * max(len(reps), 1))(*[_ptr(t, "replica") for t in reps])
         gp = (ctypes.c_void_p * max(len(gs), 1))(*[_ptr(t, "grad") for t in gs])
-        want = self.n if self.layout == "colocated" else 1
-        if len(reps) != want or len(gs) != want:
-            raise ValueError(f"need {want} replica and gradient tensors, got {len(reps)}/{len(gs)}")
+        self._check_stage_tensors(stage, reps, gs, center)
         _check(self._lib.ea_step(self._h, stage, rp, gp, _ptr(center, "center"), _stream_ptr(stream)), self._h)
 
     def step_many(self, stages, replicas, grads, centers, stream=None):
@@ -344,8 +365,7 @@ class ElasticAveraging:
             raise ValueError("stages, replicas, grads, centers must have the same length")
         rp, gp = [], []
         for j in range(len(stages)):
-            if len(replicas[j]) != want or len(grads[j]) != want:
-                raise ValueError(f"stage {stages[j]}: need {want} replica and gradient tensors")
+            self._check_stage_tensors(stages[j], list(replicas[j]), list(grads[j]), centers[j])
             rp += [_ptr(t, "replica") for t in replicas[j]]
             gp += [_ptr(t, "grad") for t in grads[j]]
         k = max(len(stages), 1)
@@ -361,8 +381,8 @@ class ElasticAveraging:
         stages = [int(s) for s in stages]
         rp, gp = [], []
         for j in range(len(stages)):
-            if len(replicas[j]) != self.n or len(host_grads[j]) != self.n:
-                raise ValueError(f"stage {stages[j]}: need {self.n} replica and gradient tensors")
+            self._check_stage_tensors(stages[j], list(replicas[j]), list(host_grads[j]), centers[j])
+            _numel(host_centers_out[j], self._p(stages[j]), f"stage {stages[j]} host center output")
             rp += [_ptr(t, "replica") for t in replicas[j]]
             gp += [_host_ptr(t, "host grad") for t in host_grads[j]]
         k = max(len(stages), 1)
@@ -399,18 +419,27 @@ class ElasticAveraging:
         _check(self._lib.ea_sync(self._h, _stream_ptr(stream)), self._h)
 
     def spread_local(self, stage: int, replica, grad, center, contrib, stream=None):
+        p, cap = self._p(stage), self.center_capacity(stage)
+        _numel(replica, p, "replica")
+        _numel(grad, p, "gradient")
+        _numel(center, cap, "center (ea_center_capacity)")
+        _numel(contrib, cap, "contribution buffer (ea_center_capacity)")
         _check(self._lib.ea_spread_local(self._h, stage, _ptr(replica, "replica"), _ptr(grad, "grad"),
                                          _ptr(center, "center"), _ptr(contrib, "contrib"), _stream_ptr(stream)),
                self._h)
 
     def spread_apply(self, stage: int, center_shard, reduced, stream=None):
+        k = self.shard_elems(stage)
+        _numel(center_shard, k, "center shard (ea_shard_elems)")
+        _numel(reduced, k, "reduced shard (ea_shard_elems)")
         _check(self._lib.ea_spread_apply(self._h, stage, _ptr(center_shard, "center_shard"),
                                          _ptr(reduced, "reduced"), _stream_ptr(stream)), self._h)
 
     # -- optimizer state
     def state(self, stage: int, replica: int, slot: int = 0):
         """Zero-copy torch view of library-owned optimizer state: slot 0 = SGD
-        momentum / Adam first moment / ASGD average ax, slot 1 = Adam second moment."""
+        momentum / Adam first moment / ASGD average ax, slot 1 = Adam second moment,
+        SLOT_CENTER_PREV = the stale center x~_{t-1} (staleness 1, replica 0)."""
         ptr = ctypes.c_void_p()
         _check(self._lib.ea_get_state(self._h, stage, replica, slot, ctypes.byref(ptr)), self._h)
         return _device_view(ptr.value, self.stage_params[stage], self.device)
@@ -419,6 +448,7 @@ class ElasticAveraging:
         return self.state(stage, replica, 0)
 
     def set_state(self, stage: int, replica: int, src, slot: int = 0, stream=None):
+        _numel(src, self._p(stage), "state source")
         _check(self._lib.ea_set_state(self._h, stage, replica, slot, _ptr(src, "state"), _stream_ptr(stream)),
                self._h)
 

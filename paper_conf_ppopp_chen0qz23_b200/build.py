@@ -86,5 +86,25 @@ def build(force: bool = False, verbose: bool = False) -> str:
     return LIB_PATH
 
 
+NCCL_EMU_SRC = os.path.join(ROOT, "tests", "nccl_emu", "nccl_emu.cu")
+NCCL_EMU_LIB = os.path.join(ROOT, "tests", "nccl_emu", "libnccl_emu.so")
+
+
+def build_nccl_emu(force: bool = False) -> str:
+    """Test infrastructure: the in-process NCCL emulation (tests/nccl_emu, LD_PRELOAD) that runs the
+    library's NCCL spread path with N > 1 ranks on one GPU.  Not linked into the product library."""
+    if not force and os.path.exists(NCCL_EMU_LIB) and os.path.getmtime(NCCL_EMU_LIB) >= os.path.getmtime(NCCL_EMU_SRC):
+        return NCCL_EMU_LIB
+    nccl_inc, _ = nccl_dirs()
+    tmp = NCCL_EMU_LIB + ".tmp"
+    cmd = [nvcc(), *ARCH, "-O2", "-std=c++17", "-Xcompiler", "-fPIC", "-shared", "-cudart", "static", "-I", nccl_inc,
+           NCCL_EMU_SRC, "-o", tmp]
+    res = subprocess.run(cmd, capture_output=True, text=True)
+    if res.returncode != 0:
+        raise RuntimeError(f"nvcc failed on {NCCL_EMU_SRC}:\n{res.stdout}\n{res.stderr}")
+    os.replace(tmp, NCCL_EMU_LIB)
+    return NCCL_EMU_LIB
+
+
 if __name__ == "__main__":
     print(build(force="--force" in sys.argv, verbose="-v" in sys.argv))

@@ -53,6 +53,7 @@ struct ea_ctx {
   std::vector<size_t> contrib_off;       // per-stage offset into contrib (floats)
   std::vector<cudaEvent_t> ev_ag;        // per stage: its last all-gather (center final) on the side stream
   std::vector<cudaEvent_t> ev_loc;       // per stage: its last local kernel on the caller's stream
+  std::vector<cudaEvent_t> ev_snap;      // per stage, staleness 1: x~_t copied into prev on the side stream
   float* reduced = nullptr;  // max P_pad/N floats
   ncclComm_t comm = nullptr;
   // EA_SPREAD with exchange == EA_XCHG_P2P (fused peer-memory kernel)
@@ -61,6 +62,7 @@ struct ea_ctx {
   std::vector<size_t> x_inbox, x_outbox, x_arrive, x_ready;  // per-stage byte offsets into xbuf
   std::vector<int64_t> x_nchunks, x_slots;
   int64_t x_chunk = 0;  // floats per exchange chunk (p2p_chunk() at ea_init; every rank must agree)
+  uint32_t* d_xctl = nullptr;  // device: [n_stages] exchange epochs, [n_stages] exchange tickets, [1] abort flag
   std::vector<char*> peer_base;   // world entries, as mapped on this device (self = xbuf)
   std::vector<char> peer_ipc;     // 1 = opened with cudaIpcOpenMemHandle (closed at destroy)
   bool p2p_ready = false;
@@ -73,6 +75,9 @@ struct ea_ctx {
   cudaEvent_t ev_h2d[2] = {nullptr, nullptr}, ev_kern[2] = {nullptr, nullptr}, ev_d2h = nullptr;
   std::string err;
 };
+
+// SMs the spread layout's local kernel leaves free for the side-stream exchange (knob AVGPIPE_EA_SPREAD_RESERVE_SMS).
+constexpr int kSpreadReserveSms = 0;
 
 // Elements per pipelined chunk of the host-buffer path (a multiple of 64).  AVGPIPE_EA_HOST_CHUNK
 // (elements, measurement knob) overrides it up to the staging capacity.
@@ -199,7 +204,8 @@ ea_status advance(ea_ctx* h, const int32_t* stages, int count, cudaStream_t s) {
     cp.opt = h->cfg.optimizer;
     cp.beta1 = h->cfg.beta1; cp.beta2 = h->cfg.beta2; cp.lr = (double)h->cfg.lr;
     cp.lambd = h->cfg.asgd_lambd; cp.asgd_alpha = h->cfg.asgd_alpha; cp.t0 = h->cfg.asgd_t0;
-    cudaError_t e = ea::launch_advance_steps(h->d_steps, h->d_coef, l, cp, s);
+    uint32_t* xepoch = h->d_xctl;  // the peer-memory exchange's own epoch (ea_set_step never touches it)
+    cudaError_t e = ea::launch_advance_steps(h->d_steps, xepoch, h->d_coef, l, cp, s);
     if (e != cudaSuccess) return cuda_fail(h, e, "step-counter kernel launch");
   }
   return EA_OK;
@@ -209,6 +215,16 @@ void free_ctx(ea_ctx* h) {
   if (!h) return;
   cudaSetDevice(h->cfg.device);
   if (h->side) cudaStreamSynchronize(h->side);
+  if (h->comm && h->xbuf && h->p2p_ready && h->cfg.world > 1) {
+    // peers may still read this rank's outbox / write its inbox through their IPC mappings: a barrier
+    // over the communicator (every rank destroys its handle) before the exchange buffer is freed
+    int* one = nullptr;
+    if (cudaMalloc(&one, sizeof(int)) == cudaSuccess) {
+      if (ncclAllReduce(one, one, 1, ncclInt32, ncclSum, h->comm, h->side) == ncclSuccess)
+        cudaStreamSynchronize(h->side);
+      cudaFree(one);
+    }
+  }
   if (h->comm) ncclCommDestroy(h->comm);
   for (auto& slot : h->state)
     for (float* m : slot) if (m) cudaFree(m);
@@ -216,6 +232,7 @@ void free_ctx(ea_ctx* h) {
   if (h->contrib) cudaFree(h->contrib);
   for (cudaEvent_t ev : h->ev_ag) if (ev) cudaEventDestroy(ev);
   for (cudaEvent_t ev : h->ev_loc) if (ev) cudaEventDestroy(ev);
+  for (cudaEvent_t ev : h->ev_snap) if (ev) cudaEventDestroy(ev);
   if (h->reduced) cudaFree(h->reduced);
   if (h->d_steps) cudaFree(h->d_steps);
   if (h->d_coef) cudaFree(h->d_coef);
@@ -232,6 +249,7 @@ void free_ctx(ea_ctx* h) {
   for (size_t i = 0; i < h->peer_base.size(); ++i)
     if (i < h->peer_ipc.size() && h->peer_ipc[i] && h->peer_base[i]) cudaIpcCloseMemHandle(h->peer_base[i]);
   if (h->xbuf) cudaFree(h->xbuf);
+  if (h->d_xctl) cudaFree(h->d_xctl);
   if (h->err_host) cudaFreeHost(h->err_host);
   if (h->h2d) cudaStreamDestroy(h->h2d);
   if (h->d2h) cudaStreamDestroy(h->d2h);
@@ -267,6 +285,25 @@ ea_status check_stage_ptrs(ea_ctx* h, int32_t stage, float* const* replica_ptrs,
   return EA_OK;
 }
 
+// Staleness 1 (row f4, reading c28): x~_{-1} := x~_0 on the first step of a stage, unless the caller set it
+// (ea_set_state, EA_SLOT_CENTER_PREV).  Refused while `s` is capturing a CUDA graph: the copy would be captured
+// and replayed every step, turning the run into staleness 0.
+ea_status stale_prev_init(ea_ctx* h, int st, const float* center, cudaStream_t s) {
+  if (h->prev_init[st]) return EA_OK;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  cudaError_t e = cudaStreamIsCapturing(s, &cs);
+  if (e != cudaSuccess) return cuda_fail(h, e, "cudaStreamIsCapturing");
+  if (cs != cudaStreamCaptureStatusNone) {
+    set_err(h, "staleness 1: stage %d has no x~_{-1} yet; take its first step outside graph capture or set it with "
+               "ea_set_state(EA_SLOT_CENTER_PREV)", st);
+    return EA_ESTATE;
+  }
+  e = cudaMemcpyAsync(h->prev[st], center, sizeof(float) * h->p[st], cudaMemcpyDeviceToDevice, s);
+  if (e != cudaSuccess) return cuda_fail(h, e, "stale-center init");
+  h->prev_init[st] = 1;
+  return EA_OK;
+}
+
 // Co-located: `count` validated stages in as few launches as possible.
 ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, float* const* replica_ptrs,
                            const float* const* grad_ptrs, float* const* center_ptrs, cudaStream_t s) {
@@ -285,15 +322,12 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // stale center: the lane kernel with x~_{t-1} staged beside x~_t for 2 <= N <= 4 under the default variant, else
   // the replica loop (AVGPIPE_EA_FORCE_WIDE=1 selects the replica loop for A/B measurement)
   const bool stale_lane = stale && n >= 2 && n <= ea::kMaxStaleLaneN && h->variant == 0 && !force_wide;
-  auto stale_prev = [&](int st, const float* center) -> float* {
-    float* prev = h->prev[st];
-    if (!h->prev_init[st]) {  // x~_{-1} := x~_0 (c28)
-      e = cudaMemcpyAsync(prev, center, sizeof(float) * h->p[st], cudaMemcpyDeviceToDevice, s);
-      if (e != cudaSuccess) return nullptr;
-      h->prev_init[st] = 1;
+  if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
+    for (int j = 0; j < count; ++j) {
+      ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);
+      if (st2 != EA_OK) return st2;
     }
-    return prev;
-  };
+  }
   if (stale_lane) {
     for (int j0 = 0; j0 < count; j0 += ea::kMaxLaunchStages) {
       const int cnt = count - j0 < ea::kMaxLaunchStages ? count - j0 : ea::kMaxLaunchStages;
@@ -314,8 +348,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
         r.c = center_ptrs[j];
         r.p = h->p[st];
         r.scp = h->d_coef + st;
-        r.prev = stale_prev(st, center_ptrs[j]);
-        if (!r.prev) return cuda_fail(h, e, "stale-center init");
+        r.prev = h->prev[st];
       }
       e = ea::launch_colocated_batch_stale(b, n, h->hp, opt, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located stale kernel launch");
@@ -334,11 +367,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
       }
       ea_status st2 = advance(h, &stages[j], 1, s);
       if (st2 != EA_OK) return st2;
-      float* prev = nullptr;
-      if (stale) {
-        prev = stale_prev(st, center_ptrs[j]);
-        if (!prev) return cuda_fail(h, e, "stale-center init");
-      }
+      float* prev = stale ? h->prev[st] : nullptr;
       e = ea::launch_colocated_wide(t, n, center_ptrs[j], prev, h->p[st], h->hp, opt, h->d_coef + st, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located kernel launch");
     }
@@ -370,6 +399,29 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   return EA_OK;
 }
 
+// Row a8 knobs (measurement).  The exchange runs on the library's side stream beside the caller's
+// compute, so its own kernels take few SMs: AVGPIPE_EA_SIDE_CTAS (default num_sms/4) caps spread_apply's grid.
+// The local kernels of the spread layout run on the caller's stream with persistent grids that would hold every
+// SM for their whole duration and keep the previous stage's side-stream exchange (NCCL's kernels, or
+// p2p_exchange) from being scheduled at all: AVGPIPE_EA_SPREAD_RESERVE_SMS SMs are left free for it.
+int side_ctas(int num_sms) {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_SIDE_CTAS");
+    return e ? std::atoi(e) : 0;
+  }();
+  if (v > 0) return v;
+  return num_sms / 4 > 0 ? num_sms / 4 : 1;
+}
+
+int spread_local_sms(int num_sms) {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_SPREAD_RESERVE_SMS");
+    return e ? std::atoi(e) : kSpreadReserveSms;
+  }();
+  const int k = num_sms - (v > 0 ? v : 0);
+  return k >= 1 ? k : 1;
+}
+
 // Spread: one stage's exchange on the side stream (rows a6-a8).
 ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s);
 
@@ -384,23 +436,37 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
   const int64_t pad = h->p_pad[stage], shard = pad / n;
   float* own = center_ptr + shard * h->cfg.rank;
   float* contrib = h->contrib + h->contrib_off[stage];
-  // Local phase on the CALLER's stream (x_i, state and r_i ready there, in stream order): it reads the
-  // center, so it waits for this stage's previous all-gather (a no-op wait when that finished long ago).
-  if ((e = cudaStreamWaitEvent(s, h->ev_ag[stage], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  const bool stale = h->cfg.staleness == 1;
+  // Local phase on the CALLER's stream (x_i, state and r_i ready there, in stream order).  Synchronous center:
+  // it reads x~_t, so it waits for this stage's previous all-gather (a no-op wait when that finished long ago).
+  // Staleness 1 (row f4, reading c28): it reads x~_{t-1} from prev, which the previous exchange snapshotted
+  // before its reduce-scatter -- so that whole exchange overlaps this iteration (P:112 asynchronous queues).
+  if (stale) {
+    ea_status st0 = stale_prev_init(h, stage, center_ptr, s);
+    if (st0 != EA_OK) return st0;
+  }
+  if ((e = cudaStreamWaitEvent(s, stale ? h->ev_snap[stage] : h->ev_ag[stage], 0)) != cudaSuccess)
+    return cuda_fail(h, e, "cudaStreamWaitEvent");
   ea_status st2 = advance(h, &stage, 1, s);
   if (st2 != EA_OK) return st2;
-  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0), center_ptr, contrib,
-                              h->p[stage], pad, h->hp, h->cfg.optimizer, h->d_coef + stage, h->num_sms, s);
+  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0),
+                              stale ? h->prev[stage] : center_ptr, contrib, h->p[stage], pad, h->hp,
+                              h->cfg.optimizer, h->d_coef + stage, spread_local_sms(h->num_sms), s);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
   if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   // Exchange on the side stream: reduce-scatter -> owner-shard update -> in-place all-gather.  The caller's
   // stream does not wait for it; the next local step of this stage (or ea_sync) does.
   if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
     return cuda_fail(h, e, "cudaStreamWaitEvent");
+  if (stale) {  // prev <- x~_t (final: the previous all-gather precedes this on the side stream)
+    e = cudaMemcpyAsync(h->prev[stage], center_ptr, sizeof(float) * h->p[stage], cudaMemcpyDeviceToDevice, h->side);
+    if (e != cudaSuccess) return cuda_fail(h, e, "stale-center snapshot");
+    if ((e = cudaEventRecord(h->ev_snap[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  }
   ncclResult_t r = ncclReduceScatter(contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
                                      h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
-  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, h->side);
+  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, side_ctas(h->num_sms), h->side);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
   r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
@@ -458,6 +524,9 @@ ea_status p2p_alloc(ea_ctx* h) {
   cudaError_t e;
   if ((e = cudaMalloc(&h->xbuf, off)) != cudaSuccess) return cuda_fail(h, e, "exchange buffer");
   if ((e = cudaMemset(h->xbuf, 0, off)) != cudaSuccess) return cuda_fail(h, e, "exchange buffer init");
+  const size_t ctl = sizeof(uint32_t) * (2 * (size_t)h->cfg.n_stages + 1);
+  if ((e = cudaMalloc(&h->d_xctl, ctl)) != cudaSuccess || (e = cudaMemset(h->d_xctl, 0, ctl)) != cudaSuccess)
+    return cuda_fail(h, e, "exchange control words");
   if ((e = cudaHostAlloc(&h->err_host, sizeof(uint32_t), cudaHostAllocMapped)) != cudaSuccess)
     return cuda_fail(h, e, "error flag");
   *h->err_host = 0;
@@ -515,7 +584,18 @@ ea_status p2p_ipc_connect(ea_ctx* h) {
   return p2p_open_handles(h, all.data());
 }
 
-// One stage of the fused peer-memory exchange, on the caller's stream.
+// CTAs of p2p_exchange (phases B/C on the side stream).  Its work is NVLink/latency-bound and it runs beside
+// the next forward, so it takes a fraction of the SMs; knob AVGPIPE_EA_P2P_XCTAS (1..4096) for measurement.
+int p2p_exchange_ctas(int num_sms) {
+  const char* e = std::getenv("AVGPIPE_EA_P2P_XCTAS");
+  const long long v = e ? std::atoll(e) : 0;
+  if (v >= 1 && v <= 4096) return static_cast<int>(v);
+  return num_sms / 3 > 0 ? num_sms / 3 : 1;
+}
+
+// One stage of the peer-memory exchange: p2p_push (local update + contributions into the owners' inboxes) on
+// the caller's stream after this stage's previous exchange, p2p_exchange (owner reduction, center update, pull
+// of the other shards) on the side stream, which the caller's stream never waits for (row a8).
 ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, float* center_ptr, cudaStream_t s) {
   if (!h->p2p_ready) {
     set_err(h, "peer-memory exchange not connected (needs an NCCL id at ea_init or ea_p2p_connect)");
@@ -547,19 +627,30 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   a.slots = h->x_slots[stage];
   a.rank = h->cfg.rank;
   a.world = n;
-  ea_status st2 = advance(h, &stage, 1, s);
-  if (st2 != EA_OK) return st2;
-  a.stepp = h->d_steps + stage;
+  a.epochp = h->d_xctl + stage;
+  a.tickets = h->d_xctl + h->cfg.n_stages + stage;
+  a.abort = h->d_xctl + 2 * h->cfg.n_stages;
   a.scp = h->d_coef + stage;
   a.hp = h->hp;
   a.err = h->err_dev;
   a.timeout_ns = p2p_timeout_ns();
   a.sc_fence = p2p_sc_fence();
-  // all ranks' kernels must be resident together: ranks sharing this device share its SMs
-  int max_ctas = h->num_sms * ea::p2p_blocks_per_sm(h->cfg.optimizer) / h->same_device_ranks;
+  cudaError_t e;
+  // the push reads the center: after this stage's previous exchange (a no-op wait when long finished)
+  if ((e = cudaStreamWaitEvent(s, h->ev_ag[stage], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
+  ea_status st2 = advance(h, &stage, 1, s);
+  if (st2 != EA_OK) return st2;
+  // ranks sharing this device (virtual ranks) share its SMs
+  int max_ctas = spread_local_sms(h->num_sms) * ea::p2p_blocks_per_sm(h->cfg.optimizer) / h->same_device_ranks;
   if (max_ctas < 1) max_ctas = 1;
-  cudaError_t e = ea::launch_spread_p2p(a, v, h->cfg.optimizer, max_ctas, s);
-  if (e != cudaSuccess) return cuda_fail(h, e, "peer-memory exchange kernel launch");
+  if ((e = ea::launch_p2p_push(a, v, h->cfg.optimizer, max_ctas, s)) != cudaSuccess)
+    return cuda_fail(h, e, "peer-memory push kernel launch");
+  if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
+    return cuda_fail(h, e, "cudaStreamWaitEvent");
+  if ((e = ea::launch_p2p_exchange(a, v, p2p_exchange_ctas(h->num_sms), h->side)) != cudaSuccess)
+    return cuda_fail(h, e, "peer-memory exchange kernel launch");
+  if ((e = cudaEventRecord(h->ev_ag[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   return EA_OK;
 }
 
@@ -586,6 +677,21 @@ ea_status host_path_resources(ea_ctx* h) {
       (e = cudaEventCreateWithFlags(&h->ev_d2h, cudaEventDisableTiming)) != cudaSuccess)
     return cuda_fail(h, e, "host-path resources");
   return EA_OK;
+}
+
+// Slot EA_SLOT_CENTER_PREV: the stale center x~_{t-1} of a staleness-1 handle (P_s floats, replica 0).
+bool prev_slot(const ea_ctx* h, int32_t replica, int32_t slot) {
+  return slot == EA_SLOT_CENTER_PREV && h->cfg.staleness == 1 && replica == 0;
+}
+
+float* slot_ptr(const ea_ctx* h, int32_t stage, int32_t replica, int32_t slot) {
+  return slot == EA_SLOT_CENTER_PREV ? h->prev[stage] : state_ptr(h, slot, stage, replica);
+}
+
+bool slot_ok(const ea_ctx* h, int32_t stage, int32_t replica, int32_t slot) {
+  if (stage < 0 || stage >= h->cfg.n_stages) return false;
+  if (prev_slot(h, replica, slot)) return true;
+  return replica >= 0 && replica < replicas_here(h) && slot >= 0 && slot < state_slots(h);
 }
 
 }  // namespace
@@ -625,8 +731,8 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
   if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
   if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
   if (c.staleness != 0 && c.staleness != 1) { set_err(nullptr, "staleness must be 0 or 1"); return EA_EINVAL; }
-  if (c.staleness == 1 && c.layout != EA_COLOCATED) {
-    set_err(nullptr, "staleness 1 is supported for EA_COLOCATED");
+  if (c.staleness == 1 && c.layout == EA_SPREAD && c.exchange != EA_XCHG_NCCL) {
+    set_err(nullptr, "staleness 1 in EA_SPREAD needs the NCCL exchange (the peer-memory exchange is one step)");
     return EA_EINVAL;
   }
   if (c.layout == EA_SPREAD && c.exchange == EA_XCHG_P2P && c.world > ea::kMaxWorld) {
@@ -695,7 +801,9 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     }
   }
   if (c.layout == EA_SPREAD) {
-    if ((e = cudaStreamCreateWithFlags(&h->side, cudaStreamNonBlocking)) != cudaSuccess ||
+    int prio_lo = 0, prio_hi = 0;  // the exchange's CTAs go first when SMs free up (it is short and latency-bound)
+    cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
+    if ((e = cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_done, cudaEventDisableTiming)) != cudaSuccess ||
         (c.exchange == EA_XCHG_NCCL && (e = cudaMalloc(&h->contrib, sizeof(float) * sum_pad)) != cudaSuccess) ||
         (e = cudaMalloc(&h->reduced, sizeof(float) * (max_pad / c.n_pipelines))) != cudaSuccess) {
@@ -704,16 +812,19 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
       return r;
     }
     for (int st = 0; st < c.n_stages; ++st) {
-      cudaEvent_t a = nullptr, b = nullptr;
+      cudaEvent_t a = nullptr, b = nullptr, d = nullptr;
       if ((e = cudaEventCreateWithFlags(&a, cudaEventDisableTiming)) != cudaSuccess ||
-          (e = cudaEventCreateWithFlags(&b, cudaEventDisableTiming)) != cudaSuccess) {
+          (e = cudaEventCreateWithFlags(&b, cudaEventDisableTiming)) != cudaSuccess ||
+          (e = cudaEventCreateWithFlags(&d, cudaEventDisableTiming)) != cudaSuccess) {
         if (a) cudaEventDestroy(a);
+        if (b) cudaEventDestroy(b);
         ea_status r = cuda_fail(nullptr, e, "per-stage events");
         free_ctx(h);
         return r;
       }
       h->ev_ag.push_back(a);
       h->ev_loc.push_back(b);
+      h->ev_snap.push_back(d);
     }
     if (nccl_id) {  // NULL: external-collective mode (phase calls only)
       ncclUniqueId uid;
@@ -1025,7 +1136,7 @@ ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const
   }
   cudaError_t e = cudaSetDevice(dev);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaSetDevice");
-  e = ea::launch_spread_apply(center_shard, reduced, h->p_pad[stage] / h->cfg.n_pipelines, h->hp.inv_n, h->num_sms,
+  e = ea::launch_spread_apply(center_shard, reduced, h->p_pad[stage] / h->cfg.n_pipelines, h->hp.inv_n, h->num_sms, 0,
                               static_cast<cudaStream_t>(stream));
   if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
   return EA_OK;
@@ -1033,19 +1144,18 @@ ea_status ea_spread_apply(ea_handle h, int32_t stage, float* center_shard, const
 
 ea_status ea_get_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, float** state_dev) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
-  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || !state_dev ||
-      slot < 0 || slot >= state_slots(h)) {
-    set_err(h, "bad stage/replica/slot or NULL out pointer (this optimizer has %d state slot(s))", state_slots(h));
+  if (!state_dev || !slot_ok(h, stage, replica, slot)) {
+    set_err(h, "bad stage/replica/slot or NULL out pointer (this optimizer has %d state slot(s); "
+               "EA_SLOT_CENTER_PREV needs staleness 1 and replica 0)", state_slots(h));
     return EA_EINVAL;
   }
-  *state_dev = state_ptr(h, slot, stage, replica);
+  *state_dev = slot_ptr(h, stage, replica, slot);
   return EA_OK;
 }
 
 ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot, const float* src, void* stream) {
   if (!h) { set_err(nullptr, "handle is NULL"); return EA_EINVAL; }
-  if (stage < 0 || stage >= h->cfg.n_stages || replica < 0 || replica >= replicas_here(h) || slot < 0 ||
-      slot >= state_slots(h) || !src || !is_device_ptr(src, h->cfg.device)) {
+  if (!slot_ok(h, stage, replica, slot) || !src || !is_device_ptr(src, h->cfg.device)) {
     set_err(h, "bad stage/replica/slot or src is not a device pointer");
     return EA_EINVAL;
   }
@@ -1054,9 +1164,9 @@ ea_status ea_set_state(ea_handle h, int32_t stage, int32_t replica, int32_t slot
   cudaStream_t s = static_cast<cudaStream_t>(stream);
   ea_status st = join_side(h, s);  // order after pending side-stream work on this state
   if (st != EA_OK) return st;
-  e = cudaMemcpyAsync(state_ptr(h, slot, stage, replica), src, sizeof(float) * h->p[stage], cudaMemcpyDeviceToDevice,
-                      s);
+  e = cudaMemcpyAsync(slot_ptr(h, stage, replica, slot), src, sizeof(float) * h->p[stage], cudaMemcpyDeviceToDevice, s);
   if (e != cudaSuccess) return cuda_fail(h, e, "cudaMemcpyAsync");
+  if (slot == EA_SLOT_CENTER_PREV) h->prev_init[stage] = 1;
   return EA_OK;
 }
 

@@ -55,9 +55,10 @@ struct StageList {
   int count;
 };
 
-// On `s`: for every listed stage, ++steps[stage] and recompute coef[stage] (double precision).
-cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, const CoefParams& cp,
-                                 cudaStream_t s);
+// On `s`: for every listed stage, ++steps[stage], ++xepoch[stage] (if xepoch is not null: the peer-memory
+// exchange's epoch) and recompute coef[stage] (double precision).
+cudaError_t launch_advance_steps(int64_t* steps, uint32_t* xepoch, StepCoef* coef, const StageList& list,
+                                 const CoefParams& cp, cudaStream_t s);
 
 constexpr int kMaxReplicas = 64;      // EA_MAX_REPLICAS
 constexpr int kMaxFusedN = 8;         // replicas handled by the compile-time-N kernels
@@ -144,19 +145,25 @@ struct P2PArgs {
   int64_t chunk;       // floats per chunk (multiple of 4)
   int64_t nchunks, slots;
   int rank, world;
-  const int64_t* stepp;  // device: this stage's step count (>= 1), the exchange epoch
+  const uint32_t* epochp;  // device: this stage's exchange epoch (>= 1; advanced on the stream, never by ea_set_step)
+  uint32_t* tickets;   // device: this stage's work-item ticket of p2p_exchange (zeroed before each launch)
+  uint32_t* abort;     // device: set by the first timed-out wait; later waits fail at once
   Hyper hp;
-  const StepCoef* scp;   // device: Adam coefficients
+  const StepCoef* scp;   // device: the step's optimizer coefficients
   uint32_t* err;       // host-mapped error flag (timeouts)
   uint64_t timeout_ns;
   int sc_fence;        // 1: fence.sc.sys before each release (knob AVGPIPE_EA_P2P_FENCE=1; default 0)
 };
 
-cudaError_t launch_spread_p2p(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);
+// Phase A (local update, contributions pushed into the owners' inboxes): never waits.
+cudaError_t launch_p2p_push(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);
+// Phases B (owner reduction + center update) and C (pull the other owners' chunks), ticket-ordered.
+cudaError_t launch_p2p_exchange(const P2PArgs& a, const P2PView& v, int max_ctas, cudaStream_t s);
 int p2p_blocks_per_sm(int opt);
 
-// Spread shard epilogue (row a5): shard[k] += reduced[k] * inv_n for k < count.
+// Spread shard epilogue (row a5): shard[k] += reduced[k] * inv_n for k < count.  max_ctas > 0 caps the grid
+// (the library's side stream runs it beside the caller's compute).
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,
-                                cudaStream_t s);
+                                int max_ctas, cudaStream_t s);
 
 }  // namespace ea

@@ -21,6 +21,7 @@
 #include <cstdlib>
 
 #include "ea_internal.h"
+#include "ea_update.cuh"
 
 namespace ea {
 namespace {
@@ -71,70 +72,6 @@ struct Mem {
                    : "memory");
   }
 };
-
-// ---------------------------------------------------------------- the math
-// One (replica, element) update; returns the replica's contribution r_i.
-// m: SGD momentum / Adam first moment / ASGD average; v: Adam second moment (SGD, ASGD: untouched).
-template <int OPT>
-__device__ __forceinline__ float ea_elem(float& x, float g, float& m, float& v, float c, const Hyper& hp,
-                                         const StepCoef& sc) {
-  float delta;
-  if constexpr (OPT == kOptSGD) {
-    const float gg = fmaf(hp.wd, x, g);             // g + lambda*x
-    const float mn = fmaf(hp.momentum, m, gg);      // mu*m + g'
-    const float d = hp.nesterov ? fmaf(hp.momentum, mn, gg) : mn;
-    delta = -hp.lr * d;                             // local update Delta_i (Step 1)
-    m = mn;
-  } else if constexpr (OPT == kOptASGD) {
-    // torch.optim.ASGD (reading c29): x_local = x (1 - l eta_t) - eta_t g', so Delta = -eta_t (g' + l x);
-    // the average tracks the optimizer's own iterate x + Delta (mu_t == 1: a copy, as torch does)
-    const float gg = fmaf(hp.wd, x, g);
-    delta = -sc.step_size * fmaf(hp.asgd_lambd, x, gg);
-    const float xl = x + delta;
-    m = sc.inv_sqrt_bc2 == 1.f ? xl : fmaf(sc.inv_sqrt_bc2, xl - m, m);
-  } else {
-    const float gg = OPT == kOptAdam ? fmaf(hp.wd, x, g) : g;
-    const float mn = fmaf(hp.beta1, m, hp.one_minus_beta1 * gg);
-    const float vn = fmaf(hp.beta2, v, hp.one_minus_beta2 * (gg * gg));
-    const float denom = fmaf(sqrtf(vn), sc.inv_sqrt_bc2, hp.eps);
-    delta = -sc.step_size * (mn / denom);
-    if constexpr (OPT == kOptAdamW) delta = fmaf(-hp.lr_wd, x, delta);
-    m = mn;
-    v = vn;
-  }
-  const float gap = x - c;                          // x_i - x~ (pre-step values, c1/c2)
-  const float r = fmaf(hp.beta, gap, hp.rho * delta);
-  x = fmaf(-hp.alpha, gap, x) + delta;              // (1-a)x + a*x~ + Delta (Step 2)
-  return r;
-}
-
-template <int OPT>
-__device__ __forceinline__ float4 ea_vec(float4& x, float4 g, float4& m, float4& v, float4 c, const Hyper& hp,
-                                         const StepCoef& sc) {
-  float4 r;
-  r.x = ea_elem<OPT>(x.x, g.x, m.x, v.x, c.x, hp, sc);
-  r.y = ea_elem<OPT>(x.y, g.y, m.y, v.y, c.y, hp, sc);
-  r.z = ea_elem<OPT>(x.z, g.z, m.z, v.z, c.z, hp, sc);
-  r.w = ea_elem<OPT>(x.w, g.w, m.w, v.w, c.w, hp, sc);
-  return r;
-}
-
-__device__ __forceinline__ void add4(float4& a, float4 b) {
-  a.x += b.x; a.y += b.y; a.z += b.z; a.w += b.w;
-}
-__device__ __forceinline__ float4 center_apply(float4 c, float4 acc, float inv_n) {
-  return make_float4(fmaf(acc.x, inv_n, c.x), fmaf(acc.y, inv_n, c.y), fmaf(acc.z, inv_n, c.z),
-                     fmaf(acc.w, inv_n, c.w));
-}
-
-template <int OPT>
-__device__ __forceinline__ StepCoef load_coef(const StepCoef* scp) {
-  if constexpr (OPT == kOptSGD) {
-    return StepCoef{0.f, 0.f};
-  } else {
-    return *scp;
-  }
-}
 
 // Scalar tail of one stage: elements [4*(p/4), p) (fewer than 4), one thread.
 // STALE: the replicas see st.prev[j] (x~_{t-1}) and st.prev[j] becomes x~_t (row f4).
@@ -1048,11 +985,13 @@ cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v
 // Step counter + the step's coefficients, on the stream (graph-capturable): Adam(W) bias corrections, or
 // ASGD's eta_t and mu_t (torch.optim.ASGD's state after t-1 steps: eta = lr / (1 + l lr (t-1))^a,
 // mu = 1 / max(1, t-1-t0); eta_1 = lr, mu_1 = 1).
-__global__ void advance_steps(int64_t* steps, StepCoef* coef, const StageList list, const CoefParams cp) {
+__global__ void advance_steps(int64_t* steps, uint32_t* xepoch, StepCoef* coef, const StageList list,
+                              const CoefParams cp) {
   const int i = threadIdx.x;
   if (i >= list.count) return;
   const int s = list.idx[i];
   const int64_t t = ++steps[s];
+  if (xepoch) ++xepoch[s];
   if (cp.opt == kOptASGD) {
     const double k = (double)(t - 1);
     coef[s].step_size = static_cast<float>(cp.lr / pow(1.0 + cp.lambd * cp.lr * k, cp.asgd_alpha));
@@ -1067,10 +1006,10 @@ __global__ void advance_steps(int64_t* steps, StepCoef* coef, const StageList li
 
 }  // namespace
 
-cudaError_t launch_advance_steps(int64_t* steps, StepCoef* coef, const StageList& list, const CoefParams& cp,
-                                 cudaStream_t s) {
+cudaError_t launch_advance_steps(int64_t* steps, uint32_t* xepoch, StepCoef* coef, const StageList& list,
+                                 const CoefParams& cp, cudaStream_t s) {
   if (list.count <= 0) return cudaSuccess;
-  advance_steps<<<1, 32, 0, s>>>(steps, coef, list, cp);
+  advance_steps<<<1, 32, 0, s>>>(steps, xepoch, coef, list, cp);
   return cudaGetLastError();
 }
 
@@ -1146,11 +1085,12 @@ cudaError_t launch_spread_local(float* x, const float* g, float* m, float* v, co
 }
 
 cudaError_t launch_spread_apply(float* shard, const float* reduced, int64_t count, float inv_n, int num_sms,
-                                cudaStream_t s) {
+                                int max_ctas, cudaStream_t s) {
   if (count <= 0) return cudaSuccess;
   const int64_t nvec = count / 4;
   const int64_t units = (nvec + kThreads - 1) / kThreads;
-  const int grid = persistent_grid(spread_apply, units < 1 ? 1 : units, num_sms);
+  int grid = persistent_grid(spread_apply, units < 1 ? 1 : units, num_sms);
+  if (max_ctas > 0 && grid > max_ctas) grid = max_ctas;  // side stream: a small SM footprint beside the compute
   spread_apply<<<grid, kThreads, 0, s>>>(shard, reduced, nvec, count, inv_n);
   return cudaGetLastError();
 }

@@ -82,6 +82,7 @@ class CollectiveSpread:
         self.group = group
         self.rank = dist.get_rank(group)
         self.world = dist.get_world_size(group)
+        self.handle = handle
         self.local_fn = local_fn or handle.spread_local
         self.apply_fn = apply_fn or handle.spread_apply
         self._scratch = {}
@@ -96,7 +97,10 @@ class CollectiveSpread:
 
     def step(self, stage: int, replica, grad, center):
         import torch.distributed as dist
-        p_pad = center.numel()
+        # the library writes P_pad = ea_center_capacity floats of contribution: size everything from it
+        p_pad = self.handle.center_capacity(stage) if self.handle is not None else center.numel()
+        if center.numel() != p_pad:
+            raise ValueError(f"stage {stage}: center has {center.numel()} elements, the library expects {p_pad}")
         lo, hi = shard_bounds(p_pad, self.world, self.rank)
         contrib = self._buf(("c", stage), p_pad, center)
         self.local_fn(stage, replica, grad, center, contrib)

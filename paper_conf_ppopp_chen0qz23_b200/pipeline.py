@@ -5,44 +5,68 @@ iteration each of the N parallel pipelines pushes its batch of M
 micro-batches through the stages in the order Algorithm 1 prescribes for
 this stage (``ea_schedule`` -- `advance` forwards first, then forward/backward
 pairs, then the cool-down), exchanging activations forward and
-activation-gradients backward with the neighbouring stages (point-to-point,
-tagged by pipeline and micro-batch).  After the last backward of the
-iteration the stage's N replicas are coupled by ONE elastic-averaging step
-(``ElasticAveraging.step``, co-located layout: this GPU holds stage k of all
-N pipelines plus the reference model), and the run-time controller of
-Algorithm 1 (lines 9-10, ``ea_advance_*``) decides whether the next
-iteration forwards one more micro-batch in advance.
+activation-gradients backward with the neighbouring stages (point-to-point).
+After the last backward of the iteration the stage's N replicas are coupled
+by ONE elastic-averaging step (``ElasticAveraging.step``, co-located layout:
+this GPU holds stage k of all N pipelines plus the reference model),
+and the run-time controller of Algorithm 1 (lines 9-10, ``ea_advance_*``)
+decides whether the next iteration forwards one more micro-batch in advance.
 
-The compute of a stage is the caller's ``torch.nn.Module`` (autograd); the
-runtime owns the order, the transfers, the activation stash and the
-averaging.  Pipelines run one after another within an iteration (the simple
-policy; the paper overlaps them with one process per pipeline per GPU).
+Concurrency (P:110 "a parallel pipeline launches a process on each GPU"):
+with ``concurrent=True`` the N pipelines of a stage run at the same time, one
+host thread and one CUDA stream per pipeline, each pipeline's transfers on its
+own process group (``make_pipeline_groups``) -- so NCCL's in-order matching of
+point-to-point operations holds per pipeline, and the pipelines' activation
+transfers and compute interleave freely.  The elastic-averaging step goes on
+its own stream (``ea_stream``): it waits only for every pipeline's last
+backward (CUDA events), the host does not wait for it, and the next
+iteration's forward of pipeline i waits for it on the GPU (it reads x_i) --
+P:112 "in an asynchronous manner ... to prevent the inter-process
+communication blocking the pipeline".
+
+Transfers: with the ``nccl`` backend activations stay on the GPU
+(torch.distributed isend/recv of device tensors over NVLink); with ``gloo``
+they are staged through host memory.  The compute of a stage is the caller's
+``torch.nn.Module`` (autograd); the runtime owns the order, the transfers, the
+activation stash and the averaging.
 """
 from __future__ import annotations
 
+import threading
 import time
 from typing import Callable, List, Optional, Sequence
 
 from .binding import AdvanceController, schedule
 
 
+def make_pipeline_groups(n_pipelines: int, ranks: Optional[Sequence[int]] = None, backend: Optional[str] = None):
+    """One process group per parallel pipeline over the K stage ranks (a collective call: every stage rank
+    creates the N groups in the same order).  Pipeline i's activations and gradients travel only on group i."""
+    import torch.distributed as dist
+    ranks = list(range(dist.get_world_size())) if ranks is None else list(ranks)
+    return [dist.new_group(ranks, backend=backend) for _ in range(n_pipelines)]
+
+
 class PipelineStage:
     """Stage `stage` (0-based) of K; `replicas` = this stage's module of each of
     the N pipelines (structurally identical).  `ea` (optional) is an
     ElasticAveraging handle whose stage `ea_stage` holds these parameters,
-    flattened in `flat_params[i]` / `flat_grads[i]` (views the modules use)."""
+    flattened in `flat_params[i]` / `flat_grads[i]` (views the modules use).
+    `concurrent`: run the N pipelines at once (threads + streams; `groups` =
+    per-pipeline process groups, default `make_pipeline_groups(N)`)."""
 
     def __init__(self, replicas: Sequence, stage: int, K: int, M: int, group=None, *, ea=None, ea_stage: int = 0,
                  center=None, flat_params=None, flat_grads=None, mem_limit: Optional[float] = None,
-                 mem_per_microbatch: float = 0.0, extra_advance: int = 0, dynamic: bool = False):
+                 mem_per_microbatch: float = 0.0, extra_advance: int = 0, dynamic: bool = False,
+                 concurrent: bool = False, groups=None):
         import torch.distributed as dist
         self.replicas = list(replicas)
         self.N = len(self.replicas)
         self.stage, self.K, self.M = stage, K, M
         self.group = group
         self.rank = dist.get_rank(group)
-        self.prev = self.rank - 1 if stage > 0 else None
-        self.next = self.rank + 1 if stage < K - 1 else None
+        self.prev = stage - 1 if stage > 0 else None      # neighbour stage indices = ranks of `group`
+        self.next = stage + 1 if stage < K - 1 else None
         self.ea, self.ea_stage, self.center = ea, ea_stage, center
         self.flat_params, self.flat_grads = flat_params, flat_grads
         self.ctl = AdvanceController(K, M)
@@ -51,77 +75,153 @@ class PipelineStage:
         self.dynamic = dynamic
         self.mem_limit = mem_limit
         self.mem_per_microbatch = mem_per_microbatch
+        self.concurrent = concurrent
+        if concurrent and groups is None:
+            groups = make_pipeline_groups(self.N)
+        self.groups = list(groups) if groups is not None else [group] * self.N
         self.peak_stash = 0
         self.history: List[dict] = []
+        self._streams = None      # per-pipeline CUDA streams (concurrent, on a GPU)
+        self._ea_stream = None
+        self._ea_done = None      # event: the last EA step (the next forward of every pipeline waits for it)
 
     # ------------------------------------------------------------------ transfers
+    def _peer(self, stage_index, group):
+        import torch.distributed as dist
+        return dist.get_global_rank(group, stage_index) if group is not None else stage_index
+
     def _tag(self, pipeline: int, j: int, backward: bool) -> int:
         return ((pipeline * self.M + j) << 1) | int(backward)
 
-    def _send(self, t, dst, tag):
+    def _send(self, t, dst_stage, tag, group):
         import torch.distributed as dist
         t = t.detach().contiguous()
         if self.backend == "gloo" and t.is_cuda:      # gloo moves host tensors
             t = t.cpu()
-        return dist.isend(t, dst=dst, group=self.group, tag=tag)
+        return dist.isend(t, dst=self._peer(dst_stage, group), group=group, tag=tag)
 
-    def _recv(self, like_shape, dtype, device, src, tag):
+    def _recv(self, like_shape, dtype, device, src_stage, tag, group):
         import torch
         import torch.distributed as dist
         host = self.backend == "gloo"
         buf = torch.empty(like_shape, dtype=dtype, device="cpu" if host else device)
-        dist.recv(buf, src=src, group=self.group, tag=tag)
+        dist.recv(buf, src=self._peer(src_stage, group), group=group, tag=tag)
         return buf.to(device) if host else buf
+
+    # ------------------------------------------------------------------ one pipeline's share of an iteration
+    def _run_pipeline(self, i, ops, inputs, targets, loss_fn, act_shape, act_dtype, device):
+        """Pipeline i's ops on this stage, in Algorithm 1's order.  Returns (loss, pending sends, peak stash)."""
+        mod = self.replicas[i]
+        group = self.groups[i]
+        stash, pending, loss_sum, peak = {}, [], 0.0, 0
+        for kind, j in ops:
+            if kind == "F":
+                if self.prev is None:
+                    x = inputs[i][j]
+                else:
+                    x = self._recv(act_shape, act_dtype, device, self.prev, self._tag(i, j, False), group)
+                    x.requires_grad_(True)
+                y = mod(x)
+                if self.next is None:
+                    loss = loss_fn(y, targets[i][j]) / self.M
+                    loss_sum += float(loss.detach())
+                    stash[j] = (x, loss)
+                else:
+                    pending.append(self._send(y, self.next, self._tag(i, j, False), group))
+                    stash[j] = (x, y)
+                peak = max(peak, len(stash))
+            else:
+                x, y = stash.pop(j)
+                if self.next is None:
+                    y.backward()
+                else:
+                    gy = self._recv(y.shape, y.dtype, device, self.next, self._tag(i, j, True), group)
+                    y.backward(gy)
+                if self.prev is not None:
+                    pending.append(self._send(x.grad, self.prev, self._tag(i, j, True), group))
+        return loss_sum, pending, peak
+
+    def _cuda(self, device):
+        import torch
+        return torch.cuda.is_available() and str(device).startswith("cuda")
 
     # ------------------------------------------------------------------ one iteration
     def run_iteration(self, inputs=None, targets=None, loss_fn: Optional[Callable] = None, act_shape=None,
-                      act_dtype=None, device="cpu"):
+                      act_dtype=None, device="cpu", zero_grads: bool = False, sync: bool = True):
         """inputs[i][j] (stage 0) / targets[i][j] (last stage): micro-batch j of
         pipeline i.  act_shape: shape of the activation this stage receives
-        (stage > 0) -- and, for the backward, the shape it sends.  Returns the
-        per-pipeline summed loss on the last stage (else None)."""
+        (stage > 0) -- and, for the backward, the shape it sends.  zero_grads:
+        zero flat_grads[i] on pipeline i's stream first (ordered after the last
+        EA step, which reads them).  sync=False returns once the pipelines'
+        streams are done and leaves the EA step running on its stream (the next
+        iteration's forwards wait for it on the GPU).  Returns the per-pipeline
+        summed loss on the last stage (else None)."""
         import torch
         advance = self.ctl.advance_for_stage(self.stage)
         ops = schedule(self.K, self.M, self.stage, advance)
         t0 = time.perf_counter()
-        losses = [0.0] * self.N
-        pending = []
-        peak = 0
-        for i, mod in enumerate(self.replicas):
-            stash = {}
-            for kind, j in ops:
-                if kind == "F":
-                    if self.prev is None:
-                        x = inputs[i][j]
+        cuda = self._cuda(device)
+        results = [None] * self.N
+        if self.concurrent:
+            if cuda and self._streams is None:
+                self._streams = [torch.cuda.Stream(device=device) for _ in range(self.N)]
+            errors = []
+
+            def work(i):
+                try:
+                    if cuda:
+                        s = self._streams[i]
+                        if self._ea_done is not None:
+                            s.wait_event(self._ea_done)        # x_i was updated by the last EA step
+                        with torch.cuda.stream(s):
+                            if zero_grads and self.flat_grads is not None:
+                                self.flat_grads[i].zero_()
+                            results[i] = self._run_pipeline(i, ops, inputs, targets, loss_fn, act_shape,
+                                                            act_dtype, device)
                     else:
-                        x = self._recv(act_shape, act_dtype, device, self.prev, self._tag(i, j, False))
-                        x.requires_grad_(True)
-                    y = mod(x)
-                    if self.next is None:
-                        loss = loss_fn(y, targets[i][j]) / self.M
-                        losses[i] += float(loss.detach())
-                        stash[j] = (x, loss)
-                    else:
-                        pending.append(self._send(y, self.next, self._tag(i, j, False)))
-                        stash[j] = (x, y)
-                    peak = max(peak, len(stash))
-                else:
-                    x, y = stash.pop(j)
-                    if self.next is None:
-                        y.backward()
-                    else:
-                        gy = self._recv(y.shape, y.dtype, device, self.next, self._tag(i, j, True))
-                        y.backward(gy)
-                    if self.prev is not None:
-                        pending.append(self._send(x.grad, self.prev, self._tag(i, j, True)))
+                        results[i] = self._run_pipeline(i, ops, inputs, targets, loss_fn, act_shape, act_dtype,
+                                                        device)
+                except BaseException as e:  # pragma: no cover
+                    errors.append(e)
+
+            threads = [threading.Thread(target=work, args=(i,)) for i in range(self.N)]
+            for t in threads:
+                t.start()
+            for t in threads:
+                t.join()
+            if errors:
+                raise errors[0]
+        else:
+            for i in range(self.N):
+                if cuda and self._ea_done is not None:
+                    torch.cuda.current_stream(device).wait_event(self._ea_done)
+                if zero_grads and self.flat_grads is not None:
+                    self.flat_grads[i].zero_()
+                results[i] = self._run_pipeline(i, ops, inputs, targets, loss_fn, act_shape, act_dtype, device)
+        pending = [w for r in results for w in r[1]]
+        peak = max(r[2] for r in results)
         if self.ea is not None:
-            # this stage's last backward is done: the averaging step goes onto the stream now, so it overlaps
-            # the activation-gradient sends still in flight (they never read the parameters; P:112 "not block")
-            self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center)
+            # every pipeline's last backward of this stage is done: the averaging step goes onto its own stream
+            # behind them (events), and the host moves on -- it overlaps the activation-gradient sends still in
+            # flight (they never read the parameters) and whatever else is queued (P:112 "not block")
+            if cuda:
+                if self._ea_stream is None:
+                    self._ea_stream = torch.cuda.Stream(device=device)
+                    self._ea_done = torch.cuda.Event()
+                streams = self._streams if self.concurrent else [torch.cuda.current_stream(device)]
+                for s in streams:
+                    self._ea_stream.wait_stream(s)
+                self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center, stream=self._ea_stream)
+                self._ea_done.record(self._ea_stream)
+            else:
+                self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center)
         for w in pending:
             w.wait()
-        if torch.cuda.is_available() and str(device).startswith("cuda"):
-            torch.cuda.synchronize()
+        if cuda and sync:
+            torch.cuda.synchronize(device)
+        elif cuda:
+            for s in (self._streams if self.concurrent else [torch.cuda.current_stream(device)]):
+                s.synchronize()
         dt = time.perf_counter() - t0
         self.peak_stash = peak
         rec = {"advance": advance, "peak_stash": peak, "time": dt}
@@ -131,7 +231,7 @@ class PipelineStage:
             self._agree_on_advance()
             rec["next_advance"] = self.ctl.advance_num
         self.history.append(rec)
-        return losses if self.next is None else None
+        return [r[0] for r in results] if self.next is None else None
 
     def _agree_on_advance(self):
         """Algorithm 1 runs its adjustment on the first GPU; the other
@@ -140,6 +240,8 @@ class PipelineStage:
         import torch
         import torch.distributed as dist
         t = torch.tensor([self.ctl.advance_num], dtype=torch.int64)
+        if self.backend == "nccl":
+            t = t.cuda()
         src = dist.get_global_rank(self.group, 0) if self.group is not None else 0
         dist.broadcast(t, src=src, group=self.group)
         self.ctl.ctl.advance_num = int(t.item())

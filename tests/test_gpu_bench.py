@@ -16,9 +16,10 @@ KEYS = {"metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "
         "vs_baseline", "dtype", "data", "config", "roofline", "gpu_launches", "clocks", "e2e"}
 
 
-def _bench(*args):
+def _bench(*args, cpu=False):
+    extra = ["--cpu-seconds", "1"] if cpu else ["--no-cpu-baseline"]
     r = subprocess.run([sys.executable, "bench.py", "--steps", "5", "--warmup", "3", "--e2e-steps", "2",
-                        "--no-cpu-baseline", *args], cwd=ROOT, capture_output=True, text=True, timeout=600)
+                        *extra, *args], cwd=ROOT, capture_output=True, text=True, timeout=600)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.strip()]
     assert len(lines) == 1, r.stdout
@@ -36,13 +37,18 @@ def test_bench_default_line():
     assert d["e2e"]["h2d_bytes_per_step"] == 4 * 4 * 25_000_000 and d["e2e"]["value"] > 0
 
 
-@pytest.mark.parametrize("opt", ["adam", "sgd"])
-def test_bench_spread_world1_line(opt):
-    d = _bench("--layout", "spread", "--config", "C1", "--optimizer", opt)
+@pytest.mark.parametrize("opt,exchange", [("adam", "nccl"), ("sgd", "nccl"), ("sgd", "p2p")])
+def test_bench_spread_world1_line(opt, exchange):
+    d = _bench("--layout", "spread", "--config", "C1", "--optimizer", opt, "--exchange", exchange, cpu=True)
     assert d["config"]["layout"] == "spread" and d["n_gpus"] == 1
     r = d["roofline"]     # world 1: the local kernel's HBM roofline
-    assert r["bound"] == "hbm" and r["kernel"].startswith("spread_bulkpipe") and r["frac"] > 0
+    kern = "spread_bulkpipe" if exchange == "nccl" else "p2p_push"
+    assert r["bound"] == "hbm" and r["kernel"].startswith(kern) and r["frac"] > 0 and "traffic" in r
+    assert r["peak_source"]
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 4 * 2_000_000
+    assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
+    if exchange == "nccl":
+        assert isinstance(d["config"]["nccl"], list)      # NCCL_DEBUG=INFO summary of the library's communicator
 
 
 def test_bench_world2_line_on_one_gpu():
@@ -57,7 +63,7 @@ def test_bench_world2_line_on_one_gpu():
     env = dict(os.environ, AVGPIPE_BENCH_SHARED_GPU="1", AVGPIPE_EA_P2P_TIMEOUT_MS="120000")
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", port, "bench.py", "--gpus", "2", "--exchange", "p2p",
-           "--config", "C1", "--steps", "3", "--warmup", "3", "--e2e-steps", "2"]
+           "--config", "C1", "--steps", "3", "--warmup", "3", "--e2e-steps", "2", "--cpu-seconds", "1"]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=900, env=env)
     assert r.returncode == 0, r.stderr[-3000:]
     lines = [l for l in r.stdout.splitlines() if l.strip().startswith("{")]
@@ -65,4 +71,10 @@ def test_bench_world2_line_on_one_gpu():
     d = json.loads(lines[0])
     assert KEYS <= set(d), KEYS - set(d)
     assert d["n_gpus"] == 2 and d["config"]["layout"] == "spread" and d["config"]["exchange"] == "p2p"
-    assert d["roofline"]["bound"] == "nvlink" and d["value"] > 0 and d["e2e"]["value"] > 0
+    r = d["roofline"]
+    assert r["bound"] == "nvlink" and d["value"] > 0 and d["e2e"]["value"] > 0
+    assert "B200_PROFILING" in r["peak_source"] and "traffic" in r
+    loc = d["local_kernel_roofline"]          # the push kernel on each rank's caller stream
+    assert loc["bound"] == "hbm" and loc["kernel"] == "p2p_push" and "traffic" in loc and loc["frac"] > 0
+    cb = d["cpu_baseline"]                    # rank 0 times one stage-shard of the oracle, extrapolated
+    assert cb["kind"] == "oracle" and cb["cores"] >= 1 and "extrapolated" in cb

@@ -457,9 +457,13 @@ def test_bad_pointers_rejected_before_enqueue():
     x = [torch.zeros(p + 4, device="cuda:0") for _ in range(n)]
     c = torch.zeros(p, device="cuda:0")
     with pytest.raises(EAError, match="EA_EINVAL"):
-        h.step(0, [t[1:] for t in x], [t[:p] for t in x], c)          # 4-byte offset -> misaligned
+        h.step(0, [t[1:p + 1] for t in x], [t[:p] for t in x], c)     # 4-byte offset -> misaligned
     with pytest.raises(EAError, match="EA_EINVAL"):
         h.step(1, [t[:p] for t in x], [t[:p] for t in x], c)          # stage out of range
+    with pytest.raises(ValueError, match="elements"):
+        h.step(0, [t[:p - 4] for t in x], [t[:p] for t in x], c)      # undersized replica: never reaches the ABI
+    with pytest.raises(ValueError, match="elements"):
+        h.step(0, [t[:p] for t in x], [t[:p] for t in x], c[:p - 4])  # undersized center
     host = torch.zeros(p).pin_memory()
     import ctypes
     from paper_conf_ppopp_chen0qz23_b200 import binding

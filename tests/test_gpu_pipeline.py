@@ -48,27 +48,35 @@ def _flatten(mod, device):
     return flat, gflat
 
 
-def _worker(rank, port, q):
+def _worker(rank, port, q, concurrent=False, backend="gloo"):
     try:
-        dist.init_process_group("gloo", init_method=port, rank=rank, world_size=K)
+        dev = torch.device("cuda", rank if backend == "nccl" else 0)
+        torch.cuda.set_device(dev)
+        if backend == "nccl":
+            dist.init_process_group("nccl", init_method=port, rank=rank, world_size=K, device_id=dev)
+        else:
+            dist.init_process_group("gloo", init_method=port, rank=rank, world_size=K)
         from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
         from paper_conf_ppopp_chen0qz23_b200.pipeline import PipelineStage
-        dev = torch.device("cuda:0")
         mods = [_model(100 + i)[rank].to(dev) for i in range(N)]
         flats = [_flatten(m, dev) for m in mods]
         P = flats[0][0].numel()
         center = flats[0][0].clone()
-        ea = ElasticAveraging([P], N, beta=1.0, rho=1.0, lr=LR, momentum=MU)     # alpha = 1/N
+        ea = ElasticAveraging([P], N, beta=1.0, rho=1.0, lr=LR, momentum=MU, device=dev.index)   # alpha = 1/N
         st = PipelineStage(mods, rank, K, M, ea=ea, ea_stage=0, center=center,
-                           flat_params=[f for f, _ in flats], flat_grads=[g for _, g in flats], extra_advance=1)
+                           flat_params=[f for f, _ in flats], flat_grads=[g for _, g in flats], extra_advance=1,
+                           concurrent=concurrent)
         for it in range(ITERS):
             xs, ys = _data(it)
-            for _, g in flats:
-                g.zero_()
+            if not concurrent:
+                for _, g in flats:
+                    g.zero_()
+            # concurrent: grads zeroed on each pipeline's stream after the previous EA step, and the EA step
+            # of this iteration left running on its stream (sync=False): the next forwards wait for it on the GPU
             st.run_iteration(inputs=[[x.to(dev) for x in r] for r in xs] if rank == 0 else None,
                              targets=[[y.to(dev) for y in r] for r in ys] if rank == K - 1 else None,
                              loss_fn=torch.nn.functional.mse_loss, act_shape=(B, D), act_dtype=torch.float32,
-                             device=dev)
+                             device=dev, zero_grads=concurrent, sync=not concurrent)
         torch.cuda.synchronize()
         q.put((rank, "ok", [f.cpu().numpy() for f, _ in flats], center.cpu().numpy()))
         ea.close()
@@ -112,12 +120,17 @@ def _reference():
     return [[flat(models[i], k) for i in range(N)] for k in range(K)], centers
 
 
-def test_pipeline_with_elastic_averaging_matches_reference():
+@pytest.mark.parametrize("concurrent,backend", [(False, "gloo"), (True, "gloo"), (True, "nccl")])
+def test_pipeline_with_elastic_averaging_matches_reference(concurrent, backend):
+    """concurrent: the N pipelines at once (thread + stream + process group each), the EA step on its own
+    stream.  nccl: activations as device tensors over NCCL, one GPU per stage (needs K GPUs)."""
     import tempfile
+    if backend == "nccl" and torch.cuda.device_count() < K:
+        pytest.skip(f"NCCL activations need {K} GPUs (NCCL refuses two ranks on one device)")
     port = "file://" + os.path.join(tempfile.mkdtemp(prefix="gloo_"), "store")   # no TCP port race
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, port, q)) for r in range(K)]
+    procs = [ctx.Process(target=_worker, args=(r, port, q, concurrent, backend)) for r in range(K)]
     for p in procs:
         p.start()
     out = {}

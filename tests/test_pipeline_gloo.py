@@ -29,7 +29,7 @@ def _data(N, M, seed=0):
     return xs, ys
 
 
-def _worker(rank, K, N, M, extra, dynamic, port, q):
+def _worker(rank, K, N, M, extra, dynamic, port, q, concurrent=False):
     try:
         dist.init_process_group("gloo", init_method=port, rank=rank, world_size=K)
         from paper_conf_ppopp_chen0qz23_b200.pipeline import PipelineStage
@@ -37,7 +37,7 @@ def _worker(rank, K, N, M, extra, dynamic, port, q):
         stage_mods = [m[rank] for m in models]
         xs, ys = _data(N, M)
         st = PipelineStage(stage_mods, rank, K, M, extra_advance=extra, dynamic=dynamic, mem_limit=1e9,
-                           mem_per_microbatch=1.0)
+                           mem_per_microbatch=1.0, concurrent=concurrent)
         loss_fn = torch.nn.functional.mse_loss
         iters = 3 if dynamic else 1
         for _ in range(iters):
@@ -63,11 +63,11 @@ def _file_store():
     return "file://" + os.path.join(d, "store")
 
 
-def _run(K, N, M, extra, dynamic=False):
+def _run(K, N, M, extra, dynamic=False, concurrent=False):
     port = _file_store()
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, K, N, M, extra, dynamic, port, q)) for r in range(K)]
+    procs = [ctx.Process(target=_worker, args=(r, K, N, M, extra, dynamic, port, q, concurrent)) for r in range(K)]
     for p in procs:
         p.start()
     out = {}
@@ -94,10 +94,11 @@ def _reference_grads(N, M):
     return ref
 
 
-@pytest.mark.parametrize("extra", [0, 1, 8])
-def test_pipeline_gradients_match_reference(extra):
+@pytest.mark.parametrize("extra,concurrent", [(0, False), (1, False), (8, False), (1, True), (8, True)])
+def test_pipeline_gradients_match_reference(extra, concurrent):
+    """concurrent=True: the N pipelines run at once (one thread each, one process group per pipeline)."""
     K, N, M = 3, 2, 6
-    out = _run(K, N, M, extra)
+    out = _run(K, N, M, extra, concurrent=concurrent)
     ref = _reference_grads(N, M)
     for k in range(K):
         grads, hist = out[k]
