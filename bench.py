@@ -109,8 +109,8 @@ NVLINK_PEAK_SOURCE = ("measured reference in /opt/skills/guides/B200_PROFILING.m
 def nccl_debug_setup(rank):
     """NCCL_DEBUG=INFO into a per-rank file (unless the caller set NCCL_DEBUG), so the line can report the
     algorithm / protocol / NVLS NCCL chose for the library's communicator."""
-    if "NCCL_DEBUG" in os.environ:
-        return os.environ.get("NCCL_DEBUG_FILE")
+    if os.environ.get("NCCL_DEBUG_FILE"):
+        return os.environ["NCCL_DEBUG_FILE"]
     import tempfile
     path = os.path.join(tempfile.gettempdir(), f"avgpipe_nccl_{os.getpid()}_{rank}.log")
     os.environ["NCCL_DEBUG"] = "INFO"
@@ -125,7 +125,7 @@ def nccl_debug_summary(path, limit=12):
         return None
     import re
     keep, seen = [], set()
-    pat = re.compile(r"(algo|Algo|proto|Proto|NVLS|nvls|CollNet|Channel \d+/|channels|Ring|Tree|comm 0x.*nRanks)")
+    pat = re.compile(r"(algo|proto|nvls|collnet|channel \d+/|channels|ring|tree|nranks|p2p/|via )", re.I)
     for line in open(path, errors="replace"):
         if "NCCL INFO" not in line or not pat.search(line):
             continue
@@ -199,14 +199,21 @@ def workload_key(gpus: int, override):
 
 
 # ----------------------------------------------------------------------------- our arm
+def stale_fused(n, optimizer, variant):
+    """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1, 5..8;
+    Adam(W) up to 6) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
+    return variant == "auto" and n <= 8 and not (optimizer in ("adam", "adamw") and n > 6)
+
+
 def kernel_name(variant, optimizer, n, staleness=0):
     """The co-located kernel the library runs (its per-N default, ea_kernels.cu / ea_api.cu)."""
     force_wide = os.environ.get("AVGPIPE_EA_FORCE_WIDE", "")[:1] == "1"   # ea_api.cu measurement knob
     if force_wide:
         return "colocated_wide" + ("<stale>" if staleness else "")
     if staleness:
-        if 2 <= n <= 4 and variant == "auto":   # ea_api.cu: the lane kernel with x~_{t-1} staged beside x~_t
-            return "colocated_laneshfl<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
+        if stale_fused(n, optimizer, variant):   # ea_api.cu: x~_{t-1} staged beside x~_t, <= 8 stages per launch
+            kern = "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe"
+            return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"
     two_state = optimizer in ("adam", "adamw")
     if n > 8 or (two_state and n > 6 and variant == "auto"):
@@ -228,7 +235,7 @@ def colocated_launches(n, k, args, batched):
     ASGD, the step-counter kernel that precedes each launch."""
     coef = args.optimizer != "sgd"
     two_state = args.optimizer in ("adam", "adamw")
-    stale_lane = args.staleness and 2 <= n <= 4 and args.variant == "auto"
+    stale_lane = args.staleness and stale_fused(n, args.optimizer, args.variant)
     force_wide = os.environ.get("AVGPIPE_EA_FORCE_WIDE", "")[:1] == "1"   # ea_api.cu measurement knob
     per_stage = (n > 8 or not batched or (two_state and n > 6 and args.variant == "auto")
                  or (args.staleness and not stale_lane) or force_wide)

@@ -231,9 +231,14 @@ EA_API ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* st
  * N devices driven by one process): peers[q] is rank q's handle (peers[rank]
  * == h); every handle must call this with the same list.  Ranks created with
  * an NCCL id are connected by ea_init itself (CUDA IPC handles all-gathered
- * over NCCL) and need no call.  All ranks' ea_step kernels wait for one
- * another, so each rank must drive its own stream; ranks that share a device
- * split its SMs.  EA_ESTATE for other layouts/exchanges. */
+ * over NCCL) and need no call.  The ranks' exchange kernels wait for one
+ * another's push kernels, so each rank must drive its own stream; ranks that
+ * share a device split its SMs, and since each rank uses two streams (its
+ * caller's and the library's side stream) the process must run with
+ * CUDA_DEVICE_MAX_CONNECTIONS >= 2 * ranks + 1 (set before the CUDA context
+ * exists): with fewer hardware queues a spinning exchange kernel can sit
+ * ahead of a push it waits for in the same queue, and the wait times out.
+ * EA_ESTATE for other layouts/exchanges. */
 EA_API ea_status ea_p2p_connect(ea_handle h, const ea_handle* peers, int32_t world);
 
 /* EA_XCHG_P2P between processes without an NCCL id (the caller moves the

@@ -319,9 +319,12 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // pipeline and 0.73 lane kernel, profiles/r01_adam_nsweep.jsonl)
   const bool adam_wide = ea::two_state(opt) && n > 6 && h->variant == 0;
   const bool stale = h->cfg.staleness == 1;
-  // stale center: the lane kernel with x~_{t-1} staged beside x~_t for 2 <= N <= 4 under the default variant, else
-  // the replica loop (AVGPIPE_EA_FORCE_WIDE=1 selects the replica loop for A/B measurement)
-  const bool stale_lane = stale && n >= 2 && n <= ea::kMaxStaleLaneN && h->variant == 0 && !force_wide;
+  // stale center, default variant: one launch per <= 8 stages -- the lane kernel with x~_{t-1} staged beside x~_t
+  // for 2 <= N <= 4, the bulk-copy pipeline with x~_{t-1} as one more stream for N = 1 and 5..8 (Adam(W): up to
+  // N = 6, like the synchronous default); else the replica loop, one launch per stage (AVGPIPE_EA_FORCE_WIDE=1
+  // selects it for A/B measurement)
+  const bool stale_lane = stale && n <= ea::kMaxFusedN && !(ea::two_state(opt) && n > 6) && h->variant == 0 &&
+                          !force_wide;
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
     for (int j = 0; j < count; ++j) {
       ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);
@@ -585,12 +588,16 @@ ea_status p2p_ipc_connect(ea_ctx* h) {
 }
 
 // CTAs of p2p_exchange (phases B/C on the side stream).  Its work is NVLink/latency-bound and it runs beside
-// the next forward, so it takes a fraction of the SMs; knob AVGPIPE_EA_P2P_XCTAS (1..4096) for measurement.
-int p2p_exchange_ctas(int num_sms) {
+// the next forward, so it takes a fraction of the SMs: num_sms / 3 per device.  Ranks sharing a device (virtual
+// ranks) split that: their exchange kernels spin while other ranks' pushes on the same device still need SMs, so
+// together they must never be able to fill it (8 ranks x 49 CTAs of 32K registers did, and timed out).  Knob
+// AVGPIPE_EA_P2P_XCTAS (1..4096) for measurement.
+int p2p_exchange_ctas(const ea_ctx* h) {
   const char* e = std::getenv("AVGPIPE_EA_P2P_XCTAS");
   const long long v = e ? std::atoll(e) : 0;
   if (v >= 1 && v <= 4096) return static_cast<int>(v);
-  return num_sms / 3 > 0 ? num_sms / 3 : 1;
+  const int k = h->num_sms / (3 * (h->same_device_ranks > 0 ? h->same_device_ranks : 1));
+  return k > 0 ? k : 1;
 }
 
 // One stage of the peer-memory exchange: p2p_push (local update + contributions into the owners' inboxes) on
@@ -641,14 +648,15 @@ ea_status p2p_step(ea_ctx* h, int32_t stage, float* replica, const float* grad, 
   ea_status st2 = advance(h, &stage, 1, s);
   if (st2 != EA_OK) return st2;
   // ranks sharing this device (virtual ranks) share its SMs
-  int max_ctas = spread_local_sms(h->num_sms) * ea::p2p_blocks_per_sm(h->cfg.optimizer) / h->same_device_ranks;
-  if (max_ctas < 1) max_ctas = 1;
-  if ((e = ea::launch_p2p_push(a, v, h->cfg.optimizer, max_ctas, s)) != cudaSuccess)
+  int max_sms = spread_local_sms(h->num_sms) / h->same_device_ranks;
+  if (max_sms < 1) max_sms = 1;
+  int max_ctas = max_sms * ea::p2p_blocks_per_sm(h->cfg.optimizer);
+  if ((e = ea::launch_p2p_push(a, v, h->cfg.optimizer, max_ctas, max_sms, s)) != cudaSuccess)
     return cuda_fail(h, e, "peer-memory push kernel launch");
   if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
     return cuda_fail(h, e, "cudaStreamWaitEvent");
-  if ((e = ea::launch_p2p_exchange(a, v, p2p_exchange_ctas(h->num_sms), h->side)) != cudaSuccess)
+  if ((e = ea::launch_p2p_exchange(a, v, p2p_exchange_ctas(h), h->side)) != cudaSuccess)
     return cuda_fail(h, e, "peer-memory exchange kernel launch");
   if ((e = cudaEventRecord(h->ev_ag[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   return EA_OK;
@@ -801,9 +809,13 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     }
   }
   if (c.layout == EA_SPREAD) {
-    int prio_lo = 0, prio_hi = 0;  // the exchange's CTAs go first when SMs free up (it is short and latency-bound)
+    // the exchange's CTAs go first when SMs free up (it is short and latency-bound); knob AVGPIPE_EA_SIDE_PRIO=0
+    // keeps the default priority
+    int prio_lo = 0, prio_hi = 0;
     cudaDeviceGetStreamPriorityRange(&prio_lo, &prio_hi);
-    if ((e = cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, prio_hi)) != cudaSuccess ||
+    const char* pe = std::getenv("AVGPIPE_EA_SIDE_PRIO");
+    const int prio = (pe && pe[0] == '0') ? prio_lo : prio_hi;
+    if ((e = cudaStreamCreateWithPriority(&h->side, cudaStreamNonBlocking, prio)) != cudaSuccess ||
         (e = cudaEventCreateWithFlags(&h->ev_done, cudaEventDisableTiming)) != cudaSuccess ||
         (c.exchange == EA_XCHG_NCCL && (e = cudaMalloc(&h->contrib, sizeof(float) * sum_pad)) != cudaSuccess) ||
         (e = cudaMalloc(&h->reduced, sizeof(float) * (max_pad / c.n_pipelines))) != cudaSuccess) {

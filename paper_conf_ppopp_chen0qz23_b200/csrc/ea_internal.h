@@ -105,9 +105,9 @@ enum KernelVariant : int {
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s);
 
-// Stale center (row f4) for a batch of stages with 2 <= N <= kMaxStaleLaneN (N = 1's two 16 KB tiles
-// double-buffered exceed static shared memory), every st[].prev set: the lane kernel
-// with x~_{t-1} staged beside x~_t (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
+// Stale center (row f4) for a batch of stages with N <= kMaxFusedN, every st[].prev set: for
+// 2 <= N <= kMaxStaleLaneN the lane kernel with x~_{t-1} staged beside x~_t, otherwise the bulk-copy pipeline
+// with x~_{t-1} as one more stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
 constexpr int kMaxStaleLaneN = 4;
 cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int num_sms,
                                          cudaStream_t s);
@@ -155,8 +155,10 @@ struct P2PArgs {
   int sc_fence;        // 1: fence.sc.sys before each release (knob AVGPIPE_EA_P2P_FENCE=1; default 0)
 };
 
-// Phase A (local update, contributions pushed into the owners' inboxes): never waits.
-cudaError_t launch_p2p_push(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, cudaStream_t s);
+// Phase A (local update, contributions pushed into the owners' inboxes): never waits.  Default: the bulk-copy
+// ring kernel, one CTA per SM on at most max_sms SMs; knob AVGPIPE_EA_P2P_PUSH=plain: the register loop with up
+// to max_ctas CTAs.
+cudaError_t launch_p2p_push(const P2PArgs& a, const P2PView& v, int opt, int max_ctas, int max_sms, cudaStream_t s);
 // Phases B (owner reduction + center update) and C (pull the other owners' chunks), ticket-ordered.
 cudaError_t launch_p2p_exchange(const P2PArgs& a, const P2PView& v, int max_ctas, cudaStream_t s);
 int p2p_blocks_per_sm(int opt);

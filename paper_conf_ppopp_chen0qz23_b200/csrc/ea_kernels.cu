@@ -22,6 +22,7 @@
 
 #include "ea_internal.h"
 #include "ea_update.cuh"
+#include "ea_bulk.cuh"
 
 namespace ea {
 namespace {
@@ -344,41 +345,6 @@ __global__ void __launch_bounds__(kThreads) colocated_wide(const ReplicaTable t,
 // ============================================================================
 constexpr int kLanePasses = 4;  // float4 chunks per lane per tile
 
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-__device__ __forceinline__ void mbar_expect_tx(uint64_t* bar, uint32_t bytes) {
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-               : "memory");
-}
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-  asm volatile(
-      "{\n"
-      ".reg .pred P1;\n"
-      "WAIT_%=:\n"
-      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
-      "@!P1 bra WAIT_%=;\n"
-      "}\n" ::"r"(smem_u32(bar)),
-      "r"(parity)
-      : "memory");
-}
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-  asm volatile(
-      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-          smem_u32(dst)),
-      "l"(src), "r"(bytes), "r"(smem_u32(bar))
-      : "memory");
-}
-__device__ __forceinline__ void fence_proxy_async() {
-  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-}
-
 template <int N>
 struct LanePow2 {
   static constexpr int value = N <= 1 ? 1 : N <= 2 ? 2 : N <= 4 ? 4 : N <= 8 ? 8 : 16;
@@ -526,18 +492,19 @@ constexpr int kBulkThreads = 32 * (kBulkConsumerWarps + 1);
 // producer lanes (profiles/r01_s2_bulk_lanes_tiles.jsonl, r01_s2_issue_ab.jsonl): 4 KB copies whenever a
 // two-stage ring of them fits in 200 KB (SGD N <= 8, Adam N <= 6), else 2 KB.  Smaller copies lose: the ring
 // depth is capped, so bytes in flight per SM shrink with the tile (1 KB: 0.27-0.69 of peak).
-template <int N, int A = 3>
+template <int N, int A = 3, int X = 0>
 constexpr int default_bulk_tile() {
-  return (A * N + 1) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128;
+  return (A * N + 1 + X) * 256 * 16 * 2 <= 200 * 1024 ? 256 : 128;
 }
 
 constexpr int kMaxBulkStages = 6;  // ring depth cap (8 measured slower: profiles/r01_bulk_n4_tiles.jsonl)
 
-// A = streams per replica in the slot: 3 (x, g, m) for SGD, 4 (x, g, m, v) for Adam.
-template <int N, int TILE, int A>
+// A = streams per replica in the slot: 3 (x, g, m) for SGD, 4 (x, g, m, v) for Adam; X = extra center streams
+// (1: the stale center x~_{t-1}, row f4).
+template <int N, int TILE, int A, int X = 0>
 struct BulkGeom {
-  static constexpr int kTile = TILE;                      // float4 per array per tile
-  static constexpr int kSlotVec = (A * N + 1) * kTile;    // float4 per slot
+  static constexpr int kTile = TILE;                          // float4 per array per tile
+  static constexpr int kSlotVec = (A * N + 1 + X) * kTile;    // float4 per slot
   static constexpr int kFit = (200 * 1024) / (kSlotVec * 16);
   static constexpr int kStages = kFit > kMaxBulkStages ? kMaxBulkStages : (kFit < 2 ? 2 : kFit);
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
@@ -560,11 +527,15 @@ __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, 
 
 // SPREAD = false: co-located stages (x~ updated in place).  SPREAD = true: the spread layout's local
 // step (N = 1, one stage): x~ is only read and the contribution r goes to `contrib` (rows a1-a4).
-template <int N, int HINT, int OPT, int TILE, bool SPREAD>
+// STALE (co-located, row f4, reading c28): every stage's x~_{t-1} (st.prev) is one more stream of the slot;
+// the replicas dilute with and measure their gap to it, x~_{t+1} = x~_t + R/N, prev <- x~_t.
+template <int N, int HINT, int OPT, int TILE, bool SPREAD, bool STALE = false>
 __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& hp, float* __restrict__ contrib,
                                               int64_t p_pad, int issue_lanes) {
   constexpr int A = two_state(OPT) ? 4 : 3;
-  using G = BulkGeom<N, TILE, A>;
+  constexpr int X = STALE ? 1 : 0;
+  constexpr int NS = A * N + 1 + X;  // streams per slot
+  using G = BulkGeom<N, TILE, A, X>;
   constexpr int T = G::kTile, S = G::kStages;
   extern __shared__ __align__(128) float4 smem[];
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + S * G::kSlotVec);
@@ -597,12 +568,14 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
       float4* base = smem + slot * G::kSlotVec;
       const uint32_t bytes = static_cast<uint32_t>(nv * 16);
       const StageRefs& st = b.st[s];
-      if (lane == 0) mbar_expect_tx(&full[slot], bytes * (A * N + 1));
+      if (lane == 0) mbar_expect_tx(&full[slot], bytes * NS);
       __syncwarp();
-      for (int q = lane; q < A * N + 1 && lane < issue_lanes; q += issue_lanes) {
+      for (int q = lane; q < NS && lane < issue_lanes; q += issue_lanes) {
         const float* src;
         if (q == 0) {
           src = st.c;
+        } else if (STALE && q == A * N + 1) {
+          src = st.prev;
         } else {
           const int i = (q - 1) / A, kind = (q - 1) % A;
           src = kind == 0 ? st.x[i] : kind == 1 ? st.g[i] : kind == 2 ? st.m[i] : st.v[i];
@@ -623,6 +596,7 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
       const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
       for (int lv = threadIdx.x; lv < nv; lv += 32 * kBulkConsumerWarps) {
         const float4 c = base[lv];
+        const float4 cu = STALE ? base[(A * N + 1) * T + lv] : c;  // the center the replicas see
         float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
         const int64_t v = v0 + lv;
 #pragma unroll
@@ -631,15 +605,17 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
           const float4 g = base[(2 + A * i) * T + lv];
           float4 m = base[(3 + A * i) * T + lv];
           float4 w = A == 4 ? base[(4 + A * i) * T + lv] : make_float4(0.f, 0.f, 0.f, 0.f);
-          add4(acc, ea_vec<OPT>(x, g, m, w, c, hp, sc));
+          add4(acc, ea_vec<OPT>(x, g, m, w, cu, hp, sc));
           mem.st(st.x[i] + 4 * v, x);
           mem.st(st.m[i] + 4 * v, m);
           if (A == 4) mem.st(st.v[i] + 4 * v, w);
         }
-        if constexpr (SPREAD)
+        if constexpr (SPREAD) {
           mem.st(contrib + 4 * v, acc);
-        else
+        } else {
           mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
+          if constexpr (STALE) mem.st(st.prev + 4 * v, c);
+        }
       }
       // all consumer warps are done reading the slot, then one release-arrive hands it back
       asm volatile("bar.sync 1, %0;" ::"n"(32 * kBulkConsumerWarps) : "memory");
@@ -649,15 +625,15 @@ __device__ __forceinline__ void bulkpipe_body(const StageBatch& b, const Hyper& 
       if constexpr (SPREAD)
         spread_tail<OPT>(b.st[0], contrib, p_pad, hp);
       else
-        for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+        for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
     }
   }
 }
 
-template <int N, int HINT, int OPT, int TILE>
+template <int N, int HINT, int OPT, int TILE, bool STALE = false>
 __global__ void __launch_bounds__(kBulkThreads, 1) colocated_bulkpipe(const StageBatch b, const Hyper hp,
                                                                       int issue_lanes) {
-  bulkpipe_body<N, HINT, OPT, TILE, false>(b, hp, nullptr, 0, issue_lanes);
+  bulkpipe_body<N, HINT, OPT, TILE, false, STALE>(b, hp, nullptr, 0, issue_lanes);
 }
 
 // Spread local step (one replica) through the same bulk-copy pipeline: 4 input streams (x, g, state, x~;
@@ -854,10 +830,10 @@ int bulk_issue_lanes() {
   return v;
 }
 
-template <int N, int HINT, int OPT, int TILE>
+template <int N, int HINT, int OPT, int TILE, bool STALE = false>
 cudaError_t launch_bulkpipe_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using G = BulkGeom<N, TILE, two_state(OPT) ? 4 : 3>;
-  auto k = colocated_bulkpipe<N, HINT, OPT, TILE>;
+  using G = BulkGeom<N, TILE, two_state(OPT) ? 4 : 3, STALE ? 1 : 0>;
+  auto k = colocated_bulkpipe<N, HINT, OPT, TILE, STALE>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
   if (e != cudaSuccess) return e;
   int64_t grid = num_sms;  // one block per SM (the ring takes most of shared memory)
@@ -1039,6 +1015,18 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   }
 }
 
+// Stale center through the bulk-copy pipeline (N = 1 and 5..8: the lane kernel's double-buffered pair of
+// center tiles does not fit its static shared memory at N = 1, and it idles lanes beyond N = 4).
+template <int N>
+cudaError_t launch_stale_bulk_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
+  switch (opt) {
+    case kOptAdam: return launch_bulkpipe_t<N, 0, kOptAdam, default_bulk_tile<N, 4, 1>(), true>(b, hp, num_sms, s);
+    case kOptAdamW: return launch_bulkpipe_t<N, 0, kOptAdamW, default_bulk_tile<N, 4, 1>(), true>(b, hp, num_sms, s);
+    case kOptASGD: return launch_bulkpipe_t<N, 0, kOptASGD, default_bulk_tile<N, 3, 1>(), true>(b, hp, num_sms, s);
+    default: return launch_bulkpipe_t<N, 0, kOptSGD, default_bulk_tile<N, 3, 1>(), true>(b, hp, num_sms, s);
+  }
+}
+
 template <int N>
 cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
   switch (opt) {
@@ -1055,9 +1043,14 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   for (int t = 0; t < b.nstages; ++t)
     if (!b.st[t].prev) return cudaErrorInvalidValue;
   switch (n) {
+    case 1: return launch_stale_bulk_n<1>(b, hp, opt, num_sms, s);
     case 2: return launch_stale_n<2>(b, hp, opt, num_sms, s);
     case 3: return launch_stale_n<3>(b, hp, opt, num_sms, s);
     case 4: return launch_stale_n<4>(b, hp, opt, num_sms, s);
+    case 5: return launch_stale_bulk_n<5>(b, hp, opt, num_sms, s);
+    case 6: return launch_stale_bulk_n<6>(b, hp, opt, num_sms, s);
+    case 7: return launch_stale_bulk_n<7>(b, hp, opt, num_sms, s);
+    case 8: return launch_stale_bulk_n<8>(b, hp, opt, num_sms, s);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -77,17 +77,22 @@ def test_traffic_is_keyed_by_kernel(optimizer):
 
 
 def test_stale_kernel_name_and_launches(monkeypatch):
-    """Row f4: the lane kernel for 2 <= N <= 4 (one launch per <= 8 stages), the replica loop otherwise and
-    under the AVGPIPE_EA_FORCE_WIDE knob (one launch per stage) -- the dispatch in ea_api.cu."""
+    """Row f4: the lane kernel for 2 <= N <= 4 and the bulk-copy pipeline for N = 1, 5..8 (Adam(W) to 6), one
+    launch per <= 8 stages; the replica loop otherwise and under the AVGPIPE_EA_FORCE_WIDE knob (one launch per
+    stage) -- the dispatch in ea_api.cu."""
     import argparse
     monkeypatch.delenv("AVGPIPE_EA_FORCE_WIDE", raising=False)
     assert bench.kernel_name("auto", "sgd", 4, 1) == "colocated_laneshfl<stale>"
     assert bench.kernel_name("auto", "asgd", 2, 1) == "colocated_laneshfl<stale,asgd>"
-    assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_wide<stale>"
-    assert bench.kernel_name("auto", "sgd", 8, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_bulkpipe<stale>"
+    assert bench.kernel_name("auto", "sgd", 8, 1) == "colocated_bulkpipe<stale>"
+    assert bench.kernel_name("auto", "adam", 6, 1) == "colocated_bulkpipe<stale,adam>"
+    assert bench.kernel_name("auto", "adam", 7, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "sgd", 12, 1) == "colocated_wide<stale>"
     args = argparse.Namespace(optimizer="sgd", variant="auto", staleness=1)
     assert bench.colocated_launches(4, 4, args, True) == 1
-    assert bench.colocated_launches(8, 4, args, True) == 4
+    assert bench.colocated_launches(8, 4, args, True) == 1
+    assert bench.colocated_launches(12, 4, args, True) == 4
     monkeypatch.setenv("AVGPIPE_EA_FORCE_WIDE", "1")
     assert bench.kernel_name("auto", "sgd", 4, 1) == "colocated_wide<stale>"
     assert bench.colocated_launches(4, 4, args, True) == 4

@@ -13,7 +13,7 @@ import torch
 from oracle.ea_oracle import Hyper, ea_step, ea_step_adam
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import ElasticAveraging
-from tests._parity import TOL, hyper, rel_err
+from tests._parity import TOL, OracleStage, asgd_kw, hyper, rel_err
 
 pytestmark = pytest.mark.gpu
 
@@ -68,6 +68,75 @@ def _run_sampled(n, sizes, steps, variant, mode="combined", many=True, k=200_000
                 assert rel_err(f64(reps[i], idx), ox[i]) <= TOL, (s, t, i)
                 assert rel_err(f64(h.momentum(s, i), idx), om[i]) <= TOL, (s, t, i)
     h.close()
+
+
+def _run_trajectory(n, sizes, steps, optimizer, mode="combined", k=100_000, graph=True, checkpoints=(1, 10, 50)):
+    """100-step ACCUMULATED parity at full size: the oracle evolves only the sampled elements (the update is
+    elementwise over j), from the same initial state and with the same gradients gathered at those indices every
+    step; the GPU runs the whole stages exactly as bench.py times them (ea_step_many, default kernel, replayed as
+    one captured CUDA graph).  Compared at the checkpoints and after the last step (c13 <= 1e-5)."""
+    dev = torch.device("cuda:0")
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    hp = hyper(n, mode, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+    h = ElasticAveraging(sizes, n, alpha=hp.alpha, beta=hp.beta, rho=hp.rho, lr=hp.lr, momentum=hp.momentum,
+                         weight_decay=hp.weight_decay, optimizer=optimizer, betas=(hp.beta1, hp.beta2), eps=hp.eps,
+                         **asgd_kw(hp))
+    gen = torch.Generator(device=dev)
+    gen.manual_seed(11)
+    rng = np.random.default_rng(1)
+    state, oracle = [], []
+    f64 = lambda t_, idx: t_[idx].double().cpu().numpy()
+    for s, p in enumerate(sizes):
+        reps, c, grads = synth.device_state(n, p, dev, seed=s)
+        idx = _sample_idx(p, k, rng).to(dev)
+        state.append((reps, c, grads, idx))
+        oracle.append(OracleStage([f64(x, idx) for x in reps], f64(c, idx), optimizer))
+    order = list(reversed(range(len(sizes))))
+    run = lambda st=None: h.step_many(order, [state[s][0] for s in order], [state[s][2] for s in order],
+                                      [state[s][1] for s in order], stream=st)
+    if graph:
+        g = torch.cuda.CUDAGraph()
+        side = torch.cuda.Stream()
+        side.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(side):
+            with torch.cuda.graph(g, stream=side):
+                run(side)
+        torch.cuda.synchronize()
+        run = g.replay
+    worst = 0.0
+    for t in range(1, steps + 1):
+        for s, (reps, c, grads, idx) in enumerate(state):
+            for gr in grads:
+                gr.normal_(0.0, synth.GRAD_STD, generator=gen)
+            oracle[s].step([f64(gr, idx) for gr in grads], hp)
+        run()
+        if t in checkpoints or t == steps:
+            torch.cuda.synchronize()
+            for s, (reps, c, grads, idx) in enumerate(state):
+                o = oracle[s]
+                errs = [rel_err(f64(c, idx), o.c)]
+                for i in range(n):
+                    errs.append(rel_err(f64(reps[i], idx), o.xs[i]))
+                    errs.append(rel_err(f64(h.state(s, i, 0), idx), o.ms[i]))
+                    if optimizer in ("adam", "adamw"):
+                        errs.append(rel_err(f64(h.state(s, i, 1), idx), o.vs[i]))
+                worst = max(worst, max(errs))
+                assert max(errs) <= TOL, (optimizer, t, s, max(errs))
+    h.close()
+    return worst
+
+
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+def test_c2_full_size_100_steps_accumulated(optimizer):
+    """The north-star gate at the bench's full size: C2 (25 M params, K=4, N=4), 100 steps, sampled."""
+    cfg = synth.CONFIGS["C2"]
+    _run_trajectory(cfg.n_pipelines, cfg.stage_sizes, 100, optimizer)
+
+
+def test_c4_stage_100_steps_accumulated():
+    """One C4-sized stage (44.4 M params) co-located with N = 8 (the 1-GPU point of the C4 curve), 100 steps."""
+    cfg = synth.CONFIGS["C4"]
+    _run_trajectory(8, cfg.stage_sizes[:1], 100, "sgd", k=50_000)
 
 
 @pytest.mark.parametrize("variant", ["auto", "regloop", "laneshfl", "bulkpipe"])

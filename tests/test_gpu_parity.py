@@ -164,7 +164,7 @@ def test_asgd_replica_counts_and_sizes(n):
 
 
 # ------------------------------------------------------------------ stale center (row f4)
-@pytest.mark.parametrize("n", [1, 2, 3, 4, 8, 12])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8, 12])
 @pytest.mark.parametrize("mode", synth.MODES)
 def test_stale_center(n, mode):
     """staleness 1 (reading c28): replicas dilute with x~_{t-1}, the center moves from x~_t."""
@@ -173,7 +173,7 @@ def test_stale_center(n, mode):
 
 
 @pytest.mark.parametrize("optimizer", ["adam", "adamw"])
-@pytest.mark.parametrize("n", [1, 2, 3, 4, 8, 12])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 8, 12])
 def test_stale_center_adam(optimizer, n):
     """staleness 1 with Adam / AdamW as the local optimizer (readings c28 + c21)."""
     _run_colocated(n, [100_003, 7, 4096], 30, "combined", variants=("auto",), staleness=1, many=True,
@@ -181,7 +181,7 @@ def test_stale_center_adam(optimizer, n):
     _run_colocated(n, [65_537], 15, "paper", variants=("auto",), staleness=1, optimizer=optimizer, lr=1e-3)
 
 
-@pytest.mark.parametrize("n", [1, 2, 3, 4, 8, 12])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 6, 8, 12])
 def test_stale_center_asgd(n):
     """staleness 1 with ASGD as the local optimizer (readings c28 + c29; averaging from step 7 on)."""
     _run_colocated(n, [100_003, 7, 4096], 30, "combined", variants=("auto",), staleness=1, many=True,
@@ -193,9 +193,10 @@ def test_stale_center_c1_100_steps():
     _run_colocated(2, [1_000_000, 1_000_003], 100, "combined", variants=("auto",), staleness=1, many=True)
 
 
-@pytest.mark.parametrize("n,optimizer", [(3, "sgd"), (4, "adamw"), (2, "asgd")])
+@pytest.mark.parametrize("n,optimizer", [(3, "sgd"), (4, "adamw"), (2, "asgd"), (1, "sgd"), (6, "adam"), (8, "asgd")])
 def test_stale_center_many_stage_batches(n, optimizer):
-    """11 stages in one ea_step_many: the stale lane kernel (2 <= N <= 4) splits them into launches of 8 + 3."""
+    """11 stages in one ea_step_many: the stale lane kernel (2 <= N <= 4) / bulk-copy pipeline (N = 1, 5..8)
+    splits them into launches of 8 + 3."""
     sizes = [4096 * (k + 1) + k for k in range(11)]
     _run_colocated(n, sizes, 12, "combined", variants=("auto",), staleness=1, many=True, optimizer=optimizer,
                    lr=1e-3 if optimizer in ("adam", "adamw") else synth.LR)
@@ -360,8 +361,9 @@ def test_spread_nccl_world1_and_stream_order():
         assert rel_err(to_np(xs[s]), oracle[s].xs[0]) <= TOL
         assert rel_err(to_np(cs[s][:p]), oracle[s].c) <= TOL
         assert rel_err(to_np(h.momentum(s, 0)), oracle[s].ms[0]) <= TOL
+    buf = torch.zeros(sizes[0] + 4, device=dev)
     with pytest.raises(EAError):
-        h.step(0, [xs[0][1:]], [xs[0][1:]], cs[0])   # misaligned pointers -> EA_EINVAL
+        h.step(0, [buf[1:sizes[0] + 1]], [buf[1:sizes[0] + 1]], cs[0])   # misaligned pointers -> EA_EINVAL
     h.close()
 
 
