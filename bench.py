@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe"), default="auto")
+    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe", "split"), default="auto")
     ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw", "asgd"), default="sgd",
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam(W) and ASGD are row f1)")
     ap.add_argument("--staleness", type=int, choices=(0, 1), default=0,
@@ -200,9 +200,9 @@ def workload_key(gpus: int, override):
 
 # ----------------------------------------------------------------------------- our arm
 def stale_fused(n, optimizer, variant):
-    """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1, 5..8;
-    Adam(W) up to 6) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
-    return variant == "auto" and n <= 8 and not (optimizer in ("adam", "adamw") and n > 6)
+    """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1; N = 5 for
+    SGD/ASGD) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
+    return variant == "auto" and (n <= 4 or (n == 5 and optimizer not in ("adam", "adamw")))
 
 
 def kernel_name(variant, optimizer, n, staleness=0):

@@ -69,7 +69,7 @@ extern "C" {
 #define EA_API
 #endif
 
-#define EA_ABI_VERSION 4
+#define EA_ABI_VERSION 5
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
@@ -120,9 +120,11 @@ typedef struct {
                                    0 = library default, 1 = register-resident replica loop,
                                    2 = lane-per-replica, center tile staged by cp.async.bulk,
                                    warp-shuffle reduction, 3 = bulk-copy pipeline (every input
-                                   tile by cp.async.bulk into an mbarrier ring).  Same results
-                                   up to fp32 summation order (DESIGN.md c14).  Adam(W) always
-                                   uses 2 (or the N > 8 kernel). */
+                                   tile by cp.async.bulk into an mbarrier ring), 4 = split
+                                   register loop (two lanes per center column, N/2 replicas
+                                   each, shuffle reduction).  Same results up to fp32 summation
+                                   order (DESIGN.md c14); the default picks per N and optimizer
+                                   (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */
   double beta1, beta2;          /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999); double so
                                    that 1-beta2 keeps full precision (0.999f would be off by 1.3e-5) */

@@ -320,11 +320,11 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   const bool adam_wide = ea::two_state(opt) && n > 6 && h->variant == 0;
   const bool stale = h->cfg.staleness == 1;
   // stale center, default variant: one launch per <= 8 stages -- the lane kernel with x~_{t-1} staged beside x~_t
-  // for 2 <= N <= 4, the bulk-copy pipeline with x~_{t-1} as one more stream for N = 1 and 5..8 (Adam(W): up to
-  // N = 6, like the synchronous default); else the replica loop, one launch per stage (AVGPIPE_EA_FORCE_WIDE=1
-  // selects it for A/B measurement)
-  const bool stale_lane = stale && n <= ea::kMaxFusedN && !(ea::two_state(opt) && n > 6) && h->variant == 0 &&
-                          !force_wide;
+  // for 2 <= N <= 4, the bulk-copy pipeline with x~_{t-1} as one more stream for N = 1 (and N = 5 for SGD/ASGD);
+  // else the replica loop, one launch per stage, which measured better from N = 6 on (N = 8: 0.954 vs 0.903;
+  // Adam N = 6: 0.925 vs 0.775 of HBM peak, profiles/r02_sweep_kernels.jsonl).  AVGPIPE_EA_FORCE_WIDE=1 selects
+  // the replica loop for A/B measurement.
+  const bool stale_lane = stale && (n <= 4 || (n == 5 && !ea::two_state(opt))) && h->variant == 0 && !force_wide;
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
     for (int j = 0; j < count; ++j) {
       ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);
@@ -588,15 +588,17 @@ ea_status p2p_ipc_connect(ea_ctx* h) {
 }
 
 // CTAs of p2p_exchange (phases B/C on the side stream).  Its work is NVLink/latency-bound and it runs beside
-// the next forward, so it takes a fraction of the SMs: num_sms / 3 per device.  Ranks sharing a device (virtual
-// ranks) split that: their exchange kernels spin while other ranks' pushes on the same device still need SMs, so
-// together they must never be able to fill it (8 ranks x 49 CTAs of 32K registers did, and timed out).  Knob
-// AVGPIPE_EA_P2P_XCTAS (1..4096) for measurement.
+// the next forward, so one rank per device takes num_sms / 3.  Ranks sharing a device (virtual ranks) must
+// together never be able to fill it: their exchange kernels spin while other ranks' pushes on the same device
+// still need SMs (8 ranks x 49 CTAs of 32K registers did fill it, and timed out).  An exchange CTA holds half an
+// SM's registers, so at most num_sms of them over all ranks always leave a push CTA room on every SM (or half
+// the SMs free): num_sms / ranks each.  Knob AVGPIPE_EA_P2P_XCTAS (1..4096) for measurement.
 int p2p_exchange_ctas(const ea_ctx* h) {
   const char* e = std::getenv("AVGPIPE_EA_P2P_XCTAS");
   const long long v = e ? std::atoll(e) : 0;
   if (v >= 1 && v <= 4096) return static_cast<int>(v);
-  const int k = h->num_sms / (3 * (h->same_device_ranks > 0 ? h->same_device_ranks : 1));
+  const int ranks = h->same_device_ranks > 0 ? h->same_device_ranks : 1;
+  const int k = ranks > 1 ? h->num_sms / ranks : h->num_sms / 3;
   return k > 0 ? k : 1;
 }
 
@@ -736,7 +738,7 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (c.world != c.n_pipelines) { set_err(nullptr, "EA_SPREAD needs world == n_pipelines"); return EA_EINVAL; }
     if (c.rank < 0 || c.rank >= c.world) { set_err(nullptr, "rank %d out of [0,%d)", c.rank, c.world); return EA_EINVAL; }
   }
-  if (c.kernel_variant < 0 || c.kernel_variant > 3) { set_err(nullptr, "kernel_variant must be 0..3"); return EA_EINVAL; }
+  if (c.kernel_variant < 0 || c.kernel_variant > 4) { set_err(nullptr, "kernel_variant must be 0..4"); return EA_EINVAL; }
   if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
   if (c.staleness != 0 && c.staleness != 1) { set_err(nullptr, "staleness must be 0 or 1"); return EA_EINVAL; }
   if (c.staleness == 1 && c.layout == EA_SPREAD && c.exchange != EA_XCHG_NCCL) {

@@ -97,6 +97,7 @@ enum KernelVariant : int {
                          // into shared memory; replica reduction by warp shuffles (SGD, Adam)
   kVariantBulkPipe = 3,  // every input tile streamed by cp.async.bulk into a multi-stage smem
                          // ring (producer warp + mbarriers); consumers store from registers (SGD)
+  kVariantSplit = 4,     // split register loop: 2 lanes per center column, N/2 replicas each, shuffle reduction
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N
@@ -105,9 +106,9 @@ enum KernelVariant : int {
 cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, int opt, int variant, int num_sms,
                                    cudaStream_t s);
 
-// Stale center (row f4) for a batch of stages with N <= kMaxFusedN, every st[].prev set: for
-// 2 <= N <= kMaxStaleLaneN the lane kernel with x~_{t-1} staged beside x~_t, otherwise the bulk-copy pipeline
-// with x~_{t-1} as one more stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
+// Stale center (row f4) for a batch of stages with N <= 5, every st[].prev set: for 2 <= N <= kMaxStaleLaneN the
+// lane kernel with x~_{t-1} staged beside x~_t, for N = 1 and 5 the bulk-copy pipeline with x~_{t-1} as one more
+// stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
 constexpr int kMaxStaleLaneN = 4;
 cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int num_sms,
                                          cudaStream_t s);

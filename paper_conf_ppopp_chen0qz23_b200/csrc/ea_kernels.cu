@@ -225,6 +225,76 @@ __global__ void __launch_bounds__(kThreads, regloop_min_blocks<N, OPT>()) coloca
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
 
+// ============================================================================
+// Variant 4: split register loop -- S adjacent lanes share one float4 column of the center, each holding the
+// loads of N/S replicas in registers (all hoisted before any arithmetic), partial contributions reduced by
+// __shfl_xor over the S lanes, the first lane of the group writes x~.  For large N, where the one-thread-per-
+// column register loop needs (A N + 1) float4 of loads per thread (Adam N = 8: 200+ registers, 1 CTA/SM), this
+// keeps the bytes in flight per thread the same per replica group and the CTAs per SM high.  The S lanes of a
+// group load the same center word (one sector: no extra DRAM traffic).
+// ============================================================================
+template <int N, int S, int OPT>
+__global__ void __launch_bounds__(kThreads, 2) colocated_split(const StageBatch b, const Hyper hp) {
+  constexpr int NS = (N + S - 1) / S;  // replicas per lane
+  constexpr bool kTwo = two_state(OPT);
+  constexpr int COLS = kThreads / S;   // float4 columns per CTA pass
+  const Mem<0> mem;
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
+  if (has_coef(OPT)) {
+    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+    __syncthreads();
+  }
+  const int sub = threadIdx.x % S, col = threadIdx.x / S;
+  WaveCursor cur{0, 0};
+  int s;
+  int64_t v0, nv;
+  while (wave_item(b, COLS, cur, s, v0, nv)) {
+    const StageRefs& st = b.st[s];
+    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
+    for (int64_t base = 0; base < nv; base += COLS) {  // block-uniform bound: every lane reaches the shuffles
+      const int64_t lv = base + col;
+      const bool on = lv < nv;
+      const int64_t v = v0 + lv;
+      float4 c = make_float4(0.f, 0.f, 0.f, 0.f);
+      float4 x[NS], g[NS], m[NS], w[kTwo ? NS : 1];
+      if (on) c = mem.ld(st.c + 4 * v);
+#pragma unroll
+      for (int k = 0; k < NS; ++k) {
+        const int i = sub * NS + k;
+        if (on && i < N) {
+          x[k] = mem.ld(st.x[i] + 4 * v);
+          g[k] = mem.ld_ro(st.g[i] + 4 * v);
+          m[k] = mem.ld(st.m[i] + 4 * v);
+          if constexpr (kTwo) w[k] = mem.ld(st.v[i] + 4 * v);
+        }
+      }
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+      for (int k = 0; k < NS; ++k) {
+        const int i = sub * NS + k;
+        if (on && i < N) {
+          float4 unused = make_float4(0.f, 0.f, 0.f, 0.f);
+          float4& wv = kTwo ? w[kTwo ? k : 0] : unused;
+          add4(acc, ea_vec<OPT>(x[k], g[k], m[k], wv, c, hp, sc));
+          mem.st(st.x[i] + 4 * v, x[k]);
+          mem.st(st.m[i] + 4 * v, m[k]);
+          if constexpr (kTwo) mem.st(st.v[i] + 4 * v, wv);
+        }
+      }
+#pragma unroll
+      for (int off = 1; off < S; off <<= 1) {
+        acc.x += __shfl_xor_sync(0xffffffffu, acc.x, off);
+        acc.y += __shfl_xor_sync(0xffffffffu, acc.y, off);
+        acc.z += __shfl_xor_sync(0xffffffffu, acc.z, off);
+        acc.w += __shfl_xor_sync(0xffffffffu, acc.w, off);
+      }
+      if (on && sub == 0) mem.st(st.c + 4 * v, center_apply(c, acc, hp.inv_n));
+    }
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+}
+
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -871,8 +941,25 @@ cudaError_t launch_bulkpipe(const StageBatch& b, const Hyper& hp, int num_sms, c
   return launch_bulkpipe_t<N, HINT, OPT, default_bulk_tile<N, A>()>(b, hp, num_sms, s);
 }
 
+// Split register loop (variant 4): S = 2 lanes per column (N <= 4: S = 1 would be the plain register loop).
+template <int N, int OPT>
+cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  constexpr int S = N <= 4 ? 1 : 2;
+  auto k = colocated_split<N, S, OPT>;
+  k<<<persistent_grid(k, units_of(b, kThreads / S), num_sms), kThreads, 0, s>>>(b, hp);
+  return cudaGetLastError();
+}
+
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (variant == kVariantSplit) {
+    switch (opt) {
+      case kOptAdam: return launch_split<N, kOptAdam>(b, hp, num_sms, s);
+      case kOptAdamW: return launch_split<N, kOptAdamW>(b, hp, num_sms, s);
+      case kOptASGD: return launch_split<N, kOptASGD>(b, hp, num_sms, s);
+      default: return launch_split<N, kOptSGD>(b, hp, num_sms, s);
+    }
+  }
   if (opt == kOptASGD) {  // SGD's streams and geometry (one state vector), no L2-hint variants
     if (variant == kVariantBulkPipe) return launch_bulkpipe<N, 0, kOptASGD>(b, hp, num_sms, s);
     if (variant == kVariantRegLoop) return launch_regloop<N, 0, kOptASGD>(b, hp, num_sms, s);
@@ -1015,8 +1102,10 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   }
 }
 
-// Stale center through the bulk-copy pipeline (N = 1 and 5..8: the lane kernel's double-buffered pair of
-// center tiles does not fit its static shared memory at N = 1, and it idles lanes beyond N = 4).
+// Stale center through the bulk-copy pipeline (N = 1: the lane kernel's double-buffered pair of center tiles does
+// not fit its static shared memory; N = 5: the lane kernel would idle 3 of 8 lanes).  Measured on B200 (C2 sizes,
+// profiles/r02_sweep_kernels.jsonl): N = 1 0.964 vs 0.777 for the replica loop, N = 5 0.958 vs 0.951; from N = 6
+// on the replica loop is better and the library uses it.
 template <int N>
 cudaError_t launch_stale_bulk_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
   switch (opt) {
@@ -1048,9 +1137,6 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
     case 3: return launch_stale_n<3>(b, hp, opt, num_sms, s);
     case 4: return launch_stale_n<4>(b, hp, opt, num_sms, s);
     case 5: return launch_stale_bulk_n<5>(b, hp, opt, num_sms, s);
-    case 6: return launch_stale_bulk_n<6>(b, hp, opt, num_sms, s);
-    case 7: return launch_stale_bulk_n<7>(b, hp, opt, num_sms, s);
-    case 8: return launch_stale_bulk_n<8>(b, hp, opt, num_sms, s);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -85,13 +85,15 @@ def test_stale_kernel_name_and_launches(monkeypatch):
     assert bench.kernel_name("auto", "sgd", 4, 1) == "colocated_laneshfl<stale>"
     assert bench.kernel_name("auto", "asgd", 2, 1) == "colocated_laneshfl<stale,asgd>"
     assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_bulkpipe<stale>"
-    assert bench.kernel_name("auto", "sgd", 8, 1) == "colocated_bulkpipe<stale>"
-    assert bench.kernel_name("auto", "adam", 6, 1) == "colocated_bulkpipe<stale,adam>"
-    assert bench.kernel_name("auto", "adam", 7, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "sgd", 5, 1) == "colocated_bulkpipe<stale>"
+    assert bench.kernel_name("auto", "adam", 1, 1) == "colocated_bulkpipe<stale,adam>"
+    assert bench.kernel_name("auto", "adam", 5, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "sgd", 6, 1) == "colocated_wide<stale>"
     assert bench.kernel_name("auto", "sgd", 12, 1) == "colocated_wide<stale>"
     args = argparse.Namespace(optimizer="sgd", variant="auto", staleness=1)
     assert bench.colocated_launches(4, 4, args, True) == 1
-    assert bench.colocated_launches(8, 4, args, True) == 1
+    assert bench.colocated_launches(5, 4, args, True) == 1
+    assert bench.colocated_launches(8, 4, args, True) == 4
     assert bench.colocated_launches(12, 4, args, True) == 4
     monkeypatch.setenv("AVGPIPE_EA_FORCE_WIDE", "1")
     assert bench.kernel_name("auto", "sgd", 4, 1) == "colocated_wide<stale>"

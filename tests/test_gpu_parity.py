@@ -220,6 +220,21 @@ def test_stale_center_replica_loop_knob():
     assert r.returncode == 0 and "knob ok" in r.stdout, r.stdout[-3000:] + r.stderr[-3000:]
 
 
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+@pytest.mark.parametrize("n", [1, 3, 5, 6, 7, 8])
+def test_split_register_loop(n, optimizer):
+    """Variant 4 (two lanes per center column, N/2 replicas each, shuffle reduction): C1-sized stages + ragged
+    ones in one launch, every optimizer."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 12, "combined", variants=("split",), many=True,
+                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+
+
+def test_split_register_loop_c1_100_steps():
+    _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("split",), many=True, optimizer="adam",
+                   lr=1e-3, wd=1e-2)
+
+
 @pytest.mark.parametrize("n,optimizer", [(33, "sgd"), (64, "sgd"), (64, "adamw")])
 def test_maximum_replica_count(n, optimizer):
     """EA_MAX_REPLICAS = 64 co-located replicas (the replica-loop kernel's pointer table)."""
