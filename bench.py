@@ -220,10 +220,11 @@ def kernel_name(variant, optimizer, n, staleness=0):
         name = "colocated_wide"
     elif two_state:
         if variant == "auto":
-            variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else "bulkpipe")
+            variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else ("bulkpipe" if n == 4 else "split"))
         name = "colocated_" + variant
     elif variant == "auto":
-        name = ("colocated_bulkpipe" if n in (1, 5, 6, 7) else
+        name = ("colocated_split" if optimizer == "asgd" and n in (5, 6) else
+                "colocated_bulkpipe" if n in (1, 5, 6, 7) else
                 "colocated_laneshfl" if n <= 4 else "colocated_regloop")
     else:
         name = "colocated_" + variant
@@ -442,6 +443,14 @@ def run_ours(args, rank, world, local):
             out["roofline"] = local     # no NVLink traffic at world 1: the local kernel is the bound
             local["note"] = ("world 1: each stage's local kernel is timed while the previous stage's exchange "
                              "(side stream) shares HBM")
+            # world 1 the exchange is local HBM work too: NCCL's reduce-scatter is a copy (8 B), the shard update
+            # 12 B, the in-place all-gather nothing; p2p phase B 16 B; the stale snapshot + 8 B per element
+            xb = (20 if args.exchange == "nccl" else 16) + 8 * args.staleness
+            sb = step_bytes + sum(xb * h.center_capacity(s) for s in range(len(sizes)))
+            out["step_hbm"] = {"bytes_per_step": sb, "achieved": sb / (ms * 1e-3) / 1e9, "peak": peak,
+                               "frac": sb / (ms * 1e-3) / 1e9 / peak, "unit": "GB/s",
+                               "note": f"whole step at world 1: local kernels 28 B + exchange {xb} B per element, "
+                                       "both streams sharing HBM"}
         else:
             out["roofline"] = nvlink
             out["local_kernel_roofline"] = local

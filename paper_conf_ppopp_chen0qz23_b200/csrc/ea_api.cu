@@ -403,17 +403,21 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
 }
 
 // Row a8 knobs (measurement).  The exchange runs on the library's side stream beside the caller's
-// compute, so its own kernels take few SMs: AVGPIPE_EA_SIDE_CTAS (default num_sms/4) caps spread_apply's grid.
-// The local kernels of the spread layout run on the caller's stream with persistent grids that would hold every
-// SM for their whole duration and keep the previous stage's side-stream exchange (NCCL's kernels, or
-// p2p_exchange) from being scheduled at all: AVGPIPE_EA_SPREAD_RESERVE_SMS SMs are left free for it.
-int side_ctas(int num_sms) {
+// compute.  At world > 1 its own kernel (the shard update, P_pad/N elements) is small and takes few SMs:
+// AVGPIPE_EA_SIDE_CTAS (default num_sms/4; 0 = the persistent grid) caps spread_apply's grid.  At world 1 the
+// "exchange" is the whole center (12 B per element of local HBM traffic, as much as half the local step) and
+// the cap only stretches it out under the compute (C5 harness: EA alone 29 ms capped vs 11 ms), so it is not
+// capped.  The local kernels of the spread layout run on the caller's stream with persistent grids that hold
+// every SM for their whole duration: AVGPIPE_EA_SPREAD_RESERVE_SMS SMs can be left free for the side stream
+// (default 0: measured no gain, profiles/r02_a8_trace.md).
+int side_ctas(const ea_ctx* h) {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_SIDE_CTAS");
-    return e ? std::atoi(e) : 0;
+    return e ? std::atoi(e) : -1;
   }();
-  if (v > 0) return v;
-  return num_sms / 4 > 0 ? num_sms / 4 : 1;
+  if (v >= 0) return v;  // 0: no cap
+  if (h->cfg.world <= 1) return 0;
+  return h->num_sms / 4 > 0 ? h->num_sms / 4 : 1;
 }
 
 int spread_local_sms(int num_sms) {
@@ -469,7 +473,7 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
   ncclResult_t r = ncclReduceScatter(contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
                                      h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
-  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, side_ctas(h->num_sms), h->side);
+  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, side_ctas(h), h->side);
   if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
   r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
   if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
@@ -598,7 +602,9 @@ int p2p_exchange_ctas(const ea_ctx* h) {
   const long long v = e ? std::atoll(e) : 0;
   if (v >= 1 && v <= 4096) return static_cast<int>(v);
   const int ranks = h->same_device_ranks > 0 ? h->same_device_ranks : 1;
-  const int k = ranks > 1 ? h->num_sms / ranks : h->num_sms / 3;
+  int k = h->num_sms / 3;
+  if (ranks > 1) k = h->num_sms / ranks;
+  else if (h->cfg.world <= 1) k = 2 * h->num_sms;  // world 1: phase B over the whole center, local HBM work
   return k > 0 ? k : 1;
 }
 

@@ -1083,10 +1083,13 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // SGD: the bulk-copy pipeline for N = 1, 5, 6, 7 (0.88-0.96 / 0.95 / 0.96 / 0.955 of peak), the lane kernel
   // for N = 2..4 (0.96 / 0.93 / 0.97-0.99; a warp holds >= 8 lanes per replica row), the register loop for
   // N = 8 (0.98-0.99).  Adam(W): the lane kernel for N = 1 (0.915), the register loop for N = 2, 3 (0.96 /
-  // 0.95; bulk pipeline 0.88 / 0.90), the bulk-copy pipeline for N = 4..6 (0.97 / 0.95 / 0.93); N > 6 goes to
-  // the replica-loop kernel (ea_api.cu)
+  // 0.95; bulk pipeline 0.88 / 0.90), the bulk-copy pipeline for N = 4 (0.97), the split register loop for
+  // N = 5, 6 (round 2, same box: 0.950 / 0.930 vs 0.930 / 0.906 for the bulk pipeline); N > 6 goes to the
+  // replica-loop kernel (ea_api.cu).  ASGD: SGD's choice except the split register loop for N = 5, 6 (0.967 /
+  // 0.941 vs 0.920 / 0.937; profiles/r02_sweep_split.jsonl -- with SGD it measured below the bulk pipeline).
   if (variant == kVariantAuto && two_state(opt))
-    variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : kVariantBulkPipe);
+    variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : (n == 4 ? kVariantBulkPipe : kVariantSplit));
+  if (variant == kVariantAuto && opt == kOptASGD && (n == 5 || n == 6)) variant = kVariantSplit;
   if (variant == kVariantAuto)
     variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
   switch (n) {

@@ -272,7 +272,9 @@ __global__ void __launch_bounds__(kPushThreads, 1) p2p_push_bulk(const P2PArgs a
           }
           st4(dst + 4 * (v - e4), rv);  // peer store into the owner's inbox
         }
-        // all consumer warps are done with the slot (and, at a chunk's end, have issued all its stores)
+        // all consumer warps are done with the slot (and, at a chunk's end, have issued all its stores).  (Moving the
+        // chunk's release-add to the producer warp, off the consumers' path, measured slower on B200: 265 vs 232 us
+        // per C4 stage -- the producer's system-scope release then waits behind its own bulk copies in flight.)
         asm volatile("bar.sync 1, %0;" ::"n"(32 * kPushConsumerWarps) : "memory");
         if (threadIdx.x == 0) {
           mbar_arrive(&empty[slot]);
