@@ -389,6 +389,7 @@ def run_ours(args, rank, world, local):
                      "nccl_env": {k: v for k, v in os.environ.items() if k.startswith("NCCL_")} if spread else None,
                      "optimizer": "sgd-momentum(0.9)" if args.optimizer == "sgd" else args.optimizer,
                      "kernel": args.variant,
+                     "knobs": {k: v for k, v in os.environ.items() if k.startswith("AVGPIPE_EA_")} or None,
                      "l2": f"no flush: working set {ws_bytes / 1e9:.2f} GB per GPU > 126 MB L2"}
     if not spread:
         step_bytes = sum(bytes_colocated(n, p, args.optimizer) + 8 * p * args.staleness for p in sizes)

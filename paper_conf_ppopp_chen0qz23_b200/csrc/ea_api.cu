@@ -420,6 +420,16 @@ int side_ctas(const ea_ctx* h) {
   return h->num_sms / 4 > 0 ? h->num_sms / 4 : 1;
 }
 
+// Pieces per stage of the NCCL spread step (knob AVGPIPE_EA_SPREAD_CHUNKS, 1..64; default 1 = the whole stage).
+int spread_chunks() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_SPREAD_CHUNKS");
+    const int k = e ? std::atoi(e) : 1;
+    return k >= 1 && k <= 64 ? k : 1;
+  }();
+  return v;
+}
+
 int spread_local_sms(int num_sms) {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_SPREAD_RESERVE_SMS");
@@ -440,8 +450,7 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
   }
   cudaError_t e;
   const int n = h->cfg.n_pipelines;
-  const int64_t pad = h->p_pad[stage], shard = pad / n;
-  float* own = center_ptr + shard * h->cfg.rank;
+  const int64_t pad = h->p_pad[stage];
   float* contrib = h->contrib + h->contrib_off[stage];
   const bool stale = h->cfg.staleness == 1;
   // Local phase on the CALLER's stream (x_i, state and r_i ready there, in stream order).  Synchronous center:
@@ -456,27 +465,43 @@ ea_status spread_step(ea_ctx* h, int32_t stage, float* replica, const float* gra
     return cuda_fail(h, e, "cudaStreamWaitEvent");
   ea_status st2 = advance(h, &stage, 1, s);
   if (st2 != EA_OK) return st2;
-  e = ea::launch_spread_local(replica, grad, state_ptr(h, 0, stage, 0), state_ptr(h, 1, stage, 0),
-                              stale ? h->prev[stage] : center_ptr, contrib, h->p[stage], pad, h->hp,
-                              h->cfg.optimizer, h->d_coef + stage, spread_local_sms(h->num_sms), s);
-  if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
-  if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
-  // Exchange on the side stream: reduce-scatter -> owner-shard update -> in-place all-gather.  The caller's
-  // stream does not wait for it; the next local step of this stage (or ea_sync) does.
-  if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
-    return cuda_fail(h, e, "cudaStreamWaitEvent");
-  if (stale) {  // prev <- x~_t (final: the previous all-gather precedes this on the side stream)
-    e = cudaMemcpyAsync(h->prev[stage], center_ptr, sizeof(float) * h->p[stage], cudaMemcpyDeviceToDevice, h->side);
-    if (e != cudaSuccess) return cuda_fail(h, e, "stale-center snapshot");
-    if ((e = cudaEventRecord(h->ev_snap[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+  // Intra-stage pipelining (knob AVGPIPE_EA_SPREAD_CHUNKS = C, default 1; synchronous center only): the stage is
+  // cut into C pieces of whole 32N-float blocks; the local kernel of piece k runs on the caller's stream while
+  // piece k-1's reduce-scatter / shard update / all-gather run on the side stream.  Within piece k rank r owns
+  // block r of its N equal blocks (so the reduce-scatter and the in-place all-gather of a piece are plain NCCL
+  // calls on the piece).
+  const int chunks = stale ? 1 : spread_chunks();
+  const int64_t L = round_up((pad + chunks - 1) / chunks, 32LL * n);
+  float* m0 = state_ptr(h, 0, stage, 0);
+  float* v0 = state_ptr(h, 1, stage, 0);
+  const float* cread = stale ? h->prev[stage] : center_ptr;
+  const int64_t p = h->p[stage];
+  for (int64_t off = 0; off < pad; off += L) {
+    const int64_t len = pad - off < L ? pad - off : L, cnt = len / n;
+    const int64_t pk = p - off <= 0 ? 0 : (p - off < len ? p - off : len);  // replica elements in this piece
+    e = ea::launch_spread_local(replica + (pk ? off : 0), grad + (pk ? off : 0), m0 + (pk ? off : 0),
+                                v0 ? v0 + (pk ? off : 0) : nullptr, cread + (pk ? off : 0), contrib + off, pk, len,
+                                h->hp, h->cfg.optimizer, h->d_coef + stage, spread_local_sms(h->num_sms), s);
+    if (e != cudaSuccess) return cuda_fail(h, e, "spread local kernel launch");
+    if ((e = cudaEventRecord(h->ev_loc[stage], s)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+    // Exchange on the side stream: reduce-scatter -> owner-shard update -> in-place all-gather.  The caller's
+    // stream does not wait for it; the next local step of this stage (or ea_sync) does.
+    if ((e = cudaStreamWaitEvent(h->side, h->ev_loc[stage], 0)) != cudaSuccess)
+      return cuda_fail(h, e, "cudaStreamWaitEvent");
+    if (stale) {  // prev <- x~_t (final: the previous all-gather precedes this on the side stream)
+      e = cudaMemcpyAsync(h->prev[stage], center_ptr, sizeof(float) * p, cudaMemcpyDeviceToDevice, h->side);
+      if (e != cudaSuccess) return cuda_fail(h, e, "stale-center snapshot");
+      if ((e = cudaEventRecord(h->ev_snap[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
+    }
+    float* own = center_ptr + off + cnt * h->cfg.rank;
+    ncclResult_t r = ncclReduceScatter(contrib + off, h->reduced, static_cast<size_t>(cnt), ncclFloat, ncclSum,
+                                       h->comm, h->side);
+    if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
+    e = ea::launch_spread_apply(own, h->reduced, cnt, h->hp.inv_n, h->num_sms, side_ctas(h), h->side);
+    if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
+    r = ncclAllGather(own, center_ptr + off, static_cast<size_t>(cnt), ncclFloat, h->comm, h->side);
+    if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
   }
-  ncclResult_t r = ncclReduceScatter(contrib, h->reduced, static_cast<size_t>(shard), ncclFloat, ncclSum, h->comm,
-                                     h->side);
-  if (r != ncclSuccess) return nccl_fail(h, r, "ncclReduceScatter");
-  e = ea::launch_spread_apply(own, h->reduced, shard, h->hp.inv_n, h->num_sms, side_ctas(h), h->side);
-  if (e != cudaSuccess) return cuda_fail(h, e, "spread apply kernel launch");
-  r = ncclAllGather(own, center_ptr, static_cast<size_t>(shard), ncclFloat, h->comm, h->side);
-  if (r != ncclSuccess) return nccl_fail(h, r, "ncclAllGather");
   if ((e = cudaEventRecord(h->ev_ag[stage], h->side)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
   return EA_OK;
 }

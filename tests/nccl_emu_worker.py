@@ -139,20 +139,33 @@ def main():
             op, rank, world, send, recv, count, dtype = line.split()
             if op in ("RS", "AG") and int(world) == n:
                 per_rank[int(rank)].append((op, int(send, 16), int(recv, 16), int(count)))
+        chunks = 1 if args.staleness else int(os.environ.get("AVGPIPE_EA_SPREAD_CHUNKS", "1") or 1)
+
+        def pieces(p_pad):
+            """The library's cut of a stage into pieces of whole 32N-float blocks (ea_api.cu spread_step)."""
+            q = 32 * n
+            L = (-(-p_pad // chunks) + q - 1) // q * q
+            return [(off, min(L, p_pad - off)) for off in range(0, p_pad, L)]
+
         for r in range(n):
             h = handles[r]
             seq = per_rank[r]
-            want = [(kind, s) for _ in range(args.steps) for s in order for kind in ("RS", "AG")]
+            want = [(kind, s, off, ln) for _ in range(args.steps) for s in order
+                    for off, ln in pieces(h.center_capacity(s)) for kind in ("RS", "AG")]
             if len(seq) != len(want):
                 checks["bad"].append(f"rank {r}: {len(seq)} calls, expected {len(want)}")
                 continue
-            for (op, send, recv, count), (kind, s) in zip(seq, want):
+            for (op, send, recv, count), (kind, s, off, ln) in zip(seq, want):
                 p_pad = h.center_capacity(s)
-                lo, hi = parallel.shard_bounds(p_pad, n, r)
-                ok = op == kind and count == hi - lo == h.shard_elems(s)
+                if chunks == 1:
+                    lo, hi = parallel.shard_bounds(p_pad, n, r)
+                    ok = op == kind and count == hi - lo == h.shard_elems(s)
+                else:     # piece [off, off + ln): rank r owns its block r
+                    lo, hi = off + r * (ln // n), off + (r + 1) * (ln // n)
+                    ok = op == kind and count == ln // n
                 center = cs[r][s].data_ptr()
                 if kind == "AG":
-                    ok = ok and recv == center and send == center + 4 * lo     # in place, own shard
+                    ok = ok and recv == center + 4 * off and send == center + 4 * lo     # in place, own block
                     checks["ag"] += 1
                 else:
                     ok = ok and recv != center and send != center          # library scratch
@@ -163,6 +176,7 @@ def main():
     for h in handles:
         h.close()
     print(json.dumps({"world": n, "optimizer": opt, "staleness": args.staleness, "steps": args.steps,
+                      "chunks": int(os.environ.get("AVGPIPE_EA_SPREAD_CHUNKS", "1") or 1),
                       "max_err": max(worst.values()), "worst": worst, "padding_zero": pad_ok,
                       "collectives": checks}))
 

@@ -29,11 +29,11 @@ def _emu_lib():
     return build_nccl_emu()
 
 
-def run_emu(world, *extra, timeout=900):
+def run_emu(world, *extra, timeout=900, env_extra=None):
     lib = _emu_lib()
     with tempfile.TemporaryDirectory() as d:
         log = os.path.join(d, "calls.log")
-        env = dict(os.environ, LD_PRELOAD=lib, NCCL_EMU_LOG=log, NCCL_EMU_TIMEOUT_S="300")
+        env = dict(os.environ, LD_PRELOAD=lib, NCCL_EMU_LOG=log, NCCL_EMU_TIMEOUT_S="300", **(env_extra or {}))
         out = subprocess.run([sys.executable, os.path.join(ROOT, "tests", "nccl_emu_worker.py"), "--world",
                               str(world), *extra], capture_output=True, text=True, timeout=timeout, env=env, cwd=ROOT)
     lines = [ln for ln in out.stdout.splitlines() if ln.startswith("{")]
@@ -41,13 +41,13 @@ def run_emu(world, *extra, timeout=900):
     return json.loads(lines[-1])
 
 
-def _check(d, steps=100, stages=2):
+def _check(d, steps=100, stages=2, pieces=1):
     assert "error" not in d, d
     assert d["max_err"] <= 1e-5, d
     assert d["padding_zero"], d
     c = d["collectives"]
     assert not c["bad"], c
-    assert c["rs"] == c["ag"] == d["world"] * steps * stages, c
+    assert c["rs"] == c["ag"] == d["world"] * steps * stages * pieces, c
 
 
 @pytest.mark.parametrize("world", [2, 4, 8])
@@ -72,3 +72,12 @@ def test_stale_center_spread_world_n(world, optimizer):
     exchange took) while that exchange is still in flight (reading c28), against the stale oracle."""
     steps = 100 if optimizer == "sgd" else 30
     _check(run_emu(world, "--staleness", "1", "--optimizer", optimizer, "--steps", str(steps)), steps=steps)
+
+
+@pytest.mark.parametrize("world,chunks", [(2, 3), (4, 5), (8, 2)])
+def test_intra_stage_pipelining(world, chunks):
+    """AVGPIPE_EA_SPREAD_CHUNKS: each stage cut into pieces whose local kernel runs while the previous piece's
+    reduce-scatter / shard update / all-gather run on the side stream; every piece's calls
+    checked (rank r owns block r of each piece), parity after 60 steps."""
+    d = run_emu(world, "--steps", "60", env_extra={"AVGPIPE_EA_SPREAD_CHUNKS": str(chunks)})
+    _check(d, steps=60, pieces=chunks)

@@ -11,7 +11,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 FLOORS = {
     "test_gpu_parity.py": 226,
     "test_gpu_p2p.py": 27,
-    "test_gpu_nccl_emu.py": 14,
+    "test_gpu_nccl_emu.py": 17,
     "test_gpu_state.py": 7,
     "test_gpu_fullsize.py": 17,
     "test_gpu_bench.py": 5,
@@ -19,7 +19,7 @@ FLOORS = {
     "test_gpu_pipeline.py": 3,
     "test_gpu_fuzz.py": 120,
 }
-TOTAL_FLOOR = 424
+TOTAL_FLOOR = 427
 
 
 def test_gpu_suite_size():
