@@ -93,13 +93,15 @@ int64_t host_chunk() {
   return v;
 }
 
-// Floats per exchange chunk of the fused peer-memory spread kernel (default 8192 = 32 KB).
-// Measurement knob AVGPIPE_EA_P2P_CHUNK (a multiple of 1024 floats, 1024..65536); every rank of an
-// exchange must use the same value (it fixes the layout of the peers' inboxes).
+// Floats per exchange chunk of the peer-memory spread step (default 32768 = 128 KB: one system-scope release per
+// chunk; B200, C4 stage, round 2: 8192 / 16384 / 32768 -> push kernel 0.45 / 0.50 / 0.54 of HBM peak beside the
+// exchange at world 1, 8 virtual ranks 0.99 / - / 1.08, profiles/r02_p2p_chunks_split_grid.jsonl; round 1's fused
+// kernel preferred 8192).  Measurement knob AVGPIPE_EA_P2P_CHUNK (a multiple of 1024 floats, 1024..65536); every
+// rank of an exchange must use the same value (it fixes the layout of the peers' inboxes).
 int64_t p2p_chunk() {
   const char* e = std::getenv("AVGPIPE_EA_P2P_CHUNK");
   const long long v = e ? std::atoll(e) : 0;
-  return (v >= 1024 && v <= 65536 && v % 1024 == 0) ? v : 8192;
+  return (v >= 1024 && v <= 65536 && v % 1024 == 0) ? v : 32768;
 }
 
 namespace {

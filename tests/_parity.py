@@ -57,11 +57,14 @@ def hyper(n, mode, alpha=None, lr=synth.LR, momentum=synth.MOMENTUM, wd=0.0, nes
     """Oracle hyper-parameters equal to what the ABI carries (reading c12: the
     oracle consumes the same fp32 values upcast): alpha, beta, rho, lr,
     momentum, weight_decay, eps are float32 fields; beta1/beta2 and the ASGD
-    fields are double.  The rounding is small -- float32(0.01) is 2.2e-8
-    relative below 0.01, float32(1e-3) 4.7e-8 above, float32(0.9) 2.6e-8 below
-    -- and over 100 steps it moves x by ~1e-7 of rms(x) (lr enters Delta
-    linearly; momentum amplifies by 1/(1-mu)), two orders under the 1e-5 gate;
-    the measured effect per test is in profiles/r02_parity_margins*.jsonl."""
+    fields are double.  float32(0.01) is 2.2e-8 relative below 0.01,
+    float32(1e-3) 4.7e-8 above, float32(0.9) 2.6e-8 below.  Mostly harmless
+    (lr enters Delta linearly: ~1e-7 of rms(x) after 100 steps), except for
+    Adam with L2 decay where g' = g + lambda*x nearly cancels (|g'| <~ eps):
+    there Delta has slope lr/eps = 1e5 in g', and the 4.5e-12 the rounding of
+    lambda moves lambda*x becomes ~2e-5 of rms(x) -- measured: the C2 full-size
+    Adam test fails its first step with unrounded values
+    (profiles/r02_parity_margins.md)."""
     a, b, r = synth.mode_coeffs(mode, n, alpha)
     return Hyper(alpha=f32(a), beta=f32(b), rho=f32(r), lr=f32(lr), momentum=f32(momentum), weight_decay=f32(wd),
                  nesterov=nesterov, beta1=betas[0], beta2=betas[1], eps=f32(eps), **asgd)
