@@ -122,7 +122,8 @@ typedef struct {
                                    warp-shuffle reduction, 3 = bulk-copy pipeline (every input
                                    tile by cp.async.bulk into an mbarrier ring), 4 = split
                                    register loop (two lanes per center column, N/2 replicas
-                                   each, shuffle reduction).  Same results up to fp32 summation
+                                   each, shuffle reduction), 5 = warp per replica (contributions
+                                   reduced through shared memory).  Same results up to fp32 summation
                                    order (DESIGN.md c14); the default picks per N and optimizer
                                    (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */

@@ -98,6 +98,7 @@ enum KernelVariant : int {
   kVariantBulkPipe = 3,  // every input tile streamed by cp.async.bulk into a multi-stage smem
                          // ring (producer warp + mbarriers); consumers store from registers (SGD)
   kVariantSplit = 4,     // split register loop: 2 lanes per center column, N/2 replicas each, shuffle reduction
+  kVariantWarpRep = 5,   // warp per replica, 512 B rows, contributions reduced through shared memory
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N

@@ -295,6 +295,82 @@ __global__ void __launch_bounds__(kThreads, 2) colocated_split(const StageBatch 
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
 }
 
+// ============================================================================
+// Variant 5: warp per replica.  A CTA of 32N threads; warp i streams replica i of a tile of 32U float4 columns
+// (full 512 B rows per load instruction -- the lane kernel's rows shrink to 64 B at N = 8), keeps its U float4 of
+// x, g and the optimizer state in registers, and writes its contribution r_i to shared memory; after a block
+// barrier the N contributions of each column are summed and x~ updated.  The center is read by every warp through
+// the read-only path (one DRAM read, the other warps hit L1/L2).
+// ============================================================================
+template <int N, int OPT, int U>
+__global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(const StageBatch b, const Hyper hp) {
+  constexpr int TV = 32 * U;  // float4 columns per tile
+  constexpr bool kTwo = two_state(OPT);
+  __shared__ __align__(16) float4 s_r[N][TV];
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
+  const Mem<0> mem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  if (has_coef(OPT)) {
+    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+    __syncthreads();
+  }
+  WaveCursor cur{0, 0};
+  int s;
+  int64_t v0, nv;
+  while (wave_item(b, TV, cur, s, v0, nv)) {
+    const StageRefs& st = b.st[s];
+    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
+    float* xi = nullptr;
+    const float* gi = nullptr;
+    float* mi = nullptr;
+    float* vi = nullptr;
+#pragma unroll
+    for (int i = 0; i < N; ++i)
+      if (warp == i) {
+        xi = st.x[i];
+        gi = st.g[i];
+        mi = st.m[i];
+        if (kTwo) vi = st.v[i];
+      }
+    float4 x[U], g[U], m[U], w[U], c[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int lv = u * 32 + lane;
+      if (lv < nv) {
+        const int64_t v = v0 + lv;
+        x[u] = mem.ld(xi + 4 * v);
+        g[u] = mem.ld_ro(gi + 4 * v);
+        m[u] = mem.ld(mi + 4 * v);
+        if (kTwo) w[u] = mem.ld(vi + 4 * v);
+        c[u] = __ldg(reinterpret_cast<const float4*>(st.c) + v);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int lv = u * 32 + lane;
+      if (lv < nv) {
+        const int64_t v = v0 + lv;
+        s_r[warp][lv] = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
+        mem.st(xi + 4 * v, x[u]);
+        mem.st(mi + 4 * v, m[u]);
+        if (kTwo) mem.st(vi + 4 * v, w[u]);
+      }
+    }
+    __syncthreads();
+    for (int col = threadIdx.x; col < nv; col += 32 * N) {
+      float4 acc = s_r[0][col];
+#pragma unroll
+      for (int i = 1; i < N; ++i) add4(acc, s_r[i][col]);
+      const int64_t v = v0 + col;
+      const float4 cv = __ldg(reinterpret_cast<const float4*>(st.c) + v);
+      mem.st(st.c + 4 * v, center_apply(cv, acc, hp.inv_n));
+    }
+    __syncthreads();  // s_r is refilled by the next tile
+  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+}
+
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -950,8 +1026,26 @@ cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cuda
   return cudaGetLastError();
 }
 
+// Warp per replica (variant 5): U float4 columns per lane and tile (SGD/ASGD 4: 2 KB rows per stream per tile;
+// Adam(W) 2, for registers).
+template <int N, int OPT>
+cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  constexpr int U = two_state(OPT) ? 2 : 4;
+  auto k = colocated_warprep<N, OPT, U>;
+  k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
+  return cudaGetLastError();
+}
+
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (variant == kVariantWarpRep) {
+    switch (opt) {
+      case kOptAdam: return launch_warprep<N, kOptAdam>(b, hp, num_sms, s);
+      case kOptAdamW: return launch_warprep<N, kOptAdamW>(b, hp, num_sms, s);
+      case kOptASGD: return launch_warprep<N, kOptASGD>(b, hp, num_sms, s);
+      default: return launch_warprep<N, kOptSGD>(b, hp, num_sms, s);
+    }
+  }
   if (variant == kVariantSplit) {
     switch (opt) {
       case kOptAdam: return launch_split<N, kOptAdam>(b, hp, num_sms, s);
@@ -1002,12 +1096,11 @@ int spread_reg() {
   return v;
 }
 
-template <int OPT>
-cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
-                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
-                               cudaStream_t s) {
+template <int OPT, int TILE>
+cudaError_t launch_spread_bulk_t(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                                 int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
+                                 cudaStream_t s) {
   constexpr int A = two_state(OPT) ? 4 : 3;
-  constexpr int TILE = default_bulk_tile<1, A>();
   using G = BulkGeom<1, TILE, A>;
   auto k = spread_bulkpipe<OPT, TILE>;
   cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, G::kSmemBytes);
@@ -1029,6 +1122,19 @@ cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, con
   if (grid > units) grid = units < 1 ? 1 : units;
   k<<<static_cast<int>(grid), kBulkThreads, G::kSmemBytes, s>>>(b, hp, contrib, p_pad, bulk_issue_lanes());
   return cudaGetLastError();
+}
+
+// Spread local kernel tile (measurement knob AVGPIPE_EA_BULK_TILE = 128 | 256 | 512 float4 per stream copy;
+// default 256, i.e. 4 KB copies).
+template <int OPT>
+cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
+                               cudaStream_t s) {
+  switch (bulk_tile()) {
+    case 128: return launch_spread_bulk_t<OPT, 128>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+    case 512: return launch_spread_bulk_t<OPT, 512>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+    default: return launch_spread_bulk_t<OPT, 256>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
+  }
 }
 
 template <int OPT>

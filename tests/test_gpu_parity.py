@@ -230,6 +230,21 @@ def test_split_register_loop(n, optimizer):
                    optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
 
 
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+@pytest.mark.parametrize("n", [1, 2, 5, 6, 7, 8])
+def test_warp_per_replica(n, optimizer):
+    """Variant 5 (warp per replica, contributions reduced through shared memory): C1-sized and ragged stages in
+    one launch, every optimizer."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 12, "combined", variants=("warprep",), many=True,
+                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+
+
+def test_warp_per_replica_c1_100_steps():
+    _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warprep",), many=True, optimizer="adam",
+                   lr=1e-3, wd=1e-2)
+
+
 def test_split_register_loop_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("split",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
