@@ -202,7 +202,8 @@ def workload_key(gpus: int, override):
 def stale_fused(n, optimizer, variant):
     """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1; N = 5 for
     SGD/ASGD) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
-    return variant == "auto" and (n <= 4 or (n == 5 and optimizer not in ("adam", "adamw")))
+    return ((variant == "auto" and (n <= 4 or (n == 5 and optimizer not in ("adam", "adamw"))))
+            or (variant == "warprep" and n <= 8))
 
 
 def kernel_name(variant, optimizer, n, staleness=0):
@@ -212,7 +213,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
         return "colocated_wide" + ("<stale>" if staleness else "")
     if staleness:
         if stale_fused(n, optimizer, variant):   # ea_api.cu: x~_{t-1} staged beside x~_t, <= 8 stages per launch
-            kern = "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe"
+            kern = ("colocated_warprep" if variant == "warprep" else
+                    "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe")
             return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"
     two_state = optimizer in ("adam", "adamw")

@@ -326,7 +326,9 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // else the replica loop, one launch per stage, which measured better from N = 6 on (N = 8: 0.954 vs 0.903;
   // Adam N = 6: 0.925 vs 0.775 of HBM peak, profiles/r02_sweep_kernels.jsonl).  AVGPIPE_EA_FORCE_WIDE=1 selects
   // the replica loop for A/B measurement.
-  const bool stale_lane = stale && (n <= 4 || (n == 5 && !ea::two_state(opt))) && h->variant == 0 && !force_wide;
+  const bool stale_lane = stale && !force_wide &&
+                          ((h->variant == 0 && (n <= 4 || (n == 5 && !ea::two_state(opt)))) ||
+                           (h->variant == ea::kVariantWarpRep && n <= ea::kMaxFusedN));
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
     for (int j = 0; j < count; ++j) {
       ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);
@@ -355,7 +357,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
         r.scp = h->d_coef + st;
         r.prev = h->prev[st];
       }
-      e = ea::launch_colocated_batch_stale(b, n, h->hp, opt, h->num_sms, s);
+      e = ea::launch_colocated_batch_stale(b, n, h->hp, opt, h->variant, h->num_sms, s);
       if (e != cudaSuccess) return cuda_fail(h, e, "co-located stale kernel launch");
     }
     return EA_OK;

@@ -302,7 +302,9 @@ __global__ void __launch_bounds__(kThreads, 2) colocated_split(const StageBatch 
 // barrier the N contributions of each column are summed and x~ updated.  The center is read by every warp through
 // the read-only path (one DRAM read, the other warps hit L1/L2).
 // ============================================================================
-template <int N, int OPT, int U>
+// STALE (row f4, reading c28): the replicas read x~_{t-1} (st.prev) instead of x~_t; the reduction writes
+// x~_{t+1} = x~_t + R/N and prev <- x~_t.
+template <int N, int OPT, int U, bool STALE = false>
 __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(const StageBatch b, const Hyper hp) {
   constexpr int TV = 32 * U;  // float4 columns per tile
   constexpr bool kTwo = two_state(OPT);
@@ -342,7 +344,7 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
         g[u] = mem.ld_ro(gi + 4 * v);
         m[u] = mem.ld(mi + 4 * v);
         if (kTwo) w[u] = mem.ld(vi + 4 * v);
-        c[u] = __ldg(reinterpret_cast<const float4*>(st.c) + v);
+        c[u] = __ldg(reinterpret_cast<const float4*>(STALE ? st.prev : st.c) + v);  // the center the replicas see
       }
     }
 #pragma unroll
@@ -364,11 +366,12 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
       const int64_t v = v0 + col;
       const float4 cv = __ldg(reinterpret_cast<const float4*>(st.c) + v);
       mem.st(st.c + 4 * v, center_apply(cv, acc, hp.inv_n));
+      if (STALE) mem.st(st.prev + 4 * v, cv);
     }
     __syncthreads();  // s_r is refilled by the next tile
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
 template <int U>
@@ -1028,10 +1031,10 @@ cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cuda
 
 // Warp per replica (variant 5): U float4 columns per lane and tile (SGD/ASGD 4: 2 KB rows per stream per tile;
 // Adam(W) 2, for registers).
-template <int N, int OPT>
+template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   constexpr int U = two_state(OPT) ? 2 : 4;
-  auto k = colocated_warprep<N, OPT, U>;
+  auto k = colocated_warprep<N, OPT, U, STALE>;
   k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
@@ -1235,11 +1238,34 @@ cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int nu
   }
 }
 
-cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int num_sms,
-                                         cudaStream_t s) {
+template <int N>
+cudaError_t launch_stale_warprep_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
+  switch (opt) {
+    case kOptAdam: return launch_warprep<N, kOptAdam, true>(b, hp, num_sms, s);
+    case kOptAdamW: return launch_warprep<N, kOptAdamW, true>(b, hp, num_sms, s);
+    case kOptASGD: return launch_warprep<N, kOptASGD, true>(b, hp, num_sms, s);
+    default: return launch_warprep<N, kOptSGD, true>(b, hp, num_sms, s);
+  }
+}
+
+cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int variant,
+                                         int num_sms, cudaStream_t s) {
   if (b.nstages <= 0) return cudaSuccess;
   for (int t = 0; t < b.nstages; ++t)
     if (!b.st[t].prev) return cudaErrorInvalidValue;
+  if (variant == kVariantWarpRep) {
+    switch (n) {
+      case 1: return launch_stale_warprep_n<1>(b, hp, opt, num_sms, s);
+      case 2: return launch_stale_warprep_n<2>(b, hp, opt, num_sms, s);
+      case 3: return launch_stale_warprep_n<3>(b, hp, opt, num_sms, s);
+      case 4: return launch_stale_warprep_n<4>(b, hp, opt, num_sms, s);
+      case 5: return launch_stale_warprep_n<5>(b, hp, opt, num_sms, s);
+      case 6: return launch_stale_warprep_n<6>(b, hp, opt, num_sms, s);
+      case 7: return launch_stale_warprep_n<7>(b, hp, opt, num_sms, s);
+      case 8: return launch_stale_warprep_n<8>(b, hp, opt, num_sms, s);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   switch (n) {
     case 1: return launch_stale_bulk_n<1>(b, hp, opt, num_sms, s);
     case 2: return launch_stale_n<2>(b, hp, opt, num_sms, s);

@@ -240,6 +240,16 @@ def test_warp_per_replica(n, optimizer):
                    optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
 
 
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "asgd"])
+@pytest.mark.parametrize("n", [1, 3, 4, 6, 8])
+def test_warp_per_replica_stale(n, optimizer):
+    """Variant 5 with the stale center (row f4): the replicas read x~_{t-1}, the reduction writes x~_{t+1} and
+    rolls x~_{t-1} <- x~_t; several stages per launch."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096], 20, "combined", variants=("warprep",), many=True, optimizer=optimizer,
+                   lr=lr, staleness=1)
+
+
 def test_warp_per_replica_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warprep",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
