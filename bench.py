@@ -213,7 +213,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
         return "colocated_wide" + ("<stale>" if staleness else "")
     if staleness:
         if stale_fused(n, optimizer, variant):   # ea_api.cu: x~_{t-1} staged beside x~_t, <= 8 stages per launch
-            kern = ("colocated_warprep" if variant == "warprep" else
+            two = optimizer in ("adam", "adamw")
+            kern = ("colocated_warprep" if variant == "warprep" or (not two and n in (2, 5)) else
                     "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe")
             return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"
@@ -224,10 +225,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
         if variant == "auto":
             variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else ("bulkpipe" if n == 4 else "split"))
         name = "colocated_" + variant
-    elif variant == "auto":
-        name = ("colocated_split" if optimizer == "asgd" and n in (5, 6) else
-                "colocated_bulkpipe" if n in (1, 5, 6, 7) else
-                "colocated_laneshfl" if n <= 4 else "colocated_regloop")
+    elif variant == "auto":   # ea_kernels.cu: SGD / ASGD warp per replica except N = 2 (lane kernel)
+        name = "colocated_laneshfl" if n == 2 else "colocated_warprep"
     else:
         name = "colocated_" + variant
     return name + ("" if optimizer == "sgd" else "<" + optimizer + ">")

@@ -1030,13 +1030,28 @@ cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cuda
 }
 
 // Warp per replica (variant 5): U float4 columns per lane and tile (SGD/ASGD 4: 2 KB rows per stream per tile;
-// Adam(W) 2, for registers).
-template <int N, int OPT, bool STALE = false>
-cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  constexpr int U = two_state(OPT) ? 2 : 4;
+// Adam(W) 2 by default, for registers; measurement knob AVGPIPE_EA_WARPREP_U=4 gives Adam(W) 4 as well).
+int warprep_u4() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_WARPREP_U");
+    return (e && e[0] == '4') ? 1 : 0;
+  }();
+  return v;
+}
+
+template <int N, int OPT, int U, bool STALE>
+cudaError_t launch_warprep_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   auto k = colocated_warprep<N, OPT, U, STALE>;
   k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
   return cudaGetLastError();
+}
+
+template <int N, int OPT, bool STALE = false>
+cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  if constexpr (two_state(OPT)) {
+    if (!warprep_u4()) return launch_warprep_u<N, OPT, 2, STALE>(b, hp, num_sms, s);
+  }
+  return launch_warprep_u<N, OPT, 4, STALE>(b, hp, num_sms, s);
 }
 
 template <int N>
@@ -1198,9 +1213,11 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // 0.941 vs 0.920 / 0.937; profiles/r02_sweep_split.jsonl -- with SGD it measured below the bulk pipeline).
   if (variant == kVariantAuto && two_state(opt))
     variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : (n == 4 ? kVariantBulkPipe : kVariantSplit));
-  if (variant == kVariantAuto && opt == kOptASGD && (n == 5 || n == 6)) variant = kVariantSplit;
-  if (variant == kVariantAuto)
-    variant = (n == 1 || (n >= 5 && n <= 7)) ? kVariantBulkPipe : (n <= 4 ? kVariantLaneShfl : kVariantRegLoop);
+  // SGD-momentum and ASGD (one state vector), round 2: the warp-per-replica kernel for N = 1 and 3..8 (same box,
+  // C2 sizes: N = 1 0.937 vs 0.872 bulk pipeline, N = 3 0.986 vs 0.932 lane, N = 4 0.996-0.998 vs 0.983 lane,
+  // N = 5..8 0.979-1.0 vs 0.93-0.976; ASGD alike), the lane kernel for N = 2 (0.963 vs 0.952);
+  // profiles/r02_sweep_warprep*.jsonl.  (Its Adam instances run out of registers: 0.69-0.87.)
+  if (variant == kVariantAuto) variant = n == 2 ? kVariantLaneShfl : kVariantWarpRep;
   switch (n) {
     case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
     case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
@@ -1253,6 +1270,9 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   if (b.nstages <= 0) return cudaSuccess;
   for (int t = 0; t < b.nstages; ++t)
     if (!b.st[t].prev) return cudaErrorInvalidValue;
+  // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
+  // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
+  if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
   if (variant == kVariantWarpRep) {
     switch (n) {
       case 1: return launch_stale_warprep_n<1>(b, hp, opt, num_sms, s);

@@ -83,9 +83,10 @@ def test_stale_kernel_name_and_launches(monkeypatch):
     import argparse
     monkeypatch.delenv("AVGPIPE_EA_FORCE_WIDE", raising=False)
     assert bench.kernel_name("auto", "sgd", 4, 1) == "colocated_laneshfl<stale>"
-    assert bench.kernel_name("auto", "asgd", 2, 1) == "colocated_laneshfl<stale,asgd>"
+    assert bench.kernel_name("auto", "asgd", 2, 1) == "colocated_warprep<stale,asgd>"
+    assert bench.kernel_name("auto", "adam", 2, 1) == "colocated_laneshfl<stale,adam>"
     assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_bulkpipe<stale>"
-    assert bench.kernel_name("auto", "sgd", 5, 1) == "colocated_bulkpipe<stale>"
+    assert bench.kernel_name("auto", "sgd", 5, 1) == "colocated_warprep<stale>"
     assert bench.kernel_name("auto", "adam", 1, 1) == "colocated_bulkpipe<stale,adam>"
     assert bench.kernel_name("auto", "adam", 5, 1) == "colocated_wide<stale>"
     assert bench.kernel_name("auto", "sgd", 6, 1) == "colocated_wide<stale>"
