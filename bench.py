@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe", "split", "warprep"), default="auto")
+    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe", "split", "warprep", "warpring"), default="auto")
     ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw", "asgd"), default="sgd",
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam(W) and ASGD are row f1)")
     ap.add_argument("--staleness", type=int, choices=(0, 1), default=0,

@@ -69,7 +69,7 @@ extern "C" {
 #define EA_API
 #endif
 
-#define EA_ABI_VERSION 5
+#define EA_ABI_VERSION 6
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
@@ -123,8 +123,10 @@ typedef struct {
                                    tile by cp.async.bulk into an mbarrier ring), 4 = split
                                    register loop (two lanes per center column, N/2 replicas
                                    each, shuffle reduction), 5 = warp per replica (contributions
-                                   reduced through shared memory).  Same results up to fp32 summation
-                                   order (DESIGN.md c14); the default picks per N and optimizer
+                                   reduced through shared memory), 6 = warp per replica with its
+                                   inputs streamed through a per-lane cp.async ring (synchronous
+                                   center; with staleness 1 the replica loop runs).  Same results
+                                   up to fp32 summation order (DESIGN.md c14); the default picks per N and optimizer
                                    (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */
   double beta1, beta2;          /* Adam(W): moment rates in [0,1) (torch defaults 0.9, 0.999); double so
@@ -324,6 +326,39 @@ EA_API const char* ea_last_error(ea_handle h);
  * (cap >= 2M) and returns 2M; returns -EA_EINVAL for K < 1, M < 0, stage out
  * of range, cap < 2M or out == NULL (with M > 0).  Host only; no GPU needed. */
 EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance, ea_op* out, int32_t cap);
+
+/* ---- Point-to-point activation channel (row f2; csrc/ea_chan.cu) ----
+ * The transfers of the pipeline runtime: stage k sends activations to stage k+1 and receives activation
+ * gradients back, in Algorithm 1's order ("a parallel pipeline launches a process on each GPU",
+ * P:140-162).  A channel is ONE direction between two processes (NVLink peers, or two processes sharing a GPU).
+ * The receiving end owns a ring of `slots` message slots of `slot_bytes` and one ready word per slot, the
+ * sending end one acknowledgement word per slot, all in device memory on `device`.  Each end exports its buffer
+ * (ea_chan_export, EA_IPC_HANDLE_BYTES, cudaIpcMemHandle_t) and opens the other's (ea_chan_connect); two ends
+ * in ONE process are wired with ea_chan_pair instead (CUDA IPC cannot open a handle of its own process).
+ *
+ * ea_chan_send / ea_chan_recv enqueue on `stream` (cudaStream_t; NULL = legacy default stream) and never block
+ * the host: send = wait until the slot is free (stream wait on the local ack word) -> copy-engine copy of
+ * `bytes` from device pointer src into the receiver's slot over the peer mapping -> stream write of the
+ * receiver's ready word; recv = stream wait on the local ready word -> copy into device pointer dst -> stream
+ * write of the sender's ack word.  The k-th send matches the k-th recv (k counts calls on each end).  src must
+ * stay unmodified, and dst unread, until the stream reaches that point.  Errors: bytes > slot_bytes, a NULL
+ * buffer or the wrong end -> EA_EINVAL; not connected, or the stream is capturing a CUDA graph (the slot and
+ * round are host counters) -> EA_ESTATE; CUDA / driver failures -> EA_ECUDA.  Nothing is enqueued on error.
+ * ea_chan_destroy synchronises the device, closes the peer mapping and frees this end's buffer: both ends
+ * must be past their last operation (a caller-side barrier) before either is destroyed. */
+typedef struct ea_chan_s* ea_chan;
+EA_API ea_status ea_chan_create(int32_t device, int32_t role /* 0 = send, 1 = recv */, int64_t slot_bytes,
+                                int32_t slots, ea_chan* out);
+EA_API ea_status ea_chan_export(ea_chan c, uint8_t* handle);
+EA_API ea_status ea_chan_connect(ea_chan c, const uint8_t* peer_handle);
+EA_API ea_status ea_chan_pair(ea_chan send_end, ea_chan recv_end);
+EA_API ea_status ea_chan_send(ea_chan c, const void* src, int64_t bytes, void* stream);
+EA_API ea_status ea_chan_recv(ea_chan c, void* dst, int64_t bytes, void* stream);
+/* Messages enqueued so far on this end (-1 for NULL). */
+EA_API int64_t ea_chan_count(ea_chan c);
+EA_API ea_status ea_chan_destroy(ea_chan c);
+/* Message of the last failing call on c (c == NULL: this thread's last ea_chan_create failure). */
+EA_API const char* ea_chan_last_error(ea_chan c);
 
 /* ---- Run-time advance adjustment (Algorithm 1 lines 1, 9-10) ---- */
 

@@ -20,11 +20,12 @@ EA_OK, EA_EINVAL, EA_ECUDA, EA_ENCCL, EA_ESTATE, EA_ENOMEM = range(6)
 EA_COLOCATED, EA_SPREAD = 0, 1
 STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA_ESTATE", 5: "EA_ENOMEM"}
 LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
-VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3, "split": 4, "warprep": 5}
+VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3, "split": 4, "warprep": 5, "warpring": 6}
 OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2, "asgd": 3}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
-ABI_VERSION = 5
+IPC_HANDLE_BYTES = 64   # == EA_IPC_HANDLE_BYTES (cudaIpcMemHandle_t)
+ABI_VERSION = 6
 SLOT_CENTER_PREV = 2   # EA_SLOT_CENTER_PREV: the stale center x~_{t-1} (staleness 1)
 
 
@@ -152,6 +153,16 @@ SIGNATURES = {
                                ctypes.POINTER(ctypes.c_double)]),
     "ea_schedule": (ctypes.c_int32, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int32, ctypes.c_int32,
                                      ctypes.POINTER(EAOp), ctypes.c_int32]),
+    "ea_chan_create": (ctypes.c_int, [ctypes.c_int32, ctypes.c_int32, ctypes.c_int64, ctypes.c_int32,
+                                      ctypes.POINTER(_VP)]),
+    "ea_chan_export": (ctypes.c_int, [_VP, ctypes.c_void_p]),
+    "ea_chan_connect": (ctypes.c_int, [_VP, ctypes.c_void_p]),
+    "ea_chan_pair": (ctypes.c_int, [_VP, _VP]),
+    "ea_chan_send": (ctypes.c_int, [_VP, _VP, ctypes.c_int64, _VP]),
+    "ea_chan_recv": (ctypes.c_int, [_VP, _VP, ctypes.c_int64, _VP]),
+    "ea_chan_count": (ctypes.c_int64, [_VP]),
+    "ea_chan_destroy": (ctypes.c_int, [_VP]),
+    "ea_chan_last_error": (ctypes.c_char_p, [_VP]),
 }
 
 _lib = None
@@ -275,6 +286,74 @@ def _host_ptr(t, what: str) -> int:
     if not isinstance(t, torch.Tensor) or t.dtype != torch.float32 or t.is_cuda or not t.is_contiguous():
         raise TypeError(f"{what} must be a contiguous float32 CPU tensor (pinned for asynchronous copies)")
     return t.data_ptr()
+
+
+class Channel:
+    """One end of a point-to-point activation channel (``ea_chan_*``, row f2): role "send" or "recv", a ring
+    of `slots` messages of at most `slot_bytes` on `device`.  Wire the two ends with ``export()`` /
+    ``connect(peer_handle)`` across processes, or ``Channel.pair(send_end, recv_end)`` in one process.
+    ``send(t)`` / ``recv(t)`` enqueue on `stream` (default: the current stream); the host never waits."""
+
+    def __init__(self, role: str, slot_bytes: int, slots: int, device: Optional[int] = None):
+        import torch
+        self._lib = load_library()
+        self.role = role
+        self.slot_bytes, self.slots = int(slot_bytes), int(slots)
+        self.device = torch.cuda.current_device() if device is None else int(device)
+        h = ctypes.c_void_p()
+        st = self._lib.ea_chan_create(self.device, {"send": 0, "recv": 1}[role], self.slot_bytes, self.slots,
+                                      ctypes.byref(h))
+        if st != EA_OK:
+            raise EAError(st, (self._lib.ea_chan_last_error(None) or b"").decode())
+        self._h = h
+
+    def _check(self, st):
+        if st != EA_OK:
+            raise EAError(st, (self._lib.ea_chan_last_error(self._h) or b"").decode())
+
+    def export(self) -> bytes:
+        buf = (ctypes.c_uint8 * IPC_HANDLE_BYTES)()
+        self._check(self._lib.ea_chan_export(self._h, buf))
+        return bytes(buf)
+
+    def connect(self, peer_handle: bytes):
+        if len(peer_handle) != IPC_HANDLE_BYTES:
+            raise ValueError(f"peer handle must be {IPC_HANDLE_BYTES} bytes")
+        self._check(self._lib.ea_chan_connect(self._h, (ctypes.c_uint8 * IPC_HANDLE_BYTES).from_buffer_copy(peer_handle)))
+
+    @staticmethod
+    def pair(send_end: "Channel", recv_end: "Channel"):
+        send_end._check(send_end._lib.ea_chan_pair(send_end._h, recv_end._h))
+
+    @staticmethod
+    def _buf(t):
+        import torch
+        if not isinstance(t, torch.Tensor) or not t.is_cuda or not t.is_contiguous():
+            raise TypeError("channel buffers must be contiguous CUDA tensors")
+        return t.data_ptr(), t.numel() * t.element_size()
+
+    def send(self, t, stream=None):
+        p, n = self._buf(t)
+        self._check(self._lib.ea_chan_send(self._h, p, n, _stream_ptr(stream)))
+
+    def recv(self, t, stream=None):
+        p, n = self._buf(t)
+        self._check(self._lib.ea_chan_recv(self._h, p, n, _stream_ptr(stream)))
+
+    @property
+    def count(self) -> int:
+        return int(self._lib.ea_chan_count(self._h))
+
+    def close(self):
+        if getattr(self, "_h", None):
+            self._lib.ea_chan_destroy(self._h)
+            self._h = None
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
 
 
 class ElasticAveraging:

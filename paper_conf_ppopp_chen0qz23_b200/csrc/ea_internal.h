@@ -99,6 +99,7 @@ enum KernelVariant : int {
                          // ring (producer warp + mbarriers); consumers store from registers (SGD)
   kVariantSplit = 4,     // split register loop: 2 lanes per center column, N/2 replicas each, shuffle reduction
   kVariantWarpRep = 5,   // warp per replica, 512 B rows, contributions reduced through shared memory
+  kVariantWarpRing = 6,  // warp per replica, inputs streamed through a per-lane cp.async ring in shared memory
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N

@@ -374,6 +374,134 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
+// ============================================================================
+// Variant 6: warp per replica with a cp.async ring.  The warp-per-replica kernel keeps a tile's loads in
+// registers, so with Adam's four streams per replica few bytes are in flight per SM while a CTA computes and
+// waits at its barrier (0.69-0.87 of peak).  Here every lane copies ITS OWN 16-byte pieces of the next S-1
+// tiles (x, g, the optimizer state and x~) into shared memory with cp.async (LDGSTS: no registers held while in
+// flight) and reads back only what it copied itself -- so the ring needs no barrier and no mbarrier, only
+// cp.async.wait_group; the one block-level exchange left is the replica reduction of the contributions
+// (double-buffered, one named barrier per column group and tile).
+// CTA = G column groups x N warps; warp w: replica i = w % N, group q = w / N; a tile is G x 32U float4 columns.
+// In the reduction thread (q, i, lane) owns the columns u*32 + lane of its group with u = i (mod N), whose x~
+// it copied itself.
+// ============================================================================
+template <int N, int OPT, int U, int S>
+struct RingGeom {
+  static constexpr int G = N >= 8 ? 1 : 8 / N;           // column groups per CTA
+  static constexpr int W = N * G;                         // warps
+  static constexpr int NS = (two_state(OPT) ? 4 : 3) + 1; // x, g, m, (v), x~
+  static constexpr int TV = G * 32 * U;                   // float4 columns per tile
+  static constexpr int kRingVec = S * W * NS * U * 32;
+  static constexpr int kRedVec = N > 1 ? 2 * N * TV : 0;
+  static constexpr int kSmemBytes = (kRingVec + kRedVec) * 16;
+};
+
+__device__ __forceinline__ void cp_async16(float4* dst, const float* src) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int K>
+__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(K) : "memory"); }
+
+template <int N, int OPT, int U, int S>
+__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warpring(const StageBatch b,
+                                                                                      const Hyper hp) {
+  using RG = RingGeom<N, OPT, U, S>;
+  constexpr int TV = RG::TV, NS = RG::NS;
+  constexpr bool kTwo = two_state(OPT);
+  extern __shared__ __align__(16) float4 ring[];
+  float4* s_r = ring + RG::kRingVec;  // [2][N][TV] contributions (N > 1)
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
+  const Mem<0> mem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int rep = warp % N, grp = warp / N;
+  if (has_coef(OPT)) {
+    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+    __syncthreads();
+  }
+  // this lane's piece of slot k, stream a, unroll u
+  auto piece = [&](int k, int a, int u) -> float4* {
+    return ring + ((k * RG::W + warp) * NS + a) * (U * 32) + u * 32 + lane;
+  };
+  auto issue = [&](int k, int s, int64_t v0, int64_t nv) {
+    const StageRefs& st = b.st[s];
+    const float* src[NS];
+    src[0] = st.x[rep];
+    src[1] = st.g[rep];
+    src[2] = st.m[rep];
+    if constexpr (kTwo) src[3] = st.v[rep];
+    src[NS - 1] = st.c;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int col = grp * 32 * U + u * 32 + lane;
+      if (col < nv) {
+        const int64_t v = v0 + col;
+#pragma unroll
+        for (int a = 0; a < NS; ++a) cp_async16(piece(k, a, u), src[a] + 4 * v);
+      }
+    }
+  };
+  WaveCursor lc{0, 0}, cc{0, 0};
+  int s;
+  int64_t v0, nv;
+#pragma unroll
+  for (int k = 0; k < S - 1; ++k) {
+    if (wave_item(b, TV, lc, s, v0, nv)) issue(k, s, v0, nv);
+    cp_async_commit();
+  }
+  int slot = 0, par = 0;
+  while (wave_item(b, TV, cc, s, v0, nv)) {
+    {  // refill the slot this lane finished with in the previous tile (it reads only its own pieces)
+      int s2;
+      int64_t w0, wn;
+      if (wave_item(b, TV, lc, s2, w0, wn)) issue(slot == 0 ? S - 1 : slot - 1, s2, w0, wn);
+      cp_async_commit();
+    }
+    cp_async_wait<S - 1>();  // this lane's copies of the current tile have landed
+    const StageRefs& st = b.st[s];
+    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
+    float* xi = st.x[rep];
+    float* mi = st.m[rep];
+    float* vi = kTwo ? st.v[rep] : nullptr;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int col = grp * 32 * U + u * 32 + lane;
+      if (col < nv) {
+        const int64_t v = v0 + col;
+        float4 x = *piece(slot, 0, u), g = *piece(slot, 1, u), m = *piece(slot, 2, u);
+        float4 w = kTwo ? *piece(slot, 3, u) : make_float4(0.f, 0.f, 0.f, 0.f);
+        const float4 c = *piece(slot, NS - 1, u);
+        const float4 r = ea_vec<OPT>(x, g, m, w, c, hp, sc);
+        mem.st(xi + 4 * v, x);
+        mem.st(mi + 4 * v, m);
+        if constexpr (kTwo) mem.st(vi + 4 * v, w);
+        if constexpr (N == 1) mem.st(st.c + 4 * v, center_apply(c, r, hp.inv_n));
+        else s_r[(par * N + rep) * TV + col] = r;
+      }
+    }
+    if constexpr (N > 1) {
+      asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "n"(32 * N) : "memory");  // this group's N warps
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        if (u % N != rep) continue;
+        const int col = grp * 32 * U + u * 32 + lane;
+        if (col < nv) {
+          float4 acc = s_r[(par * N) * TV + col];
+#pragma unroll
+          for (int i = 1; i < N; ++i) add4(acc, s_r[(par * N + i) * TV + col]);
+          mem.st(st.c + 4 * (v0 + col), center_apply(*piece(slot, NS - 1, u), acc, hp.inv_n));
+        }
+      }
+      par ^= 1;  // the next tile writes the other buffer; the one after waits behind the next barrier
+    }
+    slot = slot == S - 1 ? 0 : slot + 1;
+  }
+  cp_async_wait<0>();
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+}
+
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -879,9 +1007,9 @@ int grid_knob() {
 }
 
 template <typename K>
-int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads) {
+int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads, size_t smem = 0) {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0) != cudaSuccess || per_sm < 1)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess || per_sm < 1)
     per_sm = 1;
   int64_t grid = (int64_t)num_sms * per_sm;
   const int knob = grid_knob();
@@ -1054,8 +1182,52 @@ cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_warprep_u<N, OPT, 4, STALE>(b, hp, num_sms, s);
 }
 
+// Warp per replica with a cp.async ring (variant 6): U float4 columns per lane and tile, S tiles in the ring.
+// Measurement knob AVGPIPE_EA_RING = <U><S>: 14 (default), 16, 18, 24, 23.
+int ring_geom() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_RING");
+    return e ? std::atoi(e) : 14;
+  }();
+  return v;
+}
+
+template <int N, int OPT, int U, int S>
+cudaError_t launch_warpring_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  using RG = RingGeom<N, OPT, U, S>;
+  if constexpr (RG::kSmemBytes > 227 * 1024) {
+    return cudaErrorInvalidConfiguration;
+  } else {
+    auto k = colocated_warpring<N, OPT, U, S>;
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
+    if (e != cudaSuccess) return e;
+    const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
+    k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp);
+    return cudaGetLastError();
+  }
+}
+
+template <int N, int OPT>
+cudaError_t launch_warpring(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  switch (ring_geom()) {
+    case 16: return launch_warpring_t<N, OPT, 1, 6>(b, hp, num_sms, s);
+    case 18: return launch_warpring_t<N, OPT, 1, 8>(b, hp, num_sms, s);
+    case 24: return launch_warpring_t<N, OPT, 2, 4>(b, hp, num_sms, s);
+    case 23: return launch_warpring_t<N, OPT, 2, 3>(b, hp, num_sms, s);
+    default: return launch_warpring_t<N, OPT, 1, 4>(b, hp, num_sms, s);
+  }
+}
+
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (variant == kVariantWarpRing) {
+    switch (opt) {
+      case kOptAdam: return launch_warpring<N, kOptAdam>(b, hp, num_sms, s);
+      case kOptAdamW: return launch_warpring<N, kOptAdamW>(b, hp, num_sms, s);
+      case kOptASGD: return launch_warpring<N, kOptASGD>(b, hp, num_sms, s);
+      default: return launch_warpring<N, kOptSGD>(b, hp, num_sms, s);
+    }
+  }
   if (variant == kVariantWarpRep) {
     switch (opt) {
       case kOptAdam: return launch_warprep<N, kOptAdam>(b, hp, num_sms, s);

@@ -24,11 +24,16 @@ iteration's forward of pipeline i waits for it on the GPU (it reads x_i) --
 P:112 "in an asynchronous manner ... to prevent the inter-process
 communication blocking the pipeline".
 
-Transfers: with the ``nccl`` backend activations stay on the GPU
-(torch.distributed isend/recv of device tensors over NVLink); with ``gloo``
-they are staged through host memory.  The compute of a stage is the caller's
-``torch.nn.Module`` (autograd); the runtime owns the order, the transfers, the
-activation stash and the averaging.
+Transfers (``transport``): "dist" -- torch.distributed point-to-point, device
+tensors over NCCL (NVLink) with the ``nccl`` backend, staged through host
+memory with ``gloo``; "ipc" -- the library's own activation channels
+(``binding.Channel``, ``ea_chan_*``): copy-engine copies straight into the
+receiving stage's device memory over a CUDA IPC peer mapping, handshaken by
+stream memory operations, so neither host waits for a transfer (the process
+group only carries the one-time handle exchange; two processes may share a
+GPU).  The compute of a stage is the caller's ``torch.nn.Module`` (autograd);
+the runtime owns the order, the transfers, the activation stash and the
+averaging.
 """
 from __future__ import annotations
 
@@ -36,7 +41,7 @@ import threading
 import time
 from typing import Callable, List, Optional, Sequence
 
-from .binding import AdvanceController, schedule
+from .binding import AdvanceController, Channel, schedule
 
 
 def make_pipeline_groups(n_pipelines: int, ranks: Optional[Sequence[int]] = None, backend: Optional[str] = None):
@@ -58,7 +63,8 @@ class PipelineStage:
     def __init__(self, replicas: Sequence, stage: int, K: int, M: int, group=None, *, ea=None, ea_stage: int = 0,
                  center=None, flat_params=None, flat_grads=None, mem_limit: Optional[float] = None,
                  mem_per_microbatch: float = 0.0, extra_advance: int = 0, dynamic: bool = False,
-                 concurrent: bool = False, groups=None):
+                 concurrent: bool = False, groups=None, transport: str = "dist", act_bytes: int = 0,
+                 device=None):
         import torch.distributed as dist
         self.replicas = list(replicas)
         self.N = len(self.replicas)
@@ -84,6 +90,54 @@ class PipelineStage:
         self._streams = None      # per-pipeline CUDA streams (concurrent, on a GPU)
         self._ea_stream = None
         self._ea_done = None      # event: the last EA step (the next forward of every pipeline waits for it)
+        if transport not in ("dist", "ipc"):
+            raise ValueError("transport must be 'dist' or 'ipc'")
+        self.transport = transport
+        self._chan = {}
+        if transport == "ipc":
+            self._open_channels(act_bytes, device)
+
+    # ------------------------------------------------------------------ activation channels (transport "ipc")
+    def _open_channels(self, act_bytes: int, device):
+        """Per pipeline i: a forward channel to the next stage and a backward channel from it (and the mirror
+        ends toward the previous stage), M slots of act_bytes each -- a sender never waits for a free slot, as at
+        most M messages of one direction are in flight per iteration.  The IPC handles travel once over the
+        stage process group (all_gather_object); every end then maps its peer's buffer."""
+        import torch
+        import torch.distributed as dist
+        if act_bytes <= 0:
+            raise ValueError("transport 'ipc' needs act_bytes (bytes of the largest activation message)")
+        dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
+        mine = {}
+        for i in range(self.N):
+            if self.next is not None:
+                self._chan[("F", i, "send")] = Channel("send", act_bytes, self.M, dev.index)
+                self._chan[("B", i, "recv")] = Channel("recv", act_bytes, self.M, dev.index)
+                mine[("F", i, self.stage, "send")] = self._chan[("F", i, "send")].export()
+                mine[("B", i, self.stage + 1, "recv")] = self._chan[("B", i, "recv")].export()
+            if self.prev is not None:
+                self._chan[("F", i, "recv")] = Channel("recv", act_bytes, self.M, dev.index)
+                self._chan[("B", i, "send")] = Channel("send", act_bytes, self.M, dev.index)
+                mine[("F", i, self.stage - 1, "recv")] = self._chan[("F", i, "recv")].export()
+                mine[("B", i, self.stage, "send")] = self._chan[("B", i, "send")].export()
+        allh = [None] * dist.get_world_size(self.group)
+        dist.all_gather_object(allh, mine, group=self.group)
+        for i in range(self.N):
+            if self.next is not None:      # F: stage -> stage+1 (key: source stage); B: stage+1 -> stage
+                self._chan[("F", i, "send")].connect(allh[self.stage + 1][("F", i, self.stage, "recv")])
+                self._chan[("B", i, "recv")].connect(allh[self.stage + 1][("B", i, self.stage + 1, "send")])
+            if self.prev is not None:
+                self._chan[("F", i, "recv")].connect(allh[self.stage - 1][("F", i, self.stage - 1, "send")])
+                self._chan[("B", i, "send")].connect(allh[self.stage - 1][("B", i, self.stage, "recv")])
+
+    def close(self):
+        """Free the activation channels (every stage past its last iteration first: a collective barrier)."""
+        import torch.distributed as dist
+        if self._chan:
+            dist.barrier(group=self.group)
+            for c in self._chan.values():
+                c.close()
+            self._chan = {}
 
     # ------------------------------------------------------------------ transfers
     def _peer(self, stage_index, group):
@@ -93,16 +147,23 @@ class PipelineStage:
     def _tag(self, pipeline: int, j: int, backward: bool) -> int:
         return ((pipeline * self.M + j) << 1) | int(backward)
 
-    def _send(self, t, dst_stage, tag, group):
+    def _send(self, t, dst_stage, tag, group, pipeline=0, backward=False):
         import torch.distributed as dist
         t = t.detach().contiguous()
+        if self.transport == "ipc":     # stream-ordered; t was produced on this stream, so its reuse is ordered
+            self._chan[("B" if backward else "F", pipeline, "send")].send(t)
+            return None
         if self.backend == "gloo" and t.is_cuda:      # gloo moves host tensors
             t = t.cpu()
         return dist.isend(t, dst=self._peer(dst_stage, group), group=group, tag=tag)
 
-    def _recv(self, like_shape, dtype, device, src_stage, tag, group):
+    def _recv(self, like_shape, dtype, device, src_stage, tag, group, pipeline=0, backward=False):
         import torch
         import torch.distributed as dist
+        if self.transport == "ipc":     # the GPU waits for the message, not the host
+            buf = torch.empty(like_shape, dtype=dtype, device=device)
+            self._chan[("B" if backward else "F", pipeline, "recv")].recv(buf)
+            return buf
         host = self.backend == "gloo"
         buf = torch.empty(like_shape, dtype=dtype, device="cpu" if host else device)
         dist.recv(buf, src=self._peer(src_stage, group), group=group, tag=tag)
@@ -119,7 +180,7 @@ class PipelineStage:
                 if self.prev is None:
                     x = inputs[i][j]
                 else:
-                    x = self._recv(act_shape, act_dtype, device, self.prev, self._tag(i, j, False), group)
+                    x = self._recv(act_shape, act_dtype, device, self.prev, self._tag(i, j, False), group, i)
                     x.requires_grad_(True)
                 y = mod(x)
                 if self.next is None:
@@ -127,7 +188,7 @@ class PipelineStage:
                     loss_sum += float(loss.detach())
                     stash[j] = (x, loss)
                 else:
-                    pending.append(self._send(y, self.next, self._tag(i, j, False), group))
+                    pending.append(self._send(y, self.next, self._tag(i, j, False), group, i))
                     stash[j] = (x, y)
                 peak = max(peak, len(stash))
             else:
@@ -135,10 +196,10 @@ class PipelineStage:
                 if self.next is None:
                     y.backward()
                 else:
-                    gy = self._recv(y.shape, y.dtype, device, self.next, self._tag(i, j, True), group)
+                    gy = self._recv(y.shape, y.dtype, device, self.next, self._tag(i, j, True), group, i, True)
                     y.backward(gy)
                 if self.prev is not None:
-                    pending.append(self._send(x.grad, self.prev, self._tag(i, j, True), group))
+                    pending.append(self._send(x.grad, self.prev, self._tag(i, j, True), group, i, True))
         return loss_sum, pending, peak
 
     def _cuda(self, device):
@@ -198,7 +259,7 @@ class PipelineStage:
                 if zero_grads and self.flat_grads is not None:
                     self.flat_grads[i].zero_()
                 results[i] = self._run_pipeline(i, ops, inputs, targets, loss_fn, act_shape, act_dtype, device)
-        pending = [w for r in results for w in r[1]]
+        pending = [w for r in results for w in r[1] if w is not None]
         peak = max(r[2] for r in results)
         if self.ea is not None:
             # every pipeline's last backward of this stage is done: the averaging step goes onto its own stream

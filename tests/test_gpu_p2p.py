@@ -57,6 +57,11 @@ def _run(n, sizes, steps, mode, optimizer="sgd", stage_order=None):
         for s in order:                  # every rank issues its stages in the same global order
             for r in range(n):
                 hs[r].step(s, [xs[s][r]], [grads[s][r]], centers[s][r], stream=streams[r])
+                # the gradient was allocated on the default stream and is read on streams[r]: without this the
+                # caching allocator may hand its block to the next step's gradient, whose copy (default stream)
+                # then overwrites it while this step's push still reads it (seen under compute-sanitizer racecheck,
+                # which slows the kernels enough to expose it: profiles/r02_sanitizers.md)
+                grads[s][r].record_stream(streams[r])
     for r in range(n):
         hs[r].sync(streams[r])
     torch.cuda.synchronize()

@@ -11,6 +11,8 @@ c13 metric <= 1e-5 on every x_i, m_i and x~ (tests/_parity.py):
     path at world = 1;
   * optimizer-state get/set (checkpoint/resume) and set_hyper.
 """
+import os
+
 import numpy as np
 import pytest
 import torch
@@ -18,6 +20,8 @@ import torch
 from paper_conf_ppopp_chen0qz23_b200 import synth
 from paper_conf_ppopp_chen0qz23_b200.binding import EAError, ElasticAveraging, get_unique_id
 from tests._parity import TOL, OracleStage, asgd_kw, hyper, rel_err, to_np
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 pytestmark = pytest.mark.gpu
 
@@ -248,6 +252,37 @@ def test_warp_per_replica_stale(n, optimizer):
     lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
     _run_colocated(n, [100_003, 7, 4096], 20, "combined", variants=("warprep",), many=True, optimizer=optimizer,
                    lr=lr, staleness=1)
+
+
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8])
+def test_warp_ring(n, optimizer):
+    """Variant 6 (warp per replica, inputs through a per-lane cp.async ring, contributions reduced through
+    shared memory): C1-sized and ragged stages in one launch (several ring refills per CTA, ragged last tiles,
+    the scalar tails), every optimizer."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 12, "combined", variants=("warpring",), many=True,
+                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+
+
+@pytest.mark.parametrize("geom", ["16", "18", "24", "23"])
+@pytest.mark.parametrize("n", [1, 3, 8])
+def test_warp_ring_geometries(n, geom, monkeypatch):
+    """The ring geometries behind the measurement knob AVGPIPE_EA_RING (read once per process, so each case
+    runs in a subprocess)."""
+    import subprocess
+    import sys
+    code = ("import tests.test_gpu_parity as t; "
+            f"t._run_colocated({n}, [100_003, 7, 4096, 1_000_001], 6, 'combined', variants=('warpring',), many=True, "
+            "optimizer='adam', lr=1e-3, wd=1e-2)")
+    env = dict(os.environ, AVGPIPE_EA_RING=geom)
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
+def test_warp_ring_c1_100_steps():
+    _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warpring",), many=True, optimizer="adam",
+                   lr=1e-3, wd=1e-2)
 
 
 def test_warp_per_replica_c1_100_steps():

@@ -1,5 +1,5 @@
 """End to end on one GPU: K=2 pipeline stages as 2 processes sharing cuda:0
-(activations over gloo), N=2 parallel pipelines, advance-forward order, and
+(activations over gloo, or the library's CUDA-IPC activation channels), N=2 parallel pipelines, advance-forward order, and
 after every iteration ONE fused co-located elastic-averaging step per stage
 on the stage's parameters (views into flat buffers the kernel updates in
 place).  Compared with a single-process reference: the full model's autograd
@@ -48,7 +48,7 @@ def _flatten(mod, device):
     return flat, gflat
 
 
-def _worker(rank, port, q, concurrent=False, backend="gloo"):
+def _worker(rank, port, q, concurrent=False, backend="gloo", transport="dist"):
     try:
         dev = torch.device("cuda", rank if backend == "nccl" else 0)
         torch.cuda.set_device(dev)
@@ -65,7 +65,7 @@ def _worker(rank, port, q, concurrent=False, backend="gloo"):
         ea = ElasticAveraging([P], N, beta=1.0, rho=1.0, lr=LR, momentum=MU, device=dev.index)   # alpha = 1/N
         st = PipelineStage(mods, rank, K, M, ea=ea, ea_stage=0, center=center,
                            flat_params=[f for f, _ in flats], flat_grads=[g for _, g in flats], extra_advance=1,
-                           concurrent=concurrent)
+                           concurrent=concurrent, transport=transport, act_bytes=B * D * 4, device=dev)
         for it in range(ITERS):
             xs, ys = _data(it)
             if not concurrent:
@@ -79,6 +79,7 @@ def _worker(rank, port, q, concurrent=False, backend="gloo"):
                              device=dev, zero_grads=concurrent, sync=not concurrent)
         torch.cuda.synchronize()
         q.put((rank, "ok", [f.cpu().numpy() for f, _ in flats], center.cpu().numpy()))
+        st.close()
         ea.close()
     except Exception:  # pragma: no cover
         import traceback
@@ -120,17 +121,21 @@ def _reference():
     return [[flat(models[i], k) for i in range(N)] for k in range(K)], centers
 
 
-@pytest.mark.parametrize("concurrent,backend", [(False, "gloo"), (True, "gloo"), (True, "nccl")])
-def test_pipeline_with_elastic_averaging_matches_reference(concurrent, backend):
+@pytest.mark.parametrize("concurrent,backend,transport", [(False, "gloo", "dist"), (True, "gloo", "dist"),
+                                                           (True, "nccl", "dist"), (False, "gloo", "ipc"),
+                                                           (True, "gloo", "ipc")])
+def test_pipeline_with_elastic_averaging_matches_reference(concurrent, backend, transport):
     """concurrent: the N pipelines at once (thread + stream + process group each), the EA step on its own
-    stream.  nccl: activations as device tensors over NCCL, one GPU per stage (needs K GPUs)."""
+    stream.  nccl: activations as device tensors over NCCL, one GPU per stage (needs K GPUs).  ipc: activations
+    through the library's channels (ea_chan_*: copy engine into the peer stage's memory over CUDA IPC, the GPU
+    waits for messages, not the host); both stages share cuda:0 here, the same code maps NVLink peers."""
     import tempfile
     if backend == "nccl" and torch.cuda.device_count() < K:
         pytest.skip(f"NCCL activations need {K} GPUs (NCCL refuses two ranks on one device)")
     port = "file://" + os.path.join(tempfile.mkdtemp(prefix="gloo_"), "store")   # no TCP port race
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    procs = [ctx.Process(target=_worker, args=(r, port, q, concurrent, backend)) for r in range(K)]
+    procs = [ctx.Process(target=_worker, args=(r, port, q, concurrent, backend, transport)) for r in range(K)]
     for p in procs:
         p.start()
     out = {}

@@ -41,6 +41,7 @@ def test_stale_spread_world1_real_nccl(optimizer):
             gd = torch.from_numpy(g[0]).to(DEV)
             torch.cuda.synchronize()
             h.step(s, [xs[s]], [gd], cs[s], stream=stream)
+            gd.record_stream(stream)     # allocated on the default stream, read on `stream` (see test_gpu_p2p._run)
             oracle[s].step(g, hp)
         stream.synchronize()
     h.sync(stream)
