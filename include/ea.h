@@ -124,8 +124,8 @@ typedef struct {
                                    register loop (two lanes per center column, N/2 replicas
                                    each, shuffle reduction), 5 = warp per replica (contributions
                                    reduced through shared memory), 6 = warp per replica with its
-                                   inputs streamed through a per-lane cp.async ring (synchronous
-                                   center; with staleness 1 the replica loop runs).  Same results
+                                   inputs streamed through a per-lane cp.async ring (x~_{t-1} as
+                                   one more stream with staleness 1).  Same results
                                    up to fp32 summation order (DESIGN.md c14); the default picks per N and optimizer
                                    (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */

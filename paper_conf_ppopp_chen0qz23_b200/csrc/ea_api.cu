@@ -328,7 +328,8 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // the replica loop for A/B measurement.
   const bool stale_lane = stale && !force_wide &&
                           ((h->variant == 0 && (n <= 4 || (n == 5 && !ea::two_state(opt)))) ||
-                           (h->variant == ea::kVariantWarpRep && n <= ea::kMaxFusedN));
+                           ((h->variant == ea::kVariantWarpRep || h->variant == ea::kVariantWarpRing) &&
+                            n <= ea::kMaxFusedN));
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
     for (int j = 0; j < count; ++j) {
       ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);

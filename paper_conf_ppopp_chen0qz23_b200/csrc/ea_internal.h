@@ -112,7 +112,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
 // lane kernel with x~_{t-1} staged beside x~_t, for N = 1 and 5 the bulk-copy pipeline with x~_{t-1} as one more
 // stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
 constexpr int kMaxStaleLaneN = 4;
-// variant kVariantWarpRep: the warp-per-replica kernel with x~_{t-1} for any N <= kMaxFusedN.
+// variant kVariantWarpRep / kVariantWarpRing: the warp-per-replica kernels with x~_{t-1} for any N <= kMaxFusedN.
 cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int variant,
                                          int num_sms, cudaStream_t s);
 

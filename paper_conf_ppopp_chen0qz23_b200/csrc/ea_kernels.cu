@@ -386,11 +386,13 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
 // In the reduction thread (q, i, lane) owns the columns u*32 + lane of its group with u = i (mod N), whose x~
 // it copied itself.
 // ============================================================================
-template <int N, int OPT, int U, int S>
+// STALE (row f4, reading c28): one more stream, x~_{t-1} (what the replicas see); x~_t is then copied only for
+// the columns the lane reduces, and the reduction writes x~_{t+1} and rolls x~_{t-1} <- x~_t.
+template <int N, int OPT, int U, int S, bool STALE = false>
 struct RingGeom {
   static constexpr int G = N >= 8 ? 1 : 8 / N;           // column groups per CTA
   static constexpr int W = N * G;                         // warps
-  static constexpr int NS = (two_state(OPT) ? 4 : 3) + 1; // x, g, m, (v), x~
+  static constexpr int NS = (two_state(OPT) ? 4 : 3) + 1 + (STALE ? 1 : 0);  // x, g, m, (v), (x~_{t-1}), x~_t
   static constexpr int TV = G * 32 * U;                   // float4 columns per tile
   static constexpr int kRingVec = S * W * NS * U * 32;
   static constexpr int kRedVec = N > 1 ? 2 * N * TV : 0;
@@ -404,10 +406,10 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int K>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(K) : "memory"); }
 
-template <int N, int OPT, int U, int S>
-__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warpring(const StageBatch b,
-                                                                                      const Hyper hp) {
-  using RG = RingGeom<N, OPT, U, S>;
+template <int N, int OPT, int U, int S, bool STALE = false>
+__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocated_warpring(const StageBatch b,
+                                                                                             const Hyper hp) {
+  using RG = RingGeom<N, OPT, U, S, STALE>;
   constexpr int TV = RG::TV, NS = RG::NS;
   constexpr bool kTwo = two_state(OPT);
   extern __shared__ __align__(16) float4 ring[];
@@ -431,6 +433,7 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warp
     src[1] = st.g[rep];
     src[2] = st.m[rep];
     if constexpr (kTwo) src[3] = st.v[rep];
+    if constexpr (STALE) src[NS - 2] = st.prev;
     src[NS - 1] = st.c;
 #pragma unroll
     for (int u = 0; u < U; ++u) {
@@ -438,7 +441,8 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warp
       if (col < nv) {
         const int64_t v = v0 + col;
 #pragma unroll
-        for (int a = 0; a < NS; ++a) cp_async16(piece(k, a, u), src[a] + 4 * v);
+        for (int a = 0; a < NS; ++a)   // stale: x~_t only where this lane reduces
+          if (!STALE || a != NS - 1 || u % N == rep) cp_async16(piece(k, a, u), src[a] + 4 * v);
       }
     }
   };
@@ -471,13 +475,18 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warp
         const int64_t v = v0 + col;
         float4 x = *piece(slot, 0, u), g = *piece(slot, 1, u), m = *piece(slot, 2, u);
         float4 w = kTwo ? *piece(slot, 3, u) : make_float4(0.f, 0.f, 0.f, 0.f);
-        const float4 c = *piece(slot, NS - 1, u);
+        const float4 c = *piece(slot, STALE ? NS - 2 : NS - 1, u);  // the center the replicas see
         const float4 r = ea_vec<OPT>(x, g, m, w, c, hp, sc);
         mem.st(xi + 4 * v, x);
         mem.st(mi + 4 * v, m);
         if constexpr (kTwo) mem.st(vi + 4 * v, w);
-        if constexpr (N == 1) mem.st(st.c + 4 * v, center_apply(c, r, hp.inv_n));
-        else s_r[(par * N + rep) * TV + col] = r;
+        if constexpr (N == 1) {
+          const float4 ct = STALE ? *piece(slot, NS - 1, u) : c;
+          mem.st(st.c + 4 * v, center_apply(ct, r, hp.inv_n));
+          if constexpr (STALE) mem.st(st.prev + 4 * v, ct);
+        } else {
+          s_r[(par * N + rep) * TV + col] = r;
+        }
       }
     }
     if constexpr (N > 1) {
@@ -490,7 +499,9 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warp
           float4 acc = s_r[(par * N) * TV + col];
 #pragma unroll
           for (int i = 1; i < N; ++i) add4(acc, s_r[(par * N + i) * TV + col]);
-          mem.st(st.c + 4 * (v0 + col), center_apply(*piece(slot, NS - 1, u), acc, hp.inv_n));
+          const float4 ct = *piece(slot, NS - 1, u);  // x~_t
+          mem.st(st.c + 4 * (v0 + col), center_apply(ct, acc, hp.inv_n));
+          if constexpr (STALE) mem.st(st.prev + 4 * (v0 + col), ct);
         }
       }
       par ^= 1;  // the next tile writes the other buffer; the one after waits behind the next barrier
@@ -499,7 +510,7 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S>::W) colocated_warp
   }
   cp_async_wait<0>();
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT>(b.st[t], hp);
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
 template <int U>
@@ -1192,13 +1203,13 @@ int ring_geom() {
   return v;
 }
 
-template <int N, int OPT, int U, int S>
+template <int N, int OPT, int U, int S, bool STALE = false>
 cudaError_t launch_warpring_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using RG = RingGeom<N, OPT, U, S>;
+  using RG = RingGeom<N, OPT, U, S, STALE>;
   if constexpr (RG::kSmemBytes > 227 * 1024) {
     return cudaErrorInvalidConfiguration;
   } else {
-    auto k = colocated_warpring<N, OPT, U, S>;
+    auto k = colocated_warpring<N, OPT, U, S, STALE>;
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
     if (e != cudaSuccess) return e;
     const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
@@ -1207,8 +1218,9 @@ cudaError_t launch_warpring_t(const StageBatch& b, const Hyper& hp, int num_sms,
   }
 }
 
-template <int N, int OPT>
+template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warpring(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  if constexpr (STALE) return launch_warpring_t<N, OPT, 1, 4, true>(b, hp, num_sms, s);
   switch (ring_geom()) {
     case 16: return launch_warpring_t<N, OPT, 1, 6>(b, hp, num_sms, s);
     case 18: return launch_warpring_t<N, OPT, 1, 8>(b, hp, num_sms, s);
@@ -1428,6 +1440,16 @@ cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int nu
 }
 
 template <int N>
+cudaError_t launch_stale_warpring_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
+  switch (opt) {
+    case kOptAdam: return launch_warpring<N, kOptAdam, true>(b, hp, num_sms, s);
+    case kOptAdamW: return launch_warpring<N, kOptAdamW, true>(b, hp, num_sms, s);
+    case kOptASGD: return launch_warpring<N, kOptASGD, true>(b, hp, num_sms, s);
+    default: return launch_warpring<N, kOptSGD, true>(b, hp, num_sms, s);
+  }
+}
+
+template <int N>
 cudaError_t launch_stale_warprep_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
   switch (opt) {
     case kOptAdam: return launch_warprep<N, kOptAdam, true>(b, hp, num_sms, s);
@@ -1445,6 +1467,19 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
   // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
   if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
+  if (variant == kVariantWarpRing) {
+    switch (n) {
+      case 1: return launch_stale_warpring_n<1>(b, hp, opt, num_sms, s);
+      case 2: return launch_stale_warpring_n<2>(b, hp, opt, num_sms, s);
+      case 3: return launch_stale_warpring_n<3>(b, hp, opt, num_sms, s);
+      case 4: return launch_stale_warpring_n<4>(b, hp, opt, num_sms, s);
+      case 5: return launch_stale_warpring_n<5>(b, hp, opt, num_sms, s);
+      case 6: return launch_stale_warpring_n<6>(b, hp, opt, num_sms, s);
+      case 7: return launch_stale_warpring_n<7>(b, hp, opt, num_sms, s);
+      case 8: return launch_stale_warpring_n<8>(b, hp, opt, num_sms, s);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   if (variant == kVariantWarpRep) {
     switch (n) {
       case 1: return launch_stale_warprep_n<1>(b, hp, opt, num_sms, s);

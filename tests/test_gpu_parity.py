@@ -280,6 +280,16 @@ def test_warp_ring_geometries(n, geom, monkeypatch):
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
 
 
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+@pytest.mark.parametrize("n", [1, 2, 4, 5, 8])
+def test_warp_ring_stale(n, optimizer):
+    """Variant 6 with the stale center (row f4): x~_{t-1} streamed as one more ring stream, x~_t copied only where
+    a lane reduces; the reduction writes x~_{t+1} and rolls x~_{t-1} <- x~_t; several stages per launch."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096], 20, "combined", variants=("warpring",), many=True, optimizer=optimizer,
+                   lr=lr, staleness=1)
+
+
 def test_warp_ring_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warpring",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
