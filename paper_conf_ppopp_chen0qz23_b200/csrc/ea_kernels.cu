@@ -374,6 +374,21 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
+// Scalar tail of the spread local kernels (one thread): elements [4*(p/4), p) and the zero padding
+// [p, p_pad) of the contribution (reading c18: zero padding is a fixed point of the exchange).
+template <int OPT>
+__device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
+  const StepCoef sc = load_coef<OPT>(st.scp);
+  for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
+    float x = st.x[0][j], m = st.m[0][j], v = two_state(OPT) ? st.v[0][j] : 0.f;
+    contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
+    st.x[0][j] = x;
+    st.m[0][j] = m;
+    if (two_state(OPT)) st.v[0][j] = v;
+  }
+  for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
+}
+
 // ============================================================================
 // Variant 6: warp per replica with a cp.async ring.  The warp-per-replica kernel keeps a tile's loads in
 // registers, so with Adam's four streams per replica few bytes are in flight per SM while a CTA computes and
@@ -406,9 +421,12 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int K>
 __device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(K) : "memory"); }
 
-template <int N, int OPT, int U, int S, bool STALE = false>
-__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocated_warpring(const StageBatch b,
-                                                                                             const Hyper hp) {
+// SPREAD (N = 1, one stage): the spread layout's local step -- x~ only read, the contribution r stored to
+// `contrib` (zeros over the padding [p, p_pad)) for the reduce-scatter / peer exchange (rows a1-a4).
+template <int N, int OPT, int U, int S, bool STALE = false, bool SPREAD = false>
+__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocated_warpring(
+    const StageBatch b, const Hyper hp, float* __restrict__ contrib = nullptr, int64_t p_pad = 0) {
+  static_assert(!SPREAD || (N == 1 && !STALE), "spread: one replica, synchronous center");
   using RG = RingGeom<N, OPT, U, S, STALE>;
   constexpr int TV = RG::TV, NS = RG::NS;
   constexpr bool kTwo = two_state(OPT);
@@ -480,7 +498,9 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocat
         mem.st(xi + 4 * v, x);
         mem.st(mi + 4 * v, m);
         if constexpr (kTwo) mem.st(vi + 4 * v, w);
-        if constexpr (N == 1) {
+        if constexpr (SPREAD) {
+          mem.st(contrib + 4 * v, r);
+        } else if constexpr (N == 1) {
           const float4 ct = STALE ? *piece(slot, NS - 1, u) : c;
           mem.st(st.c + 4 * v, center_apply(ct, r, hp.inv_n));
           if constexpr (STALE) mem.st(st.prev + 4 * v, ct);
@@ -509,8 +529,12 @@ __global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocat
     slot = slot == S - 1 ? 0 : slot + 1;
   }
   cp_async_wait<0>();
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
+    if constexpr (SPREAD)
+      spread_tail<OPT>(b.st[0], contrib, p_pad, hp);
+    else
+      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
+  }
 }
 
 template <int U>
@@ -797,21 +821,6 @@ struct BulkGeom {
   static constexpr int kStages = kFit > kMaxBulkStages ? kMaxBulkStages : (kFit < 2 ? 2 : kFit);
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
-
-// Scalar tail of the spread bulk pipeline (one thread): elements [4*(p/4), p) and the zero padding
-// [p, p_pad) of the contribution (reading c18: zero padding is a fixed point of the exchange).
-template <int OPT>
-__device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
-  const StepCoef sc = load_coef<OPT>(st.scp);
-  for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
-    float x = st.x[0][j], m = st.m[0][j], v = two_state(OPT) ? st.v[0][j] : 0.f;
-    contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
-    st.x[0][j] = x;
-    st.m[0][j] = m;
-    if (two_state(OPT)) st.v[0][j] = v;
-  }
-  for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
-}
 
 // SPREAD = false: co-located stages (x~ updated in place).  SPREAD = true: the spread layout's local
 // step (N = 1, one stage): x~ is only read and the contribution r goes to `contrib` (rows a1-a4).
@@ -1213,7 +1222,7 @@ cudaError_t launch_warpring_t(const StageBatch& b, const Hyper& hp, int num_sms,
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
     if (e != cudaSuccess) return e;
     const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
-    k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp);
+    k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp, nullptr, 0);
     return cudaGetLastError();
   }
 }
@@ -1289,11 +1298,11 @@ cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, float* 
 }
 
 // Spread local kernel knob (measurement): AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel
-// (spread_local); default: the bulk-copy pipeline (spread_bulkpipe).
+// (spread_local), =ring the cp.async ring kernel; default: the bulk-copy pipeline (spread_bulkpipe).
 int spread_reg() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_SPREAD_KERNEL");
-    return (e && e[0] == 'r') ? 1 : 0;
+    return (e && e[0] == 'r' && e[1] == 'e') ? 1 : (e && e[0] == 'r' && e[1] == 'i') ? 2 : 0;
   }();
   return v;
 }
@@ -1339,10 +1348,37 @@ cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, con
   }
 }
 
+// Spread local step on the cp.async ring kernel (N = 1 geometry: 8 independent warps per CTA).
+template <int OPT>
+cudaError_t launch_spread_ring(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
+                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
+                               cudaStream_t s) {
+  using RG = RingGeom<1, OPT, 1, 4>;
+  auto k = colocated_warpring<1, OPT, 1, 4, false, true>;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
+  if (e != cudaSuccess) return e;
+  StageBatch b;
+  b.nstages = 1;
+  StageRefs& r = b.st[0];
+  for (int i = 0; i < kMaxFusedN; ++i) {
+    r.x[i] = i == 0 ? x : nullptr;
+    r.g[i] = i == 0 ? g : nullptr;
+    r.m[i] = i == 0 ? m : nullptr;
+    r.v[i] = i == 0 ? v : nullptr;
+  }
+  r.c = const_cast<float*>(center);  // read only (SPREAD)
+  r.p = p;
+  r.scp = sc;
+  const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
+  k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp, contrib, p_pad);
+  return cudaGetLastError();
+}
+
 template <int OPT>
 cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
                                     float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
+  if (spread_reg() == 2) return launch_spread_ring<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   if (!spread_reg()) return launch_spread_bulk<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   constexpr int U = two_state(OPT) ? 2 : 4;
   const int64_t nvec = p / 4;

@@ -408,6 +408,22 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 
         h.close()
 
 
+@pytest.mark.parametrize("kernel", ["ring", "reg"])
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "asgd"])
+def test_spread_local_kernel_variants(kernel, optimizer):
+    """The spread local step on the other kernels behind AVGPIPE_EA_SPREAD_KERNEL (ring: the cp.async ring kernel
+    with the contribution to the exchange buffer and the padding zeroed; reg: the register kernel), 4 virtual ranks
+    (the knob is read once per process: a subprocess per case)."""
+    import subprocess
+    import sys
+    code = ("import tests.test_gpu_parity as t; "
+            f"t.test_spread_decomposition_virtual_ranks(4, 'combined', '{optimizer}', sizes=(1_000_003, 200_003, 64), "
+            "steps=12)")
+    env = dict(os.environ, AVGPIPE_EA_SPREAD_KERNEL=kernel)
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
 @pytest.mark.parametrize("n,mode", [(2, m) for m in synth.MODES] + [(4, m) for m in synth.MODES] + [(8, "combined")])
 def test_spread_decomposition_c1_100_steps(n, mode):
     """North-star gate for the NCCL layout's kernels: C1 + tail stage, 100 steps, N = 2/4/8 virtual ranks."""
