@@ -224,7 +224,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
         name = "colocated_wide"
     elif two_state:
         if variant == "auto":
-            variant = "laneshfl" if n == 1 else ("regloop" if n <= 3 else ("bulkpipe" if n == 4 else "split"))
+            variant = ("laneshfl" if n == 1 else "regloop" if n <= 3 else "bulkpipe" if n == 4 else
+                       "warprep" if n == 5 else "split")
         name = "colocated_" + variant
     elif variant == "auto":   # ea_kernels.cu: SGD / ASGD warp per replica except N = 2 (lane kernel)
         name = "colocated_laneshfl" if n == 2 else "colocated_warprep"

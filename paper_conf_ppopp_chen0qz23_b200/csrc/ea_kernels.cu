@@ -1177,12 +1177,13 @@ cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cuda
   return cudaGetLastError();
 }
 
-// Warp per replica (variant 5): U float4 columns per lane and tile (SGD/ASGD 4: 2 KB rows per stream per tile;
-// Adam(W) 2 by default, for registers; measurement knob AVGPIPE_EA_WARPREP_U=4 gives Adam(W) 4 as well).
+// Warp per replica (variant 5): U = 4 float4 columns per lane and tile (2 KB rows per stream per tile), every
+// optimizer (Adam(W) with U = 4, round 2 session g/h: N = 5 0.974 vs 0.69-0.87 with U = 2); measurement knob
+// AVGPIPE_EA_WARPREP_U=2 gives Adam(W) U = 2.
 int warprep_u4() {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_WARPREP_U");
-    return (e && e[0] == '4') ? 1 : 0;
+    return (e && e[0] == '2') ? 0 : 1;
   }();
   return v;
 }
@@ -1431,8 +1432,12 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // N = 5, 6 (round 2, same box: 0.950 / 0.930 vs 0.930 / 0.906 for the bulk pipeline); N > 6 goes to the
   // replica-loop kernel (ea_api.cu).  ASGD: SGD's choice except the split register loop for N = 5, 6 (0.967 /
   // 0.941 vs 0.920 / 0.937; profiles/r02_sweep_split.jsonl -- with SGD it measured below the bulk pipeline).
+  // Round 2 session h (same box, C2 sizes): Adam N = 5 on the warp-per-replica kernel with U = 4, 0.974 (session
+  // g) / split 0.944-0.950; N = 2, 3 within 1% of the register loop (0.960 / 0.941 vs 0.948 / 0.940), kept.
   if (variant == kVariantAuto && two_state(opt))
-    variant = n == 1 ? kVariantLaneShfl : (n <= 3 ? kVariantRegLoop : (n == 4 ? kVariantBulkPipe : kVariantSplit));
+    variant = n == 1 ? kVariantLaneShfl
+                     : (n <= 3 ? kVariantRegLoop
+                               : (n == 4 ? kVariantBulkPipe : (n == 5 ? kVariantWarpRep : kVariantSplit)));
   // SGD-momentum and ASGD (one state vector), round 2: the warp-per-replica kernel for N = 1 and 3..8 (same box,
   // C2 sizes: N = 1 0.937 vs 0.872 bulk pipeline, N = 3 0.986 vs 0.932 lane, N = 4 0.996-0.998 vs 0.983 lane,
   // N = 5..8 0.979-1.0 vs 0.93-0.976; ASGD alike), the lane kernel for N = 2 (0.963 vs 0.952);
