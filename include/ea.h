@@ -123,9 +123,7 @@ typedef struct {
                                    tile by cp.async.bulk into an mbarrier ring), 4 = split
                                    register loop (two lanes per center column, N/2 replicas
                                    each, shuffle reduction), 5 = warp per replica (contributions
-                                   reduced through shared memory), 6 = warp per replica with its
-                                   inputs streamed through a per-lane cp.async ring (x~_{t-1} as
-                                   one more stream with staleness 1).  Same results
+                                   reduced through shared memory).  Same results
                                    up to fp32 summation order (DESIGN.md c14); the default picks per N and optimizer
                                    (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */
@@ -345,7 +343,12 @@ EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance,
  * buffer or the wrong end -> EA_EINVAL; not connected, or the stream is capturing a CUDA graph (the slot and
  * round are host counters) -> EA_ESTATE; CUDA / driver failures -> EA_ECUDA.  Nothing is enqueued on error.
  * ea_chan_destroy synchronises the device, closes the peer mapping and frees this end's buffer: both ends
- * must be past their last operation (a caller-side barrier) before either is destroyed. */
+ * must be past their last operation (a caller-side barrier) before either is destroyed.
+ * Caution: a stream that waits for a message blocks until the peer sends it; anything that synchronises the
+ * whole context meanwhile (cudaDeviceSynchronize, and the FIRST launch of a kernel under CUDA's lazy module
+ * loading) waits for it too.  If the peer sends that message only after this process enqueues more work, use
+ * CUDA_MODULE_LOADING=EAGER (the pipeline runtime requires it) and no device-wide synchronisation while
+ * messages are outstanding. */
 typedef struct ea_chan_s* ea_chan;
 EA_API ea_status ea_chan_create(int32_t device, int32_t role /* 0 = send, 1 = recv */, int64_t slot_bytes,
                                 int32_t slots, ea_chan* out);

@@ -99,7 +99,6 @@ enum KernelVariant : int {
                          // ring (producer warp + mbarriers); consumers store from registers (SGD)
   kVariantSplit = 4,     // split register loop: 2 lanes per center column, N/2 replicas each, shuffle reduction
   kVariantWarpRep = 5,   // warp per replica, 512 B rows, contributions reduced through shared memory
-  kVariantWarpRing = 6,  // warp per replica, inputs streamed through a per-lane cp.async ring in shared memory
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N
@@ -112,7 +111,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
 // lane kernel with x~_{t-1} staged beside x~_t, for N = 1 and 5 the bulk-copy pipeline with x~_{t-1} as one more
 // stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
 constexpr int kMaxStaleLaneN = 4;
-// variant kVariantWarpRep / kVariantWarpRing: the warp-per-replica kernels with x~_{t-1} for any N <= kMaxFusedN.
+// variant kVariantWarpRep: the warp-per-replica kernel with x~_{t-1} for any N <= kMaxFusedN.
 cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int variant,
                                          int num_sms, cudaStream_t s);
 

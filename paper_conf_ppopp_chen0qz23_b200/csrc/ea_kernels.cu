@@ -374,169 +374,6 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
-// Scalar tail of the spread local kernels (one thread): elements [4*(p/4), p) and the zero padding
-// [p, p_pad) of the contribution (reading c18: zero padding is a fixed point of the exchange).
-template <int OPT>
-__device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
-  const StepCoef sc = load_coef<OPT>(st.scp);
-  for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
-    float x = st.x[0][j], m = st.m[0][j], v = two_state(OPT) ? st.v[0][j] : 0.f;
-    contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
-    st.x[0][j] = x;
-    st.m[0][j] = m;
-    if (two_state(OPT)) st.v[0][j] = v;
-  }
-  for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
-}
-
-// ============================================================================
-// Variant 6: warp per replica with a cp.async ring.  The warp-per-replica kernel keeps a tile's loads in
-// registers, so with Adam's four streams per replica few bytes are in flight per SM while a CTA computes and
-// waits at its barrier (0.69-0.87 of peak).  Here every lane copies ITS OWN 16-byte pieces of the next S-1
-// tiles (x, g, the optimizer state and x~) into shared memory with cp.async (LDGSTS: no registers held while in
-// flight) and reads back only what it copied itself -- so the ring needs no barrier and no mbarrier, only
-// cp.async.wait_group; the one block-level exchange left is the replica reduction of the contributions
-// (double-buffered, one named barrier per column group and tile).
-// CTA = G column groups x N warps; warp w: replica i = w % N, group q = w / N; a tile is G x 32U float4 columns.
-// In the reduction thread (q, i, lane) owns the columns u*32 + lane of its group with u = i (mod N), whose x~
-// it copied itself.
-// ============================================================================
-// STALE (row f4, reading c28): one more stream, x~_{t-1} (what the replicas see); x~_t is then copied only for
-// the columns the lane reduces, and the reduction writes x~_{t+1} and rolls x~_{t-1} <- x~_t.
-template <int N, int OPT, int U, int S, bool STALE = false>
-struct RingGeom {
-  static constexpr int G = N >= 8 ? 1 : 8 / N;           // column groups per CTA
-  static constexpr int W = N * G;                         // warps
-  static constexpr int NS = (two_state(OPT) ? 4 : 3) + 1 + (STALE ? 1 : 0);  // x, g, m, (v), (x~_{t-1}), x~_t
-  static constexpr int TV = G * 32 * U;                   // float4 columns per tile
-  static constexpr int kRingVec = S * W * NS * U * 32;
-  static constexpr int kRedVec = N > 1 ? 2 * N * TV : 0;
-  static constexpr int kSmemBytes = (kRingVec + kRedVec) * 16;
-};
-
-__device__ __forceinline__ void cp_async16(float4* dst, const float* src) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(smem_u32(dst)), "l"(src) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int K>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(K) : "memory"); }
-
-// SPREAD (N = 1, one stage): the spread layout's local step -- x~ only read, the contribution r stored to
-// `contrib` (zeros over the padding [p, p_pad)) for the reduce-scatter / peer exchange (rows a1-a4).
-template <int N, int OPT, int U, int S, bool STALE = false, bool SPREAD = false>
-__global__ void __launch_bounds__(32 * RingGeom<N, OPT, U, S, STALE>::W) colocated_warpring(
-    const StageBatch b, const Hyper hp, float* __restrict__ contrib = nullptr, int64_t p_pad = 0) {
-  static_assert(!SPREAD || (N == 1 && !STALE), "spread: one replica, synchronous center");
-  using RG = RingGeom<N, OPT, U, S, STALE>;
-  constexpr int TV = RG::TV, NS = RG::NS;
-  constexpr bool kTwo = two_state(OPT);
-  extern __shared__ __align__(16) float4 ring[];
-  float4* s_r = ring + RG::kRingVec;  // [2][N][TV] contributions (N > 1)
-  __shared__ StepCoef s_coef[kMaxLaunchStages];
-  const Mem<0> mem;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int rep = warp % N, grp = warp / N;
-  if (has_coef(OPT)) {
-    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
-    __syncthreads();
-  }
-  // this lane's piece of slot k, stream a, unroll u
-  auto piece = [&](int k, int a, int u) -> float4* {
-    return ring + ((k * RG::W + warp) * NS + a) * (U * 32) + u * 32 + lane;
-  };
-  auto issue = [&](int k, int s, int64_t v0, int64_t nv) {
-    const StageRefs& st = b.st[s];
-    const float* src[NS];
-    src[0] = st.x[rep];
-    src[1] = st.g[rep];
-    src[2] = st.m[rep];
-    if constexpr (kTwo) src[3] = st.v[rep];
-    if constexpr (STALE) src[NS - 2] = st.prev;
-    src[NS - 1] = st.c;
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int col = grp * 32 * U + u * 32 + lane;
-      if (col < nv) {
-        const int64_t v = v0 + col;
-#pragma unroll
-        for (int a = 0; a < NS; ++a)   // stale: x~_t only where this lane reduces
-          if (!STALE || a != NS - 1 || u % N == rep) cp_async16(piece(k, a, u), src[a] + 4 * v);
-      }
-    }
-  };
-  WaveCursor lc{0, 0}, cc{0, 0};
-  int s;
-  int64_t v0, nv;
-#pragma unroll
-  for (int k = 0; k < S - 1; ++k) {
-    if (wave_item(b, TV, lc, s, v0, nv)) issue(k, s, v0, nv);
-    cp_async_commit();
-  }
-  int slot = 0, par = 0;
-  while (wave_item(b, TV, cc, s, v0, nv)) {
-    {  // refill the slot this lane finished with in the previous tile (it reads only its own pieces)
-      int s2;
-      int64_t w0, wn;
-      if (wave_item(b, TV, lc, s2, w0, wn)) issue(slot == 0 ? S - 1 : slot - 1, s2, w0, wn);
-      cp_async_commit();
-    }
-    cp_async_wait<S - 1>();  // this lane's copies of the current tile have landed
-    const StageRefs& st = b.st[s];
-    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
-    float* xi = st.x[rep];
-    float* mi = st.m[rep];
-    float* vi = kTwo ? st.v[rep] : nullptr;
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int col = grp * 32 * U + u * 32 + lane;
-      if (col < nv) {
-        const int64_t v = v0 + col;
-        float4 x = *piece(slot, 0, u), g = *piece(slot, 1, u), m = *piece(slot, 2, u);
-        float4 w = kTwo ? *piece(slot, 3, u) : make_float4(0.f, 0.f, 0.f, 0.f);
-        const float4 c = *piece(slot, STALE ? NS - 2 : NS - 1, u);  // the center the replicas see
-        const float4 r = ea_vec<OPT>(x, g, m, w, c, hp, sc);
-        mem.st(xi + 4 * v, x);
-        mem.st(mi + 4 * v, m);
-        if constexpr (kTwo) mem.st(vi + 4 * v, w);
-        if constexpr (SPREAD) {
-          mem.st(contrib + 4 * v, r);
-        } else if constexpr (N == 1) {
-          const float4 ct = STALE ? *piece(slot, NS - 1, u) : c;
-          mem.st(st.c + 4 * v, center_apply(ct, r, hp.inv_n));
-          if constexpr (STALE) mem.st(st.prev + 4 * v, ct);
-        } else {
-          s_r[(par * N + rep) * TV + col] = r;
-        }
-      }
-    }
-    if constexpr (N > 1) {
-      asm volatile("bar.sync %0, %1;" ::"r"(1 + grp), "n"(32 * N) : "memory");  // this group's N warps
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        if (u % N != rep) continue;
-        const int col = grp * 32 * U + u * 32 + lane;
-        if (col < nv) {
-          float4 acc = s_r[(par * N) * TV + col];
-#pragma unroll
-          for (int i = 1; i < N; ++i) add4(acc, s_r[(par * N + i) * TV + col]);
-          const float4 ct = *piece(slot, NS - 1, u);  // x~_t
-          mem.st(st.c + 4 * (v0 + col), center_apply(ct, acc, hp.inv_n));
-          if constexpr (STALE) mem.st(st.prev + 4 * (v0 + col), ct);
-        }
-      }
-      par ^= 1;  // the next tile writes the other buffer; the one after waits behind the next barrier
-    }
-    slot = slot == S - 1 ? 0 : slot + 1;
-  }
-  cp_async_wait<0>();
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
-    if constexpr (SPREAD)
-      spread_tail<OPT>(b.st[0], contrib, p_pad, hp);
-    else
-      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
-  }
-}
-
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -822,6 +659,21 @@ struct BulkGeom {
   static constexpr int kSmemBytes = kStages * kSlotVec * 16 + 2 * kStages * 8;
 };
 
+// Scalar tail of the spread bulk pipeline (one thread): elements [4*(p/4), p) and the zero padding
+// [p, p_pad) of the contribution (reading c18: zero padding is a fixed point of the exchange).
+template <int OPT>
+__device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, const Hyper& hp) {
+  const StepCoef sc = load_coef<OPT>(st.scp);
+  for (int64_t j = (st.p / 4) * 4; j < st.p; ++j) {
+    float x = st.x[0][j], m = st.m[0][j], v = two_state(OPT) ? st.v[0][j] : 0.f;
+    contrib[j] = ea_elem<OPT>(x, st.g[0][j], m, v, st.c[j], hp, sc);
+    st.x[0][j] = x;
+    st.m[0][j] = m;
+    if (two_state(OPT)) st.v[0][j] = v;
+  }
+  for (int64_t j = st.p; j < p_pad; ++j) contrib[j] = 0.f;
+}
+
 // SPREAD = false: co-located stages (x~ updated in place).  SPREAD = true: the spread layout's local
 // step (N = 1, one stage): x~ is only read and the contribution r goes to `contrib` (rows a1-a4).
 // STALE (co-located, row f4, reading c28): every stage's x~_{t-1} (st.prev) is one more stream of the slot;
@@ -1027,9 +879,9 @@ int grid_knob() {
 }
 
 template <typename K>
-int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads, size_t smem = 0) {
+int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads) {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess || per_sm < 1)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0) != cudaSuccess || per_sm < 1)
     per_sm = 1;
   int64_t grid = (int64_t)num_sms * per_sm;
   const int knob = grid_knob();
@@ -1178,7 +1030,7 @@ cudaError_t launch_split(const StageBatch& b, const Hyper& hp, int num_sms, cuda
 }
 
 // Warp per replica (variant 5): U = 4 float4 columns per lane and tile (2 KB rows per stream per tile), every
-// optimizer (Adam(W) with U = 4, round 2 session g/h: N = 5 0.974 vs 0.69-0.87 with U = 2); measurement knob
+// optimizer (Adam(W) with U = 4, round 2 sessions g/h: N = 5 0.974 vs 0.69-0.87 with U = 2); measurement knob
 // AVGPIPE_EA_WARPREP_U=2 gives Adam(W) U = 2.
 int warprep_u4() {
   static const int v = [] {
@@ -1203,53 +1055,8 @@ cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_warprep_u<N, OPT, 4, STALE>(b, hp, num_sms, s);
 }
 
-// Warp per replica with a cp.async ring (variant 6): U float4 columns per lane and tile, S tiles in the ring.
-// Measurement knob AVGPIPE_EA_RING = <U><S>: 14 (default), 16, 18, 24, 23.
-int ring_geom() {
-  static const int v = [] {
-    const char* e = std::getenv("AVGPIPE_EA_RING");
-    return e ? std::atoi(e) : 14;
-  }();
-  return v;
-}
-
-template <int N, int OPT, int U, int S, bool STALE = false>
-cudaError_t launch_warpring_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  using RG = RingGeom<N, OPT, U, S, STALE>;
-  if constexpr (RG::kSmemBytes > 227 * 1024) {
-    return cudaErrorInvalidConfiguration;
-  } else {
-    auto k = colocated_warpring<N, OPT, U, S, STALE>;
-    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
-    if (e != cudaSuccess) return e;
-    const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
-    k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp, nullptr, 0);
-    return cudaGetLastError();
-  }
-}
-
-template <int N, int OPT, bool STALE = false>
-cudaError_t launch_warpring(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  if constexpr (STALE) return launch_warpring_t<N, OPT, 1, 4, true>(b, hp, num_sms, s);
-  switch (ring_geom()) {
-    case 16: return launch_warpring_t<N, OPT, 1, 6>(b, hp, num_sms, s);
-    case 18: return launch_warpring_t<N, OPT, 1, 8>(b, hp, num_sms, s);
-    case 24: return launch_warpring_t<N, OPT, 2, 4>(b, hp, num_sms, s);
-    case 23: return launch_warpring_t<N, OPT, 2, 3>(b, hp, num_sms, s);
-    default: return launch_warpring_t<N, OPT, 1, 4>(b, hp, num_sms, s);
-  }
-}
-
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
-  if (variant == kVariantWarpRing) {
-    switch (opt) {
-      case kOptAdam: return launch_warpring<N, kOptAdam>(b, hp, num_sms, s);
-      case kOptAdamW: return launch_warpring<N, kOptAdamW>(b, hp, num_sms, s);
-      case kOptASGD: return launch_warpring<N, kOptASGD>(b, hp, num_sms, s);
-      default: return launch_warpring<N, kOptSGD>(b, hp, num_sms, s);
-    }
-  }
   if (variant == kVariantWarpRep) {
     switch (opt) {
       case kOptAdam: return launch_warprep<N, kOptAdam>(b, hp, num_sms, s);
@@ -1299,11 +1106,11 @@ cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, float* 
 }
 
 // Spread local kernel knob (measurement): AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel
-// (spread_local), =ring the cp.async ring kernel; default: the bulk-copy pipeline (spread_bulkpipe).
+// (spread_local); default: the bulk-copy pipeline (spread_bulkpipe).
 int spread_reg() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_SPREAD_KERNEL");
-    return (e && e[0] == 'r' && e[1] == 'e') ? 1 : (e && e[0] == 'r' && e[1] == 'i') ? 2 : 0;
+    return (e && e[0] == 'r') ? 1 : 0;
   }();
   return v;
 }
@@ -1349,37 +1156,10 @@ cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, con
   }
 }
 
-// Spread local step on the cp.async ring kernel (N = 1 geometry: 8 independent warps per CTA).
-template <int OPT>
-cudaError_t launch_spread_ring(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
-                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
-                               cudaStream_t s) {
-  using RG = RingGeom<1, OPT, 1, 4>;
-  auto k = colocated_warpring<1, OPT, 1, 4, false, true>;
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, RG::kSmemBytes);
-  if (e != cudaSuccess) return e;
-  StageBatch b;
-  b.nstages = 1;
-  StageRefs& r = b.st[0];
-  for (int i = 0; i < kMaxFusedN; ++i) {
-    r.x[i] = i == 0 ? x : nullptr;
-    r.g[i] = i == 0 ? g : nullptr;
-    r.m[i] = i == 0 ? m : nullptr;
-    r.v[i] = i == 0 ? v : nullptr;
-  }
-  r.c = const_cast<float*>(center);  // read only (SPREAD)
-  r.p = p;
-  r.scp = sc;
-  const int grid = persistent_grid(k, units_of(b, RG::TV), num_sms, 32 * RG::W, RG::kSmemBytes);
-  k<<<grid, 32 * RG::W, RG::kSmemBytes, s>>>(b, hp, contrib, p_pad);
-  return cudaGetLastError();
-}
-
 template <int OPT>
 cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
                                     float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
-  if (spread_reg() == 2) return launch_spread_ring<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   if (!spread_reg()) return launch_spread_bulk<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   constexpr int U = two_state(OPT) ? 2 : 4;
   const int64_t nvec = p / 4;
@@ -1481,16 +1261,6 @@ cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int nu
 }
 
 template <int N>
-cudaError_t launch_stale_warpring_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
-  switch (opt) {
-    case kOptAdam: return launch_warpring<N, kOptAdam, true>(b, hp, num_sms, s);
-    case kOptAdamW: return launch_warpring<N, kOptAdamW, true>(b, hp, num_sms, s);
-    case kOptASGD: return launch_warpring<N, kOptASGD, true>(b, hp, num_sms, s);
-    default: return launch_warpring<N, kOptSGD, true>(b, hp, num_sms, s);
-  }
-}
-
-template <int N>
 cudaError_t launch_stale_warprep_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
   switch (opt) {
     case kOptAdam: return launch_warprep<N, kOptAdam, true>(b, hp, num_sms, s);
@@ -1508,19 +1278,6 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
   // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
   if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
-  if (variant == kVariantWarpRing) {
-    switch (n) {
-      case 1: return launch_stale_warpring_n<1>(b, hp, opt, num_sms, s);
-      case 2: return launch_stale_warpring_n<2>(b, hp, opt, num_sms, s);
-      case 3: return launch_stale_warpring_n<3>(b, hp, opt, num_sms, s);
-      case 4: return launch_stale_warpring_n<4>(b, hp, opt, num_sms, s);
-      case 5: return launch_stale_warpring_n<5>(b, hp, opt, num_sms, s);
-      case 6: return launch_stale_warpring_n<6>(b, hp, opt, num_sms, s);
-      case 7: return launch_stale_warpring_n<7>(b, hp, opt, num_sms, s);
-      case 8: return launch_stale_warpring_n<8>(b, hp, opt, num_sms, s);
-      default: return cudaErrorInvalidValue;
-    }
-  }
   if (variant == kVariantWarpRep) {
     switch (n) {
       case 1: return launch_stale_warprep_n<1>(b, hp, opt, num_sms, s);

@@ -103,10 +103,18 @@ class PipelineStage:
         ends toward the previous stage), M slots of act_bytes each -- a sender never waits for a free slot, as at
         most M messages of one direction are in flight per iteration.  The IPC handles travel once over the
         stage process group (all_gather_object); every end then maps its peer's buffer."""
+        import os
         import torch
         import torch.distributed as dist
         if act_bytes <= 0:
             raise ValueError("transport 'ipc' needs act_bytes (bytes of the largest activation message)")
+        if os.environ.get("CUDA_MODULE_LOADING", "LAZY").upper() != "EAGER":
+            # a stream of this process may wait on the GPU for a message the peer sends only after this process
+            # enqueued more work; with lazy loading, the first launch of a kernel synchronises the context and
+            # would wait for that stream -> deadlock across the two processes
+            raise RuntimeError("transport 'ipc' needs CUDA_MODULE_LOADING=EAGER in the environment before CUDA "
+                               "is initialised (lazy kernel loading synchronises the context, which cannot finish "
+                               "while a stream waits on the GPU for the peer stage's message)")
         dev = torch.device(device) if device is not None else torch.device("cuda", torch.cuda.current_device())
         mine = {}
         for i in range(self.N):

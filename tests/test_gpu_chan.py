@@ -66,6 +66,9 @@ def test_sender_waits_for_a_free_slot():
     s_send, s_recv = torch.cuda.Stream(), torch.cuda.Stream()
     msgs = [torch.full((1024,), float(k + 1), device="cuda") for k in range(6)]
     outs = [torch.zeros(1024, device="cuda") for _ in range(6)]
+    # load the sleep kernel now: CUDA's lazy module loading synchronises the context to load a kernel, which
+    # cannot finish while s_send waits for the receiver (include/ea.h, "Activation channels")
+    torch.cuda._sleep(1)
     torch.cuda.synchronize()
     for k in range(6):
         snd.send(msgs[k], stream=s_send)   # sends 2..5 wait on the GPU for acknowledgements
@@ -117,6 +120,7 @@ def test_channel_errors():
 
 def _ipc_worker(rank, port, q, n_msgs):
     import torch.distributed as dist
+    os.environ["CUDA_MODULE_LOADING"] = "EAGER"   # before this process initialises CUDA (see pipeline.py)
     try:
         torch.cuda.set_device(0)
         dist.init_process_group("gloo", init_method=port, rank=rank, world_size=2)

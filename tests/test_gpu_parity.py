@@ -254,47 +254,6 @@ def test_warp_per_replica_stale(n, optimizer):
                    lr=lr, staleness=1)
 
 
-@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
-@pytest.mark.parametrize("n", [1, 2, 3, 4, 5, 6, 7, 8])
-def test_warp_ring(n, optimizer):
-    """Variant 6 (warp per replica, inputs through a per-lane cp.async ring, contributions reduced through
-    shared memory): C1-sized and ragged stages in one launch (several ring refills per CTA, ragged last tiles,
-    the scalar tails), every optimizer."""
-    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
-    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 12, "combined", variants=("warpring",), many=True,
-                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
-
-
-@pytest.mark.parametrize("geom", ["16", "18", "24", "23"])
-@pytest.mark.parametrize("n", [1, 3, 8])
-def test_warp_ring_geometries(n, geom, monkeypatch):
-    """The ring geometries behind the measurement knob AVGPIPE_EA_RING (read once per process, so each case
-    runs in a subprocess)."""
-    import subprocess
-    import sys
-    code = ("import tests.test_gpu_parity as t; "
-            f"t._run_colocated({n}, [100_003, 7, 4096, 1_000_001], 6, 'combined', variants=('warpring',), many=True, "
-            "optimizer='adam', lr=1e-3, wd=1e-2)")
-    env = dict(os.environ, AVGPIPE_EA_RING=geom)
-    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
-
-
-@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
-@pytest.mark.parametrize("n", [1, 2, 4, 5, 8])
-def test_warp_ring_stale(n, optimizer):
-    """Variant 6 with the stale center (row f4): x~_{t-1} streamed as one more ring stream, x~_t copied only where
-    a lane reduces; the reduction writes x~_{t+1} and rolls x~_{t-1} <- x~_t; several stages per launch."""
-    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
-    _run_colocated(n, [100_003, 7, 4096], 20, "combined", variants=("warpring",), many=True, optimizer=optimizer,
-                   lr=lr, staleness=1)
-
-
-def test_warp_ring_c1_100_steps():
-    _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warpring",), many=True, optimizer="adam",
-                   lr=1e-3, wd=1e-2)
-
-
 def test_warp_per_replica_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warprep",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
@@ -408,12 +367,11 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 
         h.close()
 
 
-@pytest.mark.parametrize("kernel", ["ring", "reg"])
+@pytest.mark.parametrize("kernel", ["reg"])
 @pytest.mark.parametrize("optimizer", ["sgd", "adam", "asgd"])
 def test_spread_local_kernel_variants(kernel, optimizer):
-    """The spread local step on the other kernels behind AVGPIPE_EA_SPREAD_KERNEL (ring: the cp.async ring kernel
-    with the contribution to the exchange buffer and the padding zeroed; reg: the register kernel), 4 virtual ranks
-    (the knob is read once per process: a subprocess per case)."""
+    """The spread local step on the register kernel behind AVGPIPE_EA_SPREAD_KERNEL=reg (the contribution to the
+    exchange buffer, the padding zeroed), 4 virtual ranks (the knob is read once per process: a subprocess)."""
     import subprocess
     import sys
     code = ("import tests.test_gpu_parity as t; "

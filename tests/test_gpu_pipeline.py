@@ -49,6 +49,8 @@ def _flatten(mod, device):
 
 
 def _worker(rank, port, q, concurrent=False, backend="gloo", transport="dist"):
+    if transport == "ipc":
+        os.environ["CUDA_MODULE_LOADING"] = "EAGER"   # required by the ipc transport (pipeline.py), before CUDA init
     try:
         dev = torch.device("cuda", rank if backend == "nccl" else 0)
         torch.cuda.set_device(dev)
