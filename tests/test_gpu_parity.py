@@ -254,6 +254,32 @@ def test_warp_per_replica_stale(n, optimizer):
                    lr=lr, staleness=1)
 
 
+@pytest.mark.parametrize("knobs", ["AVGPIPE_EA_WARPREP_PF=1", "AVGPIPE_EA_WARPREP_PF=1 AVGPIPE_EA_WARPREP_U=2",
+                                   "AVGPIPE_EA_WARPREP_U=2"])
+def test_warp_per_replica_knobs(knobs):
+    """The software-pipelined warp-per-replica kernel (next tile's loads in flight through the barrier and the
+    reduction, double-buffered contributions) and the U = 2 geometry behind their measurement knobs: every
+    optimizer, N = 1..8, ragged stages in one launch, and the stale center (the knobs are read once per process:
+    a subprocess)."""
+    import subprocess
+    import sys
+    code = ("import tests.test_gpu_parity as t\n"
+            "for opt in ('sgd', 'adam', 'adamw', 'asgd'):\n"
+            "    lr = 1e-3 if opt in ('adam', 'adamw') else t.synth.LR\n"
+            "    for n in range(1, 9):\n"
+            "        t._run_colocated(n, [100_003, 7, 4096, 300_001], 8, 'combined', variants=('warprep',), many=True,"
+            " optimizer=opt, lr=lr, wd=0.0 if opt == 'sgd' else 1e-2)\n"
+            "    for n in (2, 5, 8):\n"
+            "        t._run_colocated(n, [100_003, 7, 4096], 8, 'combined', variants=('warprep',), many=True,"
+            " optimizer=opt, lr=lr, staleness=1)\n")
+    env = dict(os.environ)
+    for kv in knobs.split():
+        k, v = kv.split("=")
+        env[k] = v
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=env, capture_output=True, text=True, timeout=1200)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+
+
 def test_warp_per_replica_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warprep",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
