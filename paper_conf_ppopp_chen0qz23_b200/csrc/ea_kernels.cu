@@ -374,89 +374,6 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
-// Variant 5 with a software pipeline (measurement knob AVGPIPE_EA_WARPREP_PF=1): each warp issues the loads of
-// its NEXT tile before the block barrier and the replica reduction of the current one, so a CTA keeps bytes in
-// flight through its barrier and reduction phases (the plain kernel has none in flight there); the contributions
-// are double-buffered in shared memory, one barrier per tile.
-template <int N, int OPT, int U, bool STALE = false>
-__global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep_pf(const StageBatch b, const Hyper hp) {
-  constexpr int TV = 32 * U;
-  constexpr bool kTwo = two_state(OPT);
-  __shared__ __align__(16) float4 s_r[2][N][TV];
-  __shared__ StepCoef s_coef[kMaxLaunchStages];
-  const Mem<0> mem;
-  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (has_coef(OPT)) {
-    if (threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
-    __syncthreads();
-  }
-  float4 x[U], g[U], m[U], w[U], c[U];
-  auto load = [&](int s, int64_t v0, int64_t nv) {
-    const StageRefs& st = b.st[s];
-    const float* xi = st.x[warp];
-    const float* gi = st.g[warp];
-    const float* mi = st.m[warp];
-    const float* vi = kTwo ? st.v[warp] : nullptr;
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int lv = u * 32 + lane;
-      if (lv < nv) {
-        const int64_t v = v0 + lv;
-        x[u] = mem.ld(xi + 4 * v);
-        g[u] = mem.ld_ro(gi + 4 * v);
-        m[u] = mem.ld(mi + 4 * v);
-        if (kTwo) w[u] = mem.ld(vi + 4 * v);
-        c[u] = __ldg(reinterpret_cast<const float4*>(STALE ? st.prev : st.c) + v);
-      }
-    }
-  };
-  WaveCursor cur{0, 0};
-  int s;
-  int64_t v0, nv;
-  bool have = wave_item(b, TV, cur, s, v0, nv);
-  if (have) load(s, v0, nv);
-  int par = 0;
-  while (have) {
-    const StageRefs& st = b.st[s];
-    const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
-    float* xi = st.x[warp];
-    float* mi = st.m[warp];
-    float* vi = kTwo ? st.v[warp] : nullptr;
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      const int lv = u * 32 + lane;
-      if (lv < nv) {
-        const int64_t v = v0 + lv;
-        s_r[par][warp][lv] = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
-        mem.st(xi + 4 * v, x[u]);
-        mem.st(mi + 4 * v, m[u]);
-        if (kTwo) mem.st(vi + 4 * v, w[u]);
-      }
-    }
-    int s2;
-    int64_t w0, wn;
-    const bool have2 = wave_item(b, TV, cur, s2, w0, wn);
-    if (have2) load(s2, w0, wn);  // next tile in flight through the barrier and the reduction
-    __syncthreads();
-    for (int col = threadIdx.x; col < nv; col += 32 * N) {
-      float4 acc = s_r[par][0][col];
-#pragma unroll
-      for (int i = 1; i < N; ++i) add4(acc, s_r[par][i][col]);
-      const int64_t v = v0 + col;
-      const float4 cv = __ldg(reinterpret_cast<const float4*>(st.c) + v);
-      mem.st(st.c + 4 * v, center_apply(cv, acc, hp.inv_n));
-      if (STALE) mem.st(st.prev + 4 * v, cv);
-    }
-    par ^= 1;  // the next tile fills the other buffer; this one is refilled only after the next barrier
-    s = s2;
-    v0 = w0;
-    nv = wn;
-    have = have2;
-  }
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
-    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
-}
-
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -1123,22 +1040,8 @@ int warprep_u4() {
   return v;
 }
 
-// Software-pipelined warp-per-replica kernel (measurement knob AVGPIPE_EA_WARPREP_PF=1).
-int warprep_pf() {
-  static const int v = [] {
-    const char* e = std::getenv("AVGPIPE_EA_WARPREP_PF");
-    return (e && e[0] == '1') ? 1 : 0;
-  }();
-  return v;
-}
-
 template <int N, int OPT, int U, bool STALE>
 cudaError_t launch_warprep_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  if (warprep_pf()) {
-    auto k = colocated_warprep_pf<N, OPT, U, STALE>;
-    k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
-    return cudaGetLastError();
-  }
   auto k = colocated_warprep<N, OPT, U, STALE>;
   k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
   return cudaGetLastError();

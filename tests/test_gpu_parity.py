@@ -254,13 +254,10 @@ def test_warp_per_replica_stale(n, optimizer):
                    lr=lr, staleness=1)
 
 
-@pytest.mark.parametrize("knobs", ["AVGPIPE_EA_WARPREP_PF=1", "AVGPIPE_EA_WARPREP_PF=1 AVGPIPE_EA_WARPREP_U=2",
-                                   "AVGPIPE_EA_WARPREP_U=2"])
+@pytest.mark.parametrize("knobs", ["AVGPIPE_EA_WARPREP_U=2"])
 def test_warp_per_replica_knobs(knobs):
-    """The software-pipelined warp-per-replica kernel (next tile's loads in flight through the barrier and the
-    reduction, double-buffered contributions) and the U = 2 geometry behind their measurement knobs: every
-    optimizer, N = 1..8, ragged stages in one launch, and the stale center (the knobs are read once per process:
-    a subprocess)."""
+    """The U = 2 geometry of the warp-per-replica kernel behind its measurement knob: every optimizer, N = 1..8,
+    ragged stages in one launch, and the stale center (the knob is read once per process: a subprocess)."""
     import subprocess
     import sys
     code = ("import tests.test_gpu_parity as t\n"
