@@ -44,6 +44,23 @@ from typing import Callable, List, Optional, Sequence
 from .binding import AdvanceController, Channel, schedule
 
 
+def wait_streams(streams, timeout_s: float, what: str = "streams"):
+    """Host wait for CUDA streams with a deadline (failure detection for the activation channels: a stream that
+    waits on the GPU for a message the peer stage never sends -- it died or stalled -- would make synchronize()
+    block forever).  Raises TimeoutError naming `what`; the streams stay blocked."""
+    import torch
+    evs = []
+    for s in streams:
+        e = torch.cuda.Event()
+        e.record(s)
+        evs.append(e)
+    t0 = time.monotonic()
+    while not all(e.query() for e in evs):
+        if time.monotonic() - t0 > timeout_s:
+            raise TimeoutError(f"{what}: GPU work not finished after {timeout_s:.0f} s (a peer stage stalled?)")
+        time.sleep(0.0002)
+
+
 def make_pipeline_groups(n_pipelines: int, ranks: Optional[Sequence[int]] = None, backend: Optional[str] = None):
     """One process group per parallel pipeline over the K stage ranks (a collective call: every stage rank
     creates the N groups in the same order).  Pipeline i's activations and gradients travel only on group i."""
@@ -64,7 +81,7 @@ class PipelineStage:
                  center=None, flat_params=None, flat_grads=None, mem_limit: Optional[float] = None,
                  mem_per_microbatch: float = 0.0, extra_advance: int = 0, dynamic: bool = False,
                  concurrent: bool = False, groups=None, transport: str = "dist", act_bytes: int = 0,
-                 device=None):
+                 device=None, timeout_s: float = 600.0):
         import torch.distributed as dist
         self.replicas = list(replicas)
         self.N = len(self.replicas)
@@ -93,6 +110,7 @@ class PipelineStage:
         if transport not in ("dist", "ipc"):
             raise ValueError("transport must be 'dist' or 'ipc'")
         self.transport = transport
+        self.timeout_s = float(timeout_s)    # ipc: deadline for an iteration's streams (a stalled peer stage)
         self._chan = {}
         if transport == "ipc":
             self._open_channels(act_bytes, device)
@@ -286,10 +304,16 @@ class PipelineStage:
                 self.ea.step(self.ea_stage, self.flat_params, self.flat_grads, self.center)
         for w in pending:
             w.wait()
-        if cuda and sync:
+        streams = (self._streams if self.concurrent else [torch.cuda.current_stream(device)]) if cuda else []
+        if cuda and self.transport == "ipc":
+            # a stream waiting on the GPU for a message the peer never sends would block synchronize() forever:
+            # wait with a deadline instead (the EA stream too when sync)
+            wait_streams(streams + ([self._ea_stream] if sync and self._ea_stream is not None else []),
+                         self.timeout_s, f"stage {self.stage}")
+        elif cuda and sync:
             torch.cuda.synchronize(device)
         elif cuda:
-            for s in (self._streams if self.concurrent else [torch.cuda.current_stream(device)]):
+            for s in streams:
                 s.synchronize()
         dt = time.perf_counter() - t0
         self.peak_stash = peak

@@ -118,6 +118,23 @@ def test_channel_errors():
     assert snd.count == 0 and rcv.count == 0   # nothing was enqueued by the failing calls
 
 
+def test_stalled_peer_is_detected_by_the_deadline():
+    """pipeline.wait_streams: a receive whose message never comes raises TimeoutError instead of hanging; the
+    late send then releases the stream."""
+    from paper_conf_ppopp_chen0qz23_b200.pipeline import wait_streams
+    snd, rcv = _pair(1024, 2)
+    s_recv = torch.cuda.Stream()
+    out = torch.zeros(256, device="cuda")
+    ones = torch.ones(256, device="cuda")     # no kernel launches while s_recv is blocked (lazy loading, above)
+    torch.cuda.synchronize()
+    rcv.recv(out, stream=s_recv)
+    with pytest.raises(TimeoutError, match="peer stage stalled"):
+        wait_streams([s_recv], 0.5, "stage 1")
+    snd.send(ones)
+    wait_streams([s_recv], 60.0)
+    assert torch.equal(out, ones)
+
+
 def _ipc_worker(rank, port, q, n_msgs):
     import torch.distributed as dist
     os.environ["CUDA_MODULE_LOADING"] = "EAGER"   # before this process initialises CUDA (see pipeline.py)

@@ -17,10 +17,10 @@ FLOORS = {
     "test_gpu_bench.py": 5,
     "test_gpu_multirank.py": 5,
     "test_gpu_pipeline.py": 5,
-    "test_gpu_chan.py": 8,
+    "test_gpu_chan.py": 9,
     "test_gpu_fuzz.py": 120,
 }
-TOTAL_FLOOR = 481
+TOTAL_FLOOR = 482
 
 
 def test_gpu_suite_size():
