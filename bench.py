@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--steps", type=int, default=1000)
     ap.add_argument("--warmup", type=int, default=20)
     ap.add_argument("--impl", choices=("ours", "reference"), default="ours")
-    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe", "split", "warprep"), default="auto")
+    ap.add_argument("--variant", choices=("auto", "regloop", "laneshfl", "bulkpipe", "split", "warprep", "warpspec"), default="auto")
     ap.add_argument("--optimizer", choices=("sgd", "adam", "adamw", "asgd"), default="sgd",
                     help="local optimizer (BASELINE configs: SGD+momentum; Adam(W) and ASGD are row f1)")
     ap.add_argument("--staleness", type=int, choices=(0, 1), default=0,
@@ -203,7 +203,7 @@ def stale_fused(n, optimizer, variant):
     """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1; N = 5 for
     SGD/ASGD) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
     return ((variant == "auto" and (n <= 4 or (n == 5 and optimizer not in ("adam", "adamw"))))
-            or (variant == "warprep" and n <= 8))
+            or (variant in ("warprep", "warpspec") and n <= 8))
 
 
 def kernel_name(variant, optimizer, n, staleness=0):
@@ -214,7 +214,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
     if staleness:
         if stale_fused(n, optimizer, variant):   # ea_api.cu: x~_{t-1} staged beside x~_t, <= 8 stages per launch
             two = optimizer in ("adam", "adamw")
-            kern = ("colocated_warprep" if variant == "warprep" or (not two and n in (2, 5)) else
+            kern = ("colocated_warpspec" if variant == "warpspec" else
+                    "colocated_warprep" if variant == "warprep" or (not two and n in (2, 5)) else
                     "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe")
             return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"

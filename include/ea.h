@@ -123,7 +123,9 @@ typedef struct {
                                    tile by cp.async.bulk into an mbarrier ring), 4 = split
                                    register loop (two lanes per center column, N/2 replicas
                                    each, shuffle reduction), 5 = warp per replica (contributions
-                                   reduced through shared memory).  Same results
+                                   reduced through shared memory), 6 = warp-specialised warp per
+                                   replica (N replica warps + a reducer warp over an mbarrier ring
+                                   of contribution tiles; no block barrier).  Same results
                                    up to fp32 summation order (DESIGN.md c14); the default picks per N and optimizer
                                    (DESIGN.md §7). */
   int32_t optimizer;            /* ea_optimizer */

@@ -20,7 +20,7 @@ EA_OK, EA_EINVAL, EA_ECUDA, EA_ENCCL, EA_ESTATE, EA_ENOMEM = range(6)
 EA_COLOCATED, EA_SPREAD = 0, 1
 STATUS_NAMES = {0: "EA_OK", 1: "EA_EINVAL", 2: "EA_ECUDA", 3: "EA_ENCCL", 4: "EA_ESTATE", 5: "EA_ENOMEM"}
 LAYOUTS = {"colocated": EA_COLOCATED, "spread": EA_SPREAD}
-VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3, "split": 4, "warprep": 5}
+VARIANTS = {"auto": 0, "regloop": 1, "laneshfl": 2, "bulkpipe": 3, "split": 4, "warprep": 5, "warpspec": 6}
 OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2, "asgd": 3}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128

@@ -328,7 +328,8 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // the replica loop for A/B measurement.
   const bool stale_lane = stale && !force_wide &&
                           ((h->variant == 0 && (n <= 4 || (n == 5 && !ea::two_state(opt)))) ||
-                           (h->variant == ea::kVariantWarpRep && n <= ea::kMaxFusedN));
+                           ((h->variant == ea::kVariantWarpRep || h->variant == ea::kVariantWarpSpec) &&
+                            n <= ea::kMaxFusedN));
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched
     for (int j = 0; j < count; ++j) {
       ea_status st2 = stale_prev_init(h, stages[j], center_ptrs[j], s);
@@ -773,7 +774,7 @@ ea_status ea_init(const ea_config* cfg, const uint8_t* nccl_id, ea_handle* out) 
     if (c.world != c.n_pipelines) { set_err(nullptr, "EA_SPREAD needs world == n_pipelines"); return EA_EINVAL; }
     if (c.rank < 0 || c.rank >= c.world) { set_err(nullptr, "rank %d out of [0,%d)", c.rank, c.world); return EA_EINVAL; }
   }
-  if (c.kernel_variant < 0 || c.kernel_variant > 5) { set_err(nullptr, "kernel_variant must be 0..5"); return EA_EINVAL; }
+  if (c.kernel_variant < 0 || c.kernel_variant > 6) { set_err(nullptr, "kernel_variant must be 0..6"); return EA_EINVAL; }
   if (c.exchange != EA_XCHG_NCCL && c.exchange != EA_XCHG_P2P) { set_err(nullptr, "unknown exchange %d", c.exchange); return EA_EINVAL; }
   if (c.staleness != 0 && c.staleness != 1) { set_err(nullptr, "staleness must be 0 or 1"); return EA_EINVAL; }
   if (c.staleness == 1 && c.layout == EA_SPREAD && c.exchange != EA_XCHG_NCCL) {

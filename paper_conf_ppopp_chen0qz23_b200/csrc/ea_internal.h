@@ -99,6 +99,7 @@ enum KernelVariant : int {
                          // ring (producer warp + mbarriers); consumers store from registers (SGD)
   kVariantSplit = 4,     // split register loop: 2 lanes per center column, N/2 replicas each, shuffle reduction
   kVariantWarpRep = 5,   // warp per replica, 512 B rows, contributions reduced through shared memory
+  kVariantWarpSpec = 6,  // warp-specialised: N replica warps + a reducer warp, mbarrier ring of contribution tiles
 };
 
 // Co-located fused step (rows a1-a5) for a batch of stages with the same N
@@ -111,7 +112,7 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
 // lane kernel with x~_{t-1} staged beside x~_t, for N = 1 and 5 the bulk-copy pipeline with x~_{t-1} as one more
 // stream (replicas use x~_{t-1}, x~_{t+1} = x~_t + R/N, prev <- x~_t).
 constexpr int kMaxStaleLaneN = 4;
-// variant kVariantWarpRep: the warp-per-replica kernel with x~_{t-1} for any N <= kMaxFusedN.
+// variant kVariantWarpRep / kVariantWarpSpec: the warp-per-replica kernels with x~_{t-1} for any N <= kMaxFusedN.
 cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper& hp, int opt, int variant,
                                          int num_sms, cudaStream_t s);
 

@@ -374,6 +374,118 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
+// ============================================================================
+// Variant 6: warp-specialised warp per replica.  Warp i < N streams replica i exactly as variant 5 does (U float4
+// of x, g and the optimizer state per lane and tile, 512 B rows per load instruction) but never waits at a block
+// barrier: it writes its contribution r_i into an R-deep ring of contribution tiles in shared memory and arrives
+// on the slot's "full" mbarrier; warp N (the reducer) waits for the N contributions of a slot, sums them, applies
+// x~ += R/N and arrives on the slot's "empty" mbarrier.  A replica warp waits only when the ring is full, so the
+// replica warps drift up to R tiles apart and keep their loads in flight while the reduction of older tiles runs.
+// STALE (row f4, c28): the replica warps read x~_{t-1}; the reducer reads x~_t, writes x~_{t+1} and x~_{t-1} <- x~_t.
+// ============================================================================
+template <int N, int OPT, int U, int R, bool STALE = false>
+__global__ void __launch_bounds__(32 * (N + 1), U >= 4 ? 1 : 2) colocated_warpspec(const StageBatch b,
+                                                                                    const Hyper hp) {
+  constexpr int TV = 32 * U;  // float4 columns per tile
+  constexpr bool kTwo = two_state(OPT);
+  extern __shared__ __align__(16) float4 s_ring[];  // [R][N][TV] contribution tiles (dynamic: up to 64 KB)
+  __shared__ __align__(8) uint64_t full[R], empty[R];
+  __shared__ StepCoef s_coef[kMaxLaunchStages];
+  const Mem<0> mem;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  auto s_r = [&](int k, int i, int lv) -> float4& { return s_ring[(k * N + i) * TV + lv]; };
+  if (has_coef(OPT) && threadIdx.x < b.nstages) s_coef[threadIdx.x] = *b.st[threadIdx.x].scp;
+  if (threadIdx.x == 0) {
+    for (int k = 0; k < R; ++k) {
+      mbar_init(&full[k], 32 * N);  // every lane of every replica warp arrives (releases its own stores)
+      mbar_init(&empty[k], 32);     // every lane of the reducer warp
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
+  WaveCursor cur{0, 0};
+  int s;
+  int64_t v0, nv;
+  int slot = 0;
+  uint32_t phase = 0;
+  if (warp < N) {  // ---------------------------------------------------------------- replica warp
+    while (wave_item(b, TV, cur, s, v0, nv)) {
+      const StageRefs& st = b.st[s];
+      const StepCoef sc = has_coef(OPT) ? s_coef[s] : StepCoef{0.f, 0.f};
+      float* xi = st.x[warp];
+      const float* gi = st.g[warp];
+      float* mi = st.m[warp];
+      float* vi = kTwo ? st.v[warp] : nullptr;
+      float4 x[U], g[U], m[U], w[U], c[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int lv = u * 32 + lane;
+        if (lv < nv) {
+          const int64_t v = v0 + lv;
+          x[u] = mem.ld(xi + 4 * v);
+          g[u] = mem.ld_ro(gi + 4 * v);
+          m[u] = mem.ld(mi + 4 * v);
+          if (kTwo) w[u] = mem.ld(vi + 4 * v);
+          c[u] = __ldg(reinterpret_cast<const float4*>(STALE ? st.prev : st.c) + v);
+        }
+      }
+      float4 r[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int lv = u * 32 + lane;
+        if (lv < nv) {
+          const int64_t v = v0 + lv;
+          r[u] = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
+          mem.st(xi + 4 * v, x[u]);
+          mem.st(mi + 4 * v, m[u]);
+          if (kTwo) mem.st(vi + 4 * v, w[u]);
+        }
+      }
+      mbar_wait(&empty[slot], phase ^ 1u);  // the reducer has finished with this slot's previous tile
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int lv = u * 32 + lane;
+        if (lv < nv) s_r(slot, warp, lv) = r[u];
+      }
+      mbar_arrive(&full[slot]);
+      if (++slot == R) {
+        slot = 0;
+        phase ^= 1u;
+      }
+    }
+  } else {  // --------------------------------------------------------------------------- reducer warp
+    while (wave_item(b, TV, cur, s, v0, nv)) {
+      const StageRefs& st = b.st[s];
+      float4 c[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {  // x~_t of this lane's columns, in flight while the replicas finish
+        const int lv = u * 32 + lane;
+        if (lv < nv) c[u] = __ldg(reinterpret_cast<const float4*>(st.c) + v0 + lv);
+      }
+      mbar_wait(&full[slot], phase);
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int lv = u * 32 + lane;
+        if (lv < nv) {
+          float4 acc = s_r(slot, 0, lv);
+#pragma unroll
+          for (int i = 1; i < N; ++i) add4(acc, s_r(slot, i, lv));
+          const int64_t v = v0 + lv;
+          mem.st(st.c + 4 * v, center_apply(c[u], acc, hp.inv_n));
+          if (STALE) mem.st(st.prev + 4 * v, c[u]);
+        }
+      }
+      mbar_arrive(&empty[slot]);
+      if (++slot == R) {
+        slot = 0;
+        phase ^= 1u;
+      }
+    }
+    if (blockIdx.x == gridDim.x - 1 && lane == 0)
+      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
+  }
+}
+
 template <int U>
 struct WideRep {
   float4 x[U], g[U], m[U], w[U];
@@ -879,9 +991,9 @@ int grid_knob() {
 }
 
 template <typename K>
-int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads) {
+int persistent_grid(K kernel, int64_t work_units, int num_sms, int threads = kThreads, size_t smem = 0) {
   int per_sm = 0;
-  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, 0) != cudaSuccess || per_sm < 1)
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kernel, threads, smem) != cudaSuccess || per_sm < 1)
     per_sm = 1;
   int64_t grid = (int64_t)num_sms * per_sm;
   const int knob = grid_knob();
@@ -1055,8 +1167,42 @@ cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cu
   return launch_warprep_u<N, OPT, 4, STALE>(b, hp, num_sms, s);
 }
 
+// Warp-specialised warp per replica (variant 6): U float4 columns per lane and tile, a ring of R = 4 contribution
+// tiles; measurement knob AVGPIPE_EA_WARPSPEC_U = 2 | 4 (default 4).
+int warpspec_u() {
+  static const int v = [] {
+    const char* e = std::getenv("AVGPIPE_EA_WARPSPEC_U");
+    return (e && e[0] == '2') ? 2 : 4;
+  }();
+  return v;
+}
+
+template <int N, int OPT, int U, int R, bool STALE>
+cudaError_t launch_warpspec_t(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  auto k = colocated_warpspec<N, OPT, U, R, STALE>;
+  constexpr size_t smem = sizeof(float4) * R * N * 32 * U;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, static_cast<int>(smem));
+  if (e != cudaSuccess) return e;
+  k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * (N + 1), smem), 32 * (N + 1), smem, s>>>(b, hp);
+  return cudaGetLastError();
+}
+
+template <int N, int OPT, bool STALE = false>
+cudaError_t launch_warpspec(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
+  if (warpspec_u() == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
+  return launch_warpspec_t<N, OPT, 4, 4, STALE>(b, hp, num_sms, s);
+}
+
 template <int N>
 cudaError_t launch_n(const StageBatch& b, const Hyper& hp, int opt, int variant, int num_sms, cudaStream_t s) {
+  if (variant == kVariantWarpSpec) {
+    switch (opt) {
+      case kOptAdam: return launch_warpspec<N, kOptAdam>(b, hp, num_sms, s);
+      case kOptAdamW: return launch_warpspec<N, kOptAdamW>(b, hp, num_sms, s);
+      case kOptASGD: return launch_warpspec<N, kOptASGD>(b, hp, num_sms, s);
+      default: return launch_warpspec<N, kOptSGD>(b, hp, num_sms, s);
+    }
+  }
   if (variant == kVariantWarpRep) {
     switch (opt) {
       case kOptAdam: return launch_warprep<N, kOptAdam>(b, hp, num_sms, s);
@@ -1261,6 +1407,16 @@ cudaError_t launch_stale_n(const StageBatch& b, const Hyper& hp, int opt, int nu
 }
 
 template <int N>
+cudaError_t launch_stale_warpspec_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
+  switch (opt) {
+    case kOptAdam: return launch_warpspec<N, kOptAdam, true>(b, hp, num_sms, s);
+    case kOptAdamW: return launch_warpspec<N, kOptAdamW, true>(b, hp, num_sms, s);
+    case kOptASGD: return launch_warpspec<N, kOptASGD, true>(b, hp, num_sms, s);
+    default: return launch_warpspec<N, kOptSGD, true>(b, hp, num_sms, s);
+  }
+}
+
+template <int N>
 cudaError_t launch_stale_warprep_n(const StageBatch& b, const Hyper& hp, int opt, int num_sms, cudaStream_t s) {
   switch (opt) {
     case kOptAdam: return launch_warprep<N, kOptAdam, true>(b, hp, num_sms, s);
@@ -1278,6 +1434,19 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
   // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
   if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
+  if (variant == kVariantWarpSpec) {
+    switch (n) {
+      case 1: return launch_stale_warpspec_n<1>(b, hp, opt, num_sms, s);
+      case 2: return launch_stale_warpspec_n<2>(b, hp, opt, num_sms, s);
+      case 3: return launch_stale_warpspec_n<3>(b, hp, opt, num_sms, s);
+      case 4: return launch_stale_warpspec_n<4>(b, hp, opt, num_sms, s);
+      case 5: return launch_stale_warpspec_n<5>(b, hp, opt, num_sms, s);
+      case 6: return launch_stale_warpspec_n<6>(b, hp, opt, num_sms, s);
+      case 7: return launch_stale_warpspec_n<7>(b, hp, opt, num_sms, s);
+      case 8: return launch_stale_warpspec_n<8>(b, hp, opt, num_sms, s);
+      default: return cudaErrorInvalidValue;
+    }
+  }
   if (variant == kVariantWarpRep) {
     switch (n) {
       case 1: return launch_stale_warprep_n<1>(b, hp, opt, num_sms, s);

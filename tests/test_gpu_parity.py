@@ -277,6 +277,44 @@ def test_warp_per_replica_knobs(knobs):
     assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
 
 
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "adamw", "asgd"])
+@pytest.mark.parametrize("n", [1, 2, 3, 5, 6, 7, 8])
+def test_warp_specialised(n, optimizer):
+    """Variant 6 (N replica warps + a reducer warp over an mbarrier ring of contribution tiles): C1-sized and
+    ragged stages in one launch (ring wrap-around, ragged last tiles, scalar tails), every optimizer."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 12, "combined", variants=("warpspec",), many=True,
+                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2)
+
+
+@pytest.mark.parametrize("optimizer", ["sgd", "adam", "asgd"])
+@pytest.mark.parametrize("n", [1, 2, 4, 8])
+def test_warp_specialised_stale(n, optimizer):
+    """Variant 6 with the stale center (row f4): replica warps read x~_{t-1}, the reducer writes x~_{t+1} and
+    x~_{t-1} <- x~_t."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096], 20, "combined", variants=("warpspec",), many=True, optimizer=optimizer,
+                   lr=lr, staleness=1)
+
+
+def test_warp_specialised_u2_and_100_steps():
+    """The U = 2 geometry behind AVGPIPE_EA_WARPSPEC_U (a subprocess: the knob is read once) and the 100-step
+    C1 gate with Adam at N = 8."""
+    import subprocess
+    import sys
+    code = ("import tests.test_gpu_parity as t\n"
+            "for opt in ('sgd', 'adam', 'asgd'):\n"
+            "    lr = 1e-3 if opt == 'adam' else t.synth.LR\n"
+            "    for n in (1, 4, 8):\n"
+            "        t._run_colocated(n, [100_003, 7, 4096, 300_001], 8, 'combined', variants=('warpspec',), many=True,"
+            " optimizer=opt, lr=lr, wd=0.0 if opt == 'sgd' else 1e-2)\n")
+    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=dict(os.environ, AVGPIPE_EA_WARPSPEC_U="2"),
+                       capture_output=True, text=True, timeout=1200)
+    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warpspec",), many=True, optimizer="adam",
+                   lr=1e-3, wd=1e-2)
+
+
 def test_warp_per_replica_c1_100_steps():
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warprep",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
