@@ -1168,13 +1168,15 @@ cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cu
 }
 
 // Warp-specialised warp per replica (variant 6): U float4 columns per lane and tile, a ring of R = 4 contribution
-// tiles; measurement knob AVGPIPE_EA_WARPSPEC_U = 2 | 4 (default 4).
-int warpspec_u() {
+// tiles.  U = 2 for Adam(W) with the synchronous center (N = 8: 0.949 vs 0.845 with U = 4), else U = 4
+// (profiles/r02_s3_sweep_warpspec.jsonl); measurement knob AVGPIPE_EA_WARPSPEC_U = 2 | 4 overrides.
+int warpspec_u(int opt, bool stale) {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_WARPSPEC_U");
-    return (e && e[0] == '2') ? 2 : 4;
+    return e ? std::atoi(e) : 0;
   }();
-  return v;
+  if (v == 2 || v == 4) return v;
+  return (two_state(opt) && !stale) ? 2 : 4;
 }
 
 template <int N, int OPT, int U, int R, bool STALE>
@@ -1189,7 +1191,7 @@ cudaError_t launch_warpspec_t(const StageBatch& b, const Hyper& hp, int num_sms,
 
 template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warpspec(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  if (warpspec_u() == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
+  if (warpspec_u(OPT, STALE) == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
   return launch_warpspec_t<N, OPT, 4, 4, STALE>(b, hp, num_sms, s);
 }
 
@@ -1360,15 +1362,19 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // 0.941 vs 0.920 / 0.937; profiles/r02_sweep_split.jsonl -- with SGD it measured below the bulk pipeline).
   // Round 2 session h (same box, C2 sizes): Adam N = 5 on the warp-per-replica kernel with U = 4, 0.974 (session
   // g) / split 0.944-0.950; N = 2, 3 within 1% of the register loop (0.960 / 0.941 vs 0.948 / 0.940), kept.
+  // Session o: Adam N = 8 on the warp-specialised kernel (U = 2) 0.949 vs 0.924 for the replica loop (N = 7 stays
+  // on the replica loop, ea_api.cu: 0.917 vs 0.901).
   if (variant == kVariantAuto && two_state(opt))
     variant = n == 1 ? kVariantLaneShfl
                      : (n <= 3 ? kVariantRegLoop
-                               : (n == 4 ? kVariantBulkPipe : (n == 5 ? kVariantWarpRep : kVariantSplit)));
+                               : (n == 4 ? kVariantBulkPipe
+                                         : (n == 5 ? kVariantWarpRep : (n == 8 ? kVariantWarpSpec : kVariantSplit))));
   // SGD-momentum and ASGD (one state vector), round 2: the warp-per-replica kernel for N = 1 and 3..8 (same box,
   // C2 sizes: N = 1 0.937 vs 0.872 bulk pipeline, N = 3 0.986 vs 0.932 lane, N = 4 0.996-0.998 vs 0.983 lane,
   // N = 5..8 0.979-1.0 vs 0.93-0.976; ASGD alike), the lane kernel for N = 2 (0.963 vs 0.952);
   // profiles/r02_sweep_warprep*.jsonl.  (Its Adam instances run out of registers: 0.69-0.87.)
-  if (variant == kVariantAuto) variant = n == 2 ? kVariantLaneShfl : kVariantWarpRep;
+  // Session o: N = 5 on the warp-specialised kernel (SGD 1.001 / ASGD 0.995 vs 0.987 / 0.984 warp per replica).
+  if (variant == kVariantAuto) variant = n == 2 ? kVariantLaneShfl : (n == 5 ? kVariantWarpSpec : kVariantWarpRep);
   switch (n) {
     case 1: return launch_n<1>(b, hp, opt, variant, num_sms, s);
     case 2: return launch_n<2>(b, hp, opt, variant, num_sms, s);
@@ -1434,6 +1440,8 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
   // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
   if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
+  // session o: Adam(W) N = 3 on the warp-specialised kernel (0.933 vs 0.865 lane kernel)
+  if (variant == kVariantAuto && two_state(opt) && n == 3) variant = kVariantWarpSpec;
   if (variant == kVariantWarpSpec) {
     switch (n) {
       case 1: return launch_stale_warpspec_n<1>(b, hp, opt, num_sms, s);

@@ -297,6 +297,17 @@ def test_warp_specialised_stale(n, optimizer):
                    lr=lr, staleness=1)
 
 
+@pytest.mark.parametrize("n,optimizer,staleness", [(8, "adam", 0), (8, "adamw", 0), (5, "sgd", 0), (5, "asgd", 0),
+                                                   (3, "adam", 1), (3, "adamw", 1), (7, "adam", 0)])
+def test_library_default_kernel(n, optimizer, staleness):
+    """The library's own per-N choice (kernel_variant "auto") where session o moved it: Adam(W) N = 8 and
+    SGD/ASGD N = 5 to the warp-specialised kernel, the stale Adam(W) N = 3 likewise, Adam N = 7 on the replica
+    loop; 30 steps, several stages per call."""
+    lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
+    _run_colocated(n, [100_003, 7, 4096, 1_000_001], 30, "combined", variants=("auto",), many=True,
+                   optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2, staleness=staleness)
+
+
 def test_warp_specialised_u2_and_100_steps():
     """The U = 2 geometry behind AVGPIPE_EA_WARPSPEC_U (a subprocess: the knob is read once) and the 100-step
     C1 gate with Adam at N = 8."""
