@@ -73,6 +73,7 @@ extern "C" {
 #define EA_MAX_REPLICAS 64     /* co-located N limit (kernel parameter table) */
 #define EA_UNIQUE_ID_BYTES 128 /* == sizeof(ncclUniqueId) */
 #define EA_IPC_HANDLE_BYTES 64 /* == sizeof(cudaIpcMemHandle_t) */
+#define EA_CHAN_HANDLE_BYTES 80 /* ea_chan_export: the IPC handle + the end's slot_bytes, slots and role */
 #define EA_SLOT_CENTER_PREV 2  /* ea_get_state / ea_set_state slot of the stale center x~_{t-1} (staleness 1) */
 
 typedef enum {
@@ -333,8 +334,9 @@ EA_API int32_t ea_schedule(int32_t K, int32_t M, int32_t stage, int32_t advance,
  * P:140-162).  A channel is ONE direction between two processes (NVLink peers, or two processes sharing a GPU).
  * The receiving end owns a ring of `slots` message slots of `slot_bytes` and one ready word per slot, the
  * sending end one acknowledgement word per slot, all in device memory on `device`.  Each end exports its buffer
- * (ea_chan_export, EA_IPC_HANDLE_BYTES, cudaIpcMemHandle_t) and opens the other's (ea_chan_connect); two ends
- * in ONE process are wired with ea_chan_pair instead (CUDA IPC cannot open a handle of its own process).
+ * (ea_chan_export: EA_CHAN_HANDLE_BYTES = the cudaIpcMemHandle_t plus the end's geometry and role) and opens the
+ * other's (ea_chan_connect: EA_EINVAL unless the peer has the opposite role and the same slot_bytes and slots);
+ * two ends in ONE process are wired with ea_chan_pair instead (CUDA IPC cannot open a handle of its own process).
  *
  * ea_chan_send / ea_chan_recv enqueue on `stream` (cudaStream_t; NULL = legacy default stream) and never block
  * the host: send = wait until the slot is free (stream wait on the local ack word) -> copy-engine copy of

@@ -25,6 +25,7 @@ OPTIMIZERS = {"sgd": 0, "adam": 1, "adamw": 2, "asgd": 3}
 EXCHANGES = {"nccl": 0, "p2p": 1}
 UNIQUE_ID_BYTES = 128
 IPC_HANDLE_BYTES = 64   # == EA_IPC_HANDLE_BYTES (cudaIpcMemHandle_t)
+CHAN_HANDLE_BYTES = 80  # == EA_CHAN_HANDLE_BYTES (IPC handle + slot_bytes, slots, role)
 ABI_VERSION = 6
 SLOT_CENTER_PREV = 2   # EA_SLOT_CENTER_PREV: the stale center x~_{t-1} (staleness 1)
 
@@ -312,14 +313,15 @@ class Channel:
             raise EAError(st, (self._lib.ea_chan_last_error(self._h) or b"").decode())
 
     def export(self) -> bytes:
-        buf = (ctypes.c_uint8 * IPC_HANDLE_BYTES)()
+        buf = (ctypes.c_uint8 * CHAN_HANDLE_BYTES)()
         self._check(self._lib.ea_chan_export(self._h, buf))
         return bytes(buf)
 
     def connect(self, peer_handle: bytes):
-        if len(peer_handle) != IPC_HANDLE_BYTES:
-            raise ValueError(f"peer handle must be {IPC_HANDLE_BYTES} bytes")
-        self._check(self._lib.ea_chan_connect(self._h, (ctypes.c_uint8 * IPC_HANDLE_BYTES).from_buffer_copy(peer_handle)))
+        if len(peer_handle) != CHAN_HANDLE_BYTES:
+            raise ValueError(f"peer handle must be {CHAN_HANDLE_BYTES} bytes")
+        self._check(self._lib.ea_chan_connect(self._h,
+                                              (ctypes.c_uint8 * CHAN_HANDLE_BYTES).from_buffer_copy(peer_handle)))
 
     @staticmethod
     def pair(send_end: "Channel", recv_end: "Channel"):

@@ -157,20 +157,42 @@ EA_API ea_status ea_chan_create(int32_t device, int32_t role, int64_t slot_bytes
   return EA_OK;
 }
 
+// Exported handle: the CUDA IPC handle of this end's buffer, then the end's geometry and role, so that
+// ea_chan_connect can refuse a peer whose slots differ (its copies would overrun this end's ring).
+struct ChanHandle {
+  cudaIpcMemHandle_t ipc;
+  int64_t slot_bytes;
+  int32_t slots;
+  int32_t role;
+};
+static_assert(sizeof(ChanHandle) == EA_CHAN_HANDLE_BYTES, "EA_CHAN_HANDLE_BYTES");
+
 EA_API ea_status ea_chan_export(ea_chan c, uint8_t* handle) {
   if (!c || !handle) { set_err(c, "NULL channel or output"); return EA_EINVAL; }
-  static_assert(sizeof(cudaIpcMemHandle_t) == EA_IPC_HANDLE_BYTES, "IPC handle size");
+  ChanHandle h;
+  memset(&h, 0, sizeof(h));
   cudaError_t e = cudaSetDevice(c->device);
-  if (e == cudaSuccess) e = cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(handle), c->local);
+  if (e == cudaSuccess) e = cudaIpcGetMemHandle(&h.ipc, c->local);
   if (e != cudaSuccess) return cfail(c, e, "cudaIpcGetMemHandle");
+  h.slot_bytes = c->slot_bytes;
+  h.slots = c->slots;
+  h.role = c->role;
+  memcpy(handle, &h, sizeof(h));
   return EA_OK;
 }
 
 EA_API ea_status ea_chan_connect(ea_chan c, const uint8_t* peer_handle) {
   if (!c || !peer_handle) { set_err(c, "NULL channel or handle"); return EA_EINVAL; }
   if (c->peer) { set_err(c, "channel already connected"); return EA_ESTATE; }
-  cudaIpcMemHandle_t h;
-  memcpy(&h, peer_handle, sizeof(h));
+  ChanHandle ph;
+  memcpy(&ph, peer_handle, sizeof(ph));
+  if (ph.role != 1 - c->role) { set_err(c, "the peer end must have the opposite role"); return EA_EINVAL; }
+  if (ph.slot_bytes != c->slot_bytes || ph.slots != c->slots) {
+    set_err(c, "peer geometry (%lld bytes x %d slots) differs from this end's (%lld x %d)", (long long)ph.slot_bytes,
+            ph.slots, (long long)c->slot_bytes, c->slots);
+    return EA_EINVAL;
+  }
+  const cudaIpcMemHandle_t h = ph.ipc;
   void* p = nullptr;
   cudaError_t e = cudaSetDevice(c->device);
   if (e == cudaSuccess) e = cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess);

@@ -115,6 +115,14 @@ def test_channel_errors():
             snd.send(x)
     with pytest.raises(EAError):
         Channel("send", 0, 2)
+    # connect checks the exported geometry and role before mapping anything
+    other_send, other_recv3 = Channel("send", 256, 2), Channel("recv", 256, 3)
+    with pytest.raises(EAError, match="opposite role"):
+        Channel("send", 256, 2).connect(other_send.export())
+    with pytest.raises(EAError, match="differs"):
+        Channel("send", 256, 2).connect(other_recv3.export())
+    with pytest.raises(ValueError):
+        lone.connect(b"\0" * 64)
     assert snd.count == 0 and rcv.count == 0   # nothing was enqueued by the failing calls
 
 
