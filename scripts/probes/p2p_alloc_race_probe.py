@@ -5,12 +5,12 @@ without record_stream, so the caching allocator could give a gradient's block to
 the (slow) push kernel still read it.  Here the library's stream is slowed by a sleep kernel instead of the
 sanitizer: without record_stream the result differs from the oracle, with it the result matches.
 
-    python scripts/p2p_alloc_race_probe.py
+    python scripts/probes/p2p_alloc_race_probe.py
 """
 import os
 import sys
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 
 
 def run(record):

@@ -5,7 +5,7 @@ import sys
 os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")   # 2N streams of N virtual ranks (ea.h)
 import time
 
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 os.environ.setdefault("AVGPIPE_EA_P2P_TIMEOUT_MS", "5000")
 from tests.test_gpu_p2p import _run  # noqa: E402
 

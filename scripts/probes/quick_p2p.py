@@ -1,7 +1,7 @@
 """Fast sanity check of the fused peer-memory exchange with virtual ranks (run under `timeout`)."""
 import os
 import sys
-sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__)))))
 os.environ.setdefault("AVGPIPE_EA_P2P_TIMEOUT_MS", "5000")
 from tests.test_gpu_p2p import _run  # noqa: E402
 

@@ -3,7 +3,7 @@
 # hyper-parameters in the oracle, the push kernel's chunk size, the split kernel's grid.
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
 mkdir -p gpurun_out
-bash scripts/gpu_sanitize.sh
+bash scripts/sessions/gpu_sanitize.sh
 AVGPIPE_PARITY_F64_HYPER=1 AVGPIPE_PARITY_LOG=gpurun_out/parity_margins_f64hyper.jsonl timeout 1800 \
   python -m pytest tests/test_gpu_parity.py tests/test_gpu_fullsize.py -q -m gpu -k "adam or c1_100 or accumulated" > gpurun_out/pytest_f64hyper.log 2>&1
 tail -3 gpurun_out/pytest_f64hyper.log

@@ -14,7 +14,7 @@ done
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:p2p_push -s 8 -c 1 -o gpurun_out/prof_p2p_push -f \
     python bench.py --layout spread --config C4 --exchange p2p --steps 2 --warmup 1 --no-e2e --no-cpu-baseline > gpurun_out/ncu_full_p2p.log 2>&1
 for push in bulk plain; do
-  AVGPIPE_EA_P2P_PUSH=$push AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/p2p_sanitize.py > gpurun_out/san_racecheck_p2p_$push.log 2>&1
+  AVGPIPE_EA_P2P_PUSH=$push AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/probes/p2p_sanitize.py > gpurun_out/san_racecheck_p2p_$push.log 2>&1
   tail -3 gpurun_out/san_racecheck_p2p_$push.log
 done
 echo session done

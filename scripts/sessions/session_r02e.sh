@@ -28,9 +28,9 @@ for t in 256 512; do
 done
 echo session done
 for push in bulk plain; do
-  AVGPIPE_EA_P2P_PUSH=$push AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/p2p_sanitize.py > gpurun_out/san_racecheck_p2p_$push.log 2>&1
+  AVGPIPE_EA_P2P_PUSH=$push AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/probes/p2p_sanitize.py > gpurun_out/san_racecheck_p2p_$push.log 2>&1
   grep -v "^=====" gpurun_out/san_racecheck_p2p_$push.log | tail -12
 done
-AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool memcheck python scripts/p2p_sanitize.py > gpurun_out/san_memcheck_p2p.log 2>&1
+AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool memcheck python scripts/probes/p2p_sanitize.py > gpurun_out/san_memcheck_p2p.log 2>&1
 grep -v "^=====" gpurun_out/san_memcheck_p2p.log | tail -6
 echo racecheck probe done

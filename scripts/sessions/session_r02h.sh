@@ -46,7 +46,7 @@ for l in open('gpurun_out/sweep_ring.jsonl'):
     d = json.loads(l); r = d['roofline']
     print(f"{d['args']:50s} {d['knob']:18s} {r['kernel']:30s} frac {r['frac']:.3f} ms {d['ms_per_step']:.4f} {d['clocks']['reasons']}")
 PY
-AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/p2p_sanitize.py \
+AVGPIPE_EA_P2P_TIMEOUT_MS=120000 timeout 900 compute-sanitizer --tool racecheck --print-limit 20 python scripts/probes/p2p_sanitize.py \
   > gpurun_out/san_racecheck_p2p.log 2>&1; echo "rc=$?" >> gpurun_out/san_racecheck_p2p.log
 grep -E "ok|FAIL|hazard|ERROR SUMMARY|rc=" gpurun_out/san_racecheck_p2p.log | tail -12
 echo session done
