@@ -407,8 +407,9 @@ def run_ours(args, rank, world, local):
         pct = {f"p{k}": q[min(len(q) - 1, len(q) * k // 100)] for k in (10, 50, 90)}
         out["roofline"] = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                            "frac": achieved / peak,
-                           "traffic": traffic_from_profiles(cfg.name, kernel_name(args.variant, args.optimizer, n,
-                                                                                  args.staleness)),
+                           "traffic": traffic_from_profiles(cfg.name if n == cfg.n_pipelines else f"{cfg.name}@N{n}",
+                                                            kernel_name(args.variant, args.optimizer, n,
+                                                                        args.staleness)),
                            "launch_ms_pct": pct,
                            "kernel": kernel_name(args.variant, args.optimizer, n, args.staleness),
                            "bytes_per_launch": per_launch_bytes, "avg_launch_ms": avg_ms,
