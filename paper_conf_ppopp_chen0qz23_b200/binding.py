@@ -352,6 +352,11 @@ class Channel:
             self._h = None
 
     def __del__(self):  # pragma: no cover
+        # not at interpreter shutdown: ea_chan_destroy synchronises the device, which would never return if a
+        # stream still waits for a message from a peer that is gone (the process teardown frees the buffer)
+        import sys
+        if sys.is_finalizing():
+            return
         try:
             self.close()
         except Exception:
