@@ -318,15 +318,11 @@ __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, 
 // the read-only path (one DRAM read, the other warps hit L1/L2).
 // ============================================================================
 // STALE (row f4, reading c28): the replicas read x~_{t-1} (st.prev) instead of x~_t; the reduction writes
-// x~_{t+1} = x~_t + R/N and prev <- x~_t.  SPREAD (N = 1, one stage): the spread layout's local step -- x~ only
-// read, the contribution stored to `contrib` (zeros over the padding [p, p_pad)), no reduction, no barrier.
-template <int N, int OPT, int U, bool STALE = false, bool SPREAD = false>
-__global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(const StageBatch b, const Hyper hp,
-                                                                           float* __restrict__ contrib,
-                                                                           int64_t p_pad) {
-  static_assert(!SPREAD || (N == 1 && !STALE), "spread: one replica, synchronous center");
+// x~_{t+1} = x~_t + R/N and prev <- x~_t.
+template <int N, int OPT, int U, bool STALE = false>
+__global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(const StageBatch b, const Hyper hp) {
   // N = 1 with the synchronous center: the warp applies x~ += r itself (no contribution tile, no barrier)
-  constexpr bool kDirect = N == 1 && !STALE && !SPREAD;
+  constexpr bool kDirect = N == 1 && !STALE;
   constexpr int TV = 32 * U;  // float4 columns per tile
   constexpr bool kTwo = two_state(OPT);
   __shared__ __align__(16) float4 s_r[N][TV];
@@ -374,15 +370,14 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
       if (lv < nv) {
         const int64_t v = v0 + lv;
         const float4 r = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
-        if constexpr (SPREAD) mem.st(contrib + 4 * v, r);
-        else if constexpr (kDirect) mem.st(st.c + 4 * v, center_apply(c[u], r, hp.inv_n));
+        if constexpr (kDirect) mem.st(st.c + 4 * v, center_apply(c[u], r, hp.inv_n));
         else s_r[warp][lv] = r;
         mem.st(xi + 4 * v, x[u]);
         mem.st(mi + 4 * v, m[u]);
         if (kTwo) mem.st(vi + 4 * v, w[u]);
       }
     }
-    if constexpr (!SPREAD && !kDirect) {
+    if constexpr (!kDirect) {
       __syncthreads();
       for (int col = threadIdx.x; col < nv; col += 32 * N) {
         float4 acc = s_r[0][col];
@@ -396,12 +391,8 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
       __syncthreads();  // s_r is refilled by the next tile
     }
   }
-  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0) {
-    if constexpr (SPREAD)
-      spread_tail<OPT>(b.st[0], contrib, p_pad, hp);
-    else
-      for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
-  }
+  if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
+    for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
 }
 
 // ============================================================================
@@ -1171,7 +1162,7 @@ int warprep_u4() {
 template <int N, int OPT, int U, bool STALE>
 cudaError_t launch_warprep_u(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   auto k = colocated_warprep<N, OPT, U, STALE>;
-  k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp, nullptr, 0);
+  k<<<persistent_grid(k, units_of(b, 32 * U), num_sms, 32 * N), 32 * N, 0, s>>>(b, hp);
   return cudaGetLastError();
 }
 
@@ -1270,11 +1261,12 @@ cudaError_t launch_wide_opt(const ReplicaTable& t, int n, float* center, float* 
 }
 
 // Spread local kernel knob (measurement): AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel
-// (spread_local), =warp the warp-per-replica kernel; default: the bulk-copy pipeline (spread_bulkpipe).
+// (spread_local); default: the bulk-copy pipeline (spread_bulkpipe).  (A warp-per-replica spread kernel measured
+// 0.90-0.94 vs 0.94-0.97 for the bulk-copy pipeline on C3-C5 stages: profiles/r02_s3_spread_local_warp.jsonl.)
 int spread_reg() {
   static int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_SPREAD_KERNEL");
-    return (e && e[0] == 'r') ? 1 : (e && e[0] == 'w') ? 2 : 0;
+    return (e && e[0] == 'r') ? 1 : 0;
   }();
   return v;
 }
@@ -1320,33 +1312,10 @@ cudaError_t launch_spread_bulk(float* x, const float* g, float* m, float* v, con
   }
 }
 
-// Spread local step on the warp-per-replica kernel (N = 1: one warp per CTA, U = 4, no reduction).
-template <int OPT>
-cudaError_t launch_spread_warp(float* x, const float* g, float* m, float* v, const float* center, float* contrib,
-                               int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc, int num_sms,
-                               cudaStream_t s) {
-  StageBatch b;
-  b.nstages = 1;
-  StageRefs& r = b.st[0];
-  for (int i = 0; i < kMaxFusedN; ++i) {
-    r.x[i] = i == 0 ? x : nullptr;
-    r.g[i] = i == 0 ? g : nullptr;
-    r.m[i] = i == 0 ? m : nullptr;
-    r.v[i] = i == 0 ? v : nullptr;
-  }
-  r.c = const_cast<float*>(center);  // read only (SPREAD)
-  r.p = p;
-  r.scp = sc;
-  auto k = colocated_warprep<1, OPT, 4, false, true>;
-  k<<<persistent_grid(k, units_of(b, 128), num_sms, 32), 32, 0, s>>>(b, hp, contrib, p_pad);
-  return cudaGetLastError();
-}
-
 template <int OPT>
 cudaError_t launch_spread_local_opt(float* x, const float* g, float* m, float* v, const float* center,
                                     float* contrib, int64_t p, int64_t p_pad, const Hyper& hp, const StepCoef* sc,
                                     int num_sms, cudaStream_t s) {
-  if (spread_reg() == 2) return launch_spread_warp<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   if (!spread_reg()) return launch_spread_bulk<OPT>(x, g, m, v, center, contrib, p, p_pad, hp, sc, num_sms, s);
   constexpr int U = two_state(OPT) ? 2 : 4;
   const int64_t nvec = p / 4;

@@ -5,8 +5,8 @@ fraction at the algorithmic 28 B (SGD) / 36 B (Adam) per element.
 
     python scripts/bench_spread_local.py [--optimizer sgd|adam] [--reps 200]
 
-AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel, =warp the
-warp-per-replica kernel, instead of the bulk-copy pipeline (measurement knob)."""
+AVGPIPE_EA_SPREAD_KERNEL=reg selects the register kernel instead of the
+bulk-copy pipeline (measurement knob)."""
 import argparse
 import json
 import os

@@ -439,12 +439,11 @@ def test_spread_decomposition_virtual_ranks(n, mode, optimizer, sizes=(200_003, 
         h.close()
 
 
-@pytest.mark.parametrize("kernel", ["reg", "warp"])
+@pytest.mark.parametrize("kernel", ["reg"])
 @pytest.mark.parametrize("optimizer", ["sgd", "adam", "asgd"])
 def test_spread_local_kernel_variants(kernel, optimizer):
-    """The spread local step on the kernels behind AVGPIPE_EA_SPREAD_KERNEL (reg: the register kernel; warp: the
-    warp-per-replica kernel with N = 1) -- the contribution to the exchange buffer, the padding zeroed -- with 4
-    virtual ranks (the knob is read once per process: a subprocess)."""
+    """The spread local step on the register kernel behind AVGPIPE_EA_SPREAD_KERNEL=reg (the contribution to the
+    exchange buffer, the padding zeroed), 4 virtual ranks (the knob is read once per process: a subprocess)."""
     import subprocess
     import sys
     code = ("import tests.test_gpu_parity as t; "
