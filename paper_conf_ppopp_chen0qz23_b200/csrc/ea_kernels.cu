@@ -321,8 +321,6 @@ __device__ void spread_tail(const StageRefs& st, float* contrib, int64_t p_pad, 
 // x~_{t+1} = x~_t + R/N and prev <- x~_t.
 template <int N, int OPT, int U, bool STALE = false>
 __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(const StageBatch b, const Hyper hp) {
-  // N = 1 with the synchronous center: the warp applies x~ += r itself (no contribution tile, no barrier)
-  constexpr bool kDirect = N == 1 && !STALE;
   constexpr int TV = 32 * U;  // float4 columns per tile
   constexpr bool kTwo = two_state(OPT);
   __shared__ __align__(16) float4 s_r[N][TV];
@@ -370,14 +368,14 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
       if (lv < nv) {
         const int64_t v = v0 + lv;
         const float4 r = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
-        if constexpr (kDirect) mem.st(st.c + 4 * v, center_apply(c[u], r, hp.inv_n));
-        else s_r[warp][lv] = r;
+        s_r[warp][lv] = r;
         mem.st(xi + 4 * v, x[u]);
         mem.st(mi + 4 * v, m[u]);
         if (kTwo) mem.st(vi + 4 * v, w[u]);
       }
     }
-    if constexpr (!kDirect) {
+    {  // (applying x~ += r directly at N = 1, without the tile and barriers, measured slower: 0.88 vs 0.94,
+       // profiles/r02_s3_n1_direct.jsonl)
       __syncthreads();
       for (int col = threadIdx.x; col < nv; col += 32 * N) {
         float4 acc = s_r[0][col];
