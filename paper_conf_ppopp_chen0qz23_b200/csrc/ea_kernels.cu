@@ -367,27 +367,25 @@ __global__ void __launch_bounds__(32 * N, N >= 6 ? 2 : 3) colocated_warprep(cons
       const int lv = u * 32 + lane;
       if (lv < nv) {
         const int64_t v = v0 + lv;
-        const float4 r = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
-        s_r[warp][lv] = r;
+        s_r[warp][lv] = ea_vec<OPT>(x[u], g[u], m[u], w[u], c[u], hp, sc);
         mem.st(xi + 4 * v, x[u]);
         mem.st(mi + 4 * v, m[u]);
         if (kTwo) mem.st(vi + 4 * v, w[u]);
       }
     }
-    {  // (applying x~ += r directly at N = 1, without the tile and barriers, measured slower: 0.88 vs 0.94,
-       // profiles/r02_s3_n1_direct.jsonl)
-      __syncthreads();
-      for (int col = threadIdx.x; col < nv; col += 32 * N) {
-        float4 acc = s_r[0][col];
+    // (at N = 1 too: applying x~ += r directly, without the tile and barriers, measured slower -- 0.88 vs 0.94,
+    // profiles/r02_s3_n1_direct.jsonl)
+    __syncthreads();
+    for (int col = threadIdx.x; col < nv; col += 32 * N) {
+      float4 acc = s_r[0][col];
 #pragma unroll
-        for (int i = 1; i < N; ++i) add4(acc, s_r[i][col]);
-        const int64_t v = v0 + col;
-        const float4 cv = __ldg(reinterpret_cast<const float4*>(st.c) + v);
-        mem.st(st.c + 4 * v, center_apply(cv, acc, hp.inv_n));
-        if (STALE) mem.st(st.prev + 4 * v, cv);
-      }
-      __syncthreads();  // s_r is refilled by the next tile
+      for (int i = 1; i < N; ++i) add4(acc, s_r[i][col]);
+      const int64_t v = v0 + col;
+      const float4 cv = __ldg(reinterpret_cast<const float4*>(st.c) + v);
+      mem.st(st.c + 4 * v, center_apply(cv, acc, hp.inv_n));
+      if (STALE) mem.st(st.prev + 4 * v, cv);
     }
+    __syncthreads();  // s_r is refilled by the next tile
   }
   if (blockIdx.x == gridDim.x - 1 && threadIdx.x == 0)
     for (int t = 0; t < b.nstages; ++t) stage_tail<N, OPT, STALE>(b.st[t], hp);
