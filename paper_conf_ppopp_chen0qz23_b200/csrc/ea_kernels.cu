@@ -1178,7 +1178,7 @@ int warpspec_u(int opt, bool stale) {
     const char* e = std::getenv("AVGPIPE_EA_WARPSPEC_U");
     return e ? std::atoi(e) : 0;
   }();
-  if (v == 2 || v == 4) return v;
+  if (v == 2 || v == 4 || (v == 3 && two_state(opt) && !stale)) return v;
   return (two_state(opt) && !stale) ? 2 : 4;
 }
 
@@ -1195,6 +1195,9 @@ cudaError_t launch_warpspec_t(const StageBatch& b, const Hyper& hp, int num_sms,
 template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warpspec(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   if (warpspec_u(OPT, STALE) == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
+  if constexpr (two_state(OPT) && !STALE) {  // U = 3 (Adam): more bytes in flight per warp at 2 CTAs per SM
+    if (warpspec_u(OPT, STALE) == 3) return launch_warpspec_t<N, OPT, 3, 4, STALE>(b, hp, num_sms, s);
+  }
   return launch_warpspec_t<N, OPT, 4, 4, STALE>(b, hp, num_sms, s);
 }
 

@@ -309,19 +309,20 @@ def test_library_default_kernel(n, optimizer, staleness):
 
 
 def test_warp_specialised_u2_and_100_steps():
-    """The U = 2 geometry behind AVGPIPE_EA_WARPSPEC_U (a subprocess: the knob is read once) and the 100-step
-    C1 gate with Adam at N = 8."""
+    """The U = 2 / 3 / 4 geometries behind AVGPIPE_EA_WARPSPEC_U (subprocesses: the knob is read once) and the
+    100-step C1 gate with Adam at N = 8."""
     import subprocess
     import sys
     code = ("import tests.test_gpu_parity as t\n"
             "for opt in ('sgd', 'adam', 'asgd'):\n"
             "    lr = 1e-3 if opt == 'adam' else t.synth.LR\n"
-            "    for n in (1, 4, 8):\n"
+            "    for n in (1, 4, 6, 7, 8):\n"
             "        t._run_colocated(n, [100_003, 7, 4096, 300_001], 8, 'combined', variants=('warpspec',), many=True,"
             " optimizer=opt, lr=lr, wd=0.0 if opt == 'sgd' else 1e-2)\n")
-    r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=dict(os.environ, AVGPIPE_EA_WARPSPEC_U="2"),
-                       capture_output=True, text=True, timeout=1200)
-    assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
+    for u in ("2", "3", "4"):   # (3 applies to Adam(W) only; the others run their default)
+        r = subprocess.run([sys.executable, "-c", code], cwd=ROOT, env=dict(os.environ, AVGPIPE_EA_WARPSPEC_U=u),
+                           capture_output=True, text=True, timeout=1200)
+        assert r.returncode == 0, r.stdout[-2000:] + r.stderr[-4000:]
     _run_colocated(8, [1_000_000, 1_000_003], 100, "combined", variants=("warpspec",), many=True, optimizer="adam",
                    lr=1e-3, wd=1e-2)
 
