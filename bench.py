@@ -220,12 +220,12 @@ def kernel_name(variant, optimizer, n, staleness=0):
             return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"
         return "colocated_wide<stale>"
     two_state = optimizer in ("adam", "adamw")
-    if n > 8 or (two_state and n == 7 and variant == "auto"):
+    if n > 8:
         name = "colocated_wide"
     elif two_state:
         if variant == "auto":
             variant = ("laneshfl" if n == 1 else "regloop" if n <= 3 else "bulkpipe" if n == 4 else
-                       "warprep" if n == 5 else "warpspec" if n == 8 else "split")
+                       "warprep" if n == 5 else "warpspec")
         name = "colocated_" + variant
     elif variant == "auto":   # ea_kernels.cu: SGD / ASGD warp per replica, N = 2 lane kernel, N = 5 warp-specialised
         name = "colocated_laneshfl" if n == 2 else "colocated_warpspec" if n == 5 else "colocated_warprep"
@@ -241,7 +241,7 @@ def colocated_launches(n, k, args, batched):
     two_state = args.optimizer in ("adam", "adamw")
     stale_lane = args.staleness and stale_fused(n, args.optimizer, args.variant)
     force_wide = os.environ.get("AVGPIPE_EA_FORCE_WIDE", "")[:1] == "1"   # ea_api.cu measurement knob
-    per_stage = (n > 8 or not batched or (two_state and n == 7 and args.variant == "auto")
+    per_stage = (n > 8 or not batched
                  or (args.staleness and not stale_lane) or force_wide)
     launches = k if per_stage else (k + 7) // 8
     return launches * (2 if coef else 1)

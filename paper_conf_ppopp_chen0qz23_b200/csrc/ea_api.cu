@@ -317,9 +317,6 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
     const char* v = std::getenv("AVGPIPE_EA_FORCE_WIDE");
     return v && v[0] == '1';
   }();
-  // Adam with N = 7: the replica-loop kernel measured fastest (0.917 vs 0.901 warp-specialised, 0.75 bulk-copy
-  // pipeline; profiles/r01_adam_nsweep.jsonl, r02_s3_sweep_warpspec.jsonl); N = 8 runs the warp-specialised kernel
-  const bool adam_wide = ea::two_state(opt) && n == 7 && h->variant == 0;
   const bool stale = h->cfg.staleness == 1;
   // stale center, default variant: one launch per <= 8 stages -- the lane kernel with x~_{t-1} staged beside x~_t
   // for 2 <= N <= 4, the bulk-copy pipeline with x~_{t-1} as one more stream for N = 1 (and N = 5 for SGD/ASGD);
@@ -363,7 +360,7 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
     }
     return EA_OK;
   }
-  if (n > ea::kMaxFusedN || force_wide || adam_wide || stale) {  // replica loop: one launch per stage
+  if (n > ea::kMaxFusedN || force_wide || stale) {  // replica loop: one launch per stage
     for (int j = 0; j < count; ++j) {
       const int st = stages[j];
       ea::ReplicaTable t;
@@ -1029,7 +1026,7 @@ ea_status ea_step_many_host(ea_handle h, int32_t count, const int32_t* stages, f
       if ((e = cudaEventRecord(h->ev_h2d[b], h->h2d)) != cudaSuccess) return cuda_fail(h, e, "cudaEventRecord");
       if ((e = cudaStreamWaitEvent(s, h->ev_h2d[b], 0)) != cudaSuccess) return cuda_fail(h, e, "cudaStreamWaitEvent");
       // the fused step on [off, off+len) of the stage (elementwise: any chunk is a valid sub-problem)
-      if (n > ea::kMaxFusedN || (ea::two_state(opt) && n == 7 && h->variant == 0)) {
+      if (n > ea::kMaxFusedN) {
         ea::ReplicaTable t;
         for (int i = 0; i < n; ++i) {
           t.x[i] = replica_ptrs[(size_t)j * n + i] + off;

@@ -1171,15 +1171,18 @@ cudaError_t launch_warprep(const StageBatch& b, const Hyper& hp, int num_sms, cu
 }
 
 // Warp-specialised warp per replica (variant 6): U float4 columns per lane and tile, a ring of R = 4 contribution
-// tiles.  U = 2 for Adam(W) with the synchronous center (N = 8: 0.949 vs 0.845 with U = 4), else U = 4
-// (profiles/r02_s3_sweep_warpspec.jsonl); measurement knob AVGPIPE_EA_WARPSPEC_U = 2 | 4 overrides.
-int warpspec_u(int opt, bool stale) {
+// tiles.  Adam(W) with the synchronous center: U = 3 for N = 6, 7 (0.948 / 0.965; U = 2 keeps only 12 / 14 replica
+// warps per SM in flight -- registers per SM sub-partition -- 0.836 / 0.908) and U = 2 for N = 8 (0.968; U = 3
+// spills); else U = 4 (profiles/r02_s3_sweep_warpspec.jsonl, r02_s3_warpspec_u3.jsonl,
+// r02_s3_ncu_warpspec_adam678.md).  Measurement knob AVGPIPE_EA_WARPSPEC_U = 2 | 3 | 4 overrides (3: Adam only).
+int warpspec_u(int opt, bool stale, int n) {
   static const int v = [] {
     const char* e = std::getenv("AVGPIPE_EA_WARPSPEC_U");
     return e ? std::atoi(e) : 0;
   }();
-  if (v == 2 || v == 4 || (v == 3 && two_state(opt) && !stale)) return v;
-  return (two_state(opt) && !stale) ? 2 : 4;
+  const bool adam = two_state(opt) && !stale;
+  if (v == 2 || v == 4 || (v == 3 && adam)) return v;
+  return adam ? ((n == 6 || n == 7) ? 3 : 2) : 4;
 }
 
 template <int N, int OPT, int U, int R, bool STALE>
@@ -1194,9 +1197,10 @@ cudaError_t launch_warpspec_t(const StageBatch& b, const Hyper& hp, int num_sms,
 
 template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warpspec(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
-  if (warpspec_u(OPT, STALE) == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
+  const int u = warpspec_u(OPT, STALE, N);
+  if (u == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
   if constexpr (two_state(OPT) && !STALE) {  // U = 3 (Adam): more bytes in flight per warp at 2 CTAs per SM
-    if (warpspec_u(OPT, STALE) == 3) return launch_warpspec_t<N, OPT, 3, 4, STALE>(b, hp, num_sms, s);
+    if (u == 3) return launch_warpspec_t<N, OPT, 3, 4, STALE>(b, hp, num_sms, s);
   }
   return launch_warpspec_t<N, OPT, 4, 4, STALE>(b, hp, num_sms, s);
 }
@@ -1369,13 +1373,12 @@ cudaError_t launch_colocated_batch(const StageBatch& b, int n, const Hyper& hp, 
   // 0.941 vs 0.920 / 0.937; profiles/r02_sweep_split.jsonl -- with SGD it measured below the bulk pipeline).
   // Round 2 session h (same box, C2 sizes): Adam N = 5 on the warp-per-replica kernel with U = 4, 0.974 (session
   // g) / split 0.944-0.950; N = 2, 3 within 1% of the register loop (0.960 / 0.941 vs 0.948 / 0.940), kept.
-  // Session o: Adam N = 8 on the warp-specialised kernel (U = 2) 0.949 vs 0.924 for the replica loop (N = 7 stays
-  // on the replica loop, ea_api.cu: 0.917 vs 0.901).
+  // Sessions o/v: Adam N = 6..8 on the warp-specialised kernel (U = 3 / 3 / 2): 0.948 / 0.965 / 0.968 vs 0.928 split,
+  // 0.919 / 0.923 replica loop.
   if (variant == kVariantAuto && two_state(opt))
     variant = n == 1 ? kVariantLaneShfl
                      : (n <= 3 ? kVariantRegLoop
-                               : (n == 4 ? kVariantBulkPipe
-                                         : (n == 5 ? kVariantWarpRep : (n == 8 ? kVariantWarpSpec : kVariantSplit))));
+                               : (n == 4 ? kVariantBulkPipe : (n == 5 ? kVariantWarpRep : kVariantWarpSpec)));
   // SGD-momentum and ASGD (one state vector), round 2: the warp-per-replica kernel for N = 1 and 3..8 (same box,
   // C2 sizes: N = 1 0.937 vs 0.872 bulk pipeline, N = 3 0.986 vs 0.932 lane, N = 4 0.996-0.998 vs 0.983 lane,
   // N = 5..8 0.979-1.0 vs 0.93-0.976; ASGD alike), the lane kernel for N = 2 (0.963 vs 0.952);
