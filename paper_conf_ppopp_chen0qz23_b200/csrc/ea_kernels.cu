@@ -1181,7 +1181,7 @@ int warpspec_u(int opt, bool stale, int n) {
     return e ? std::atoi(e) : 0;
   }();
   const bool adam = two_state(opt) && !stale;
-  if (v == 2 || v == 4 || (v == 3 && adam)) return v;
+  if (v == 2 || v == 4 || (v == 3 && two_state(opt))) return v;
   return adam ? ((n == 6 || n == 7) ? 3 : 2) : 4;
 }
 
@@ -1199,7 +1199,7 @@ template <int N, int OPT, bool STALE = false>
 cudaError_t launch_warpspec(const StageBatch& b, const Hyper& hp, int num_sms, cudaStream_t s) {
   const int u = warpspec_u(OPT, STALE, N);
   if (u == 2) return launch_warpspec_t<N, OPT, 2, 4, STALE>(b, hp, num_sms, s);
-  if constexpr (two_state(OPT) && !STALE) {  // U = 3 (Adam): more bytes in flight per warp at 2 CTAs per SM
+  if constexpr (two_state(OPT)) {  // U = 3 (Adam): more bytes in flight per warp at 2 CTAs per SM
     if (u == 3) return launch_warpspec_t<N, OPT, 3, 4, STALE>(b, hp, num_sms, s);
   }
   return launch_warpspec_t<N, OPT, 4, 4, STALE>(b, hp, num_sms, s);
