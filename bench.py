@@ -200,9 +200,11 @@ def workload_key(gpus: int, override):
 
 # ----------------------------------------------------------------------------- our arm
 def stale_fused(n, optimizer, variant):
-    """ea_api.cu: the stale center uses the lane kernel (2 <= N <= 4) or the bulk-copy pipeline (N = 1; N = 5 for
-    SGD/ASGD) under the default variant, one launch per <= 8 stages; else the replica loop per stage."""
-    return ((variant == "auto" and (n <= 4 or (n == 5 and optimizer not in ("adam", "adamw"))))
+    """ea_api.cu: under the default variant the stale center runs one launch per <= 8 stages for N <= 4, SGD/ASGD
+    N = 5 and Adam(W) N <= 8 (bulk-copy pipeline / lane / warp-per-replica / warp-specialised kernels per N,
+    ea_kernels.cu); else the replica loop per stage."""
+    two = optimizer in ("adam", "adamw")
+    return ((variant == "auto" and (n <= 4 or (n == 5 and not two) or (two and n <= 8)))
             or (variant in ("warprep", "warpspec") and n <= 8))
 
 
@@ -214,7 +216,8 @@ def kernel_name(variant, optimizer, n, staleness=0):
     if staleness:
         if stale_fused(n, optimizer, variant):   # ea_api.cu: x~_{t-1} staged beside x~_t, <= 8 stages per launch
             two = optimizer in ("adam", "adamw")
-            kern = ("colocated_warpspec" if variant == "warpspec" or (variant == "auto" and two and n == 3) else
+            kern = ("colocated_warpspec" if variant == "warpspec" or (variant == "auto" and two and n not in (2, 4))
+                    else
                     "colocated_warprep" if variant == "warprep" or (not two and n in (2, 5)) else
                     "colocated_laneshfl" if 2 <= n <= 4 else "colocated_bulkpipe")
             return kern + "<stale" + ("" if optimizer == "sgd" else "," + optimizer) + ">"

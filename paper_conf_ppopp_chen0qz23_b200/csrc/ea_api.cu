@@ -324,7 +324,8 @@ ea_status colocated_launch(ea_ctx* h, int32_t count, const int32_t* stages, floa
   // Adam N = 6: 0.925 vs 0.775 of HBM peak, profiles/r02_sweep_kernels.jsonl).  AVGPIPE_EA_FORCE_WIDE=1 selects
   // the replica loop for A/B measurement.
   const bool stale_lane = stale && !force_wide &&
-                          ((h->variant == 0 && (n <= 4 || (n == 5 && !ea::two_state(opt)))) ||
+                          ((h->variant == 0 && (n <= 4 || (n == 5 && !ea::two_state(opt)) ||
+                                                (ea::two_state(opt) && n <= ea::kMaxFusedN))) ||
                            ((h->variant == ea::kVariantWarpRep || h->variant == ea::kVariantWarpSpec) &&
                             n <= ea::kMaxFusedN));
   if (stale) {  // validate / initialise every stage's x~_{-1} before anything is launched

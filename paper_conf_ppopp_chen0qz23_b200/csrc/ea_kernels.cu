@@ -1180,9 +1180,11 @@ int warpspec_u(int opt, bool stale, int n) {
     const char* e = std::getenv("AVGPIPE_EA_WARPSPEC_U");
     return e ? std::atoi(e) : 0;
   }();
-  const bool adam = two_state(opt) && !stale;
   if (v == 2 || v == 4 || (v == 3 && two_state(opt))) return v;
-  return adam ? ((n == 6 || n == 7) ? 3 : 2) : 4;
+  if (!two_state(opt)) return 4;
+  // stale center (session x, profiles/r02_s3_stale_warpspec.jsonl): the same per-N choice except N = 3 (U = 4)
+  if (stale && n == 3) return 4;
+  return (n == 6 || n == 7) ? 3 : 2;
 }
 
 template <int N, int OPT, int U, int R, bool STALE>
@@ -1450,8 +1452,9 @@ cudaError_t launch_colocated_batch_stale(const StageBatch& b, int n, const Hyper
   // default (round 2, profiles/r02_sweep_warprep_stale.jsonl): SGD/ASGD N = 2 and 5 on the warp-per-replica
   // kernel (0.969 vs 0.923 lane, 0.971 vs 0.958 bulk pipeline); N = 1 the bulk pipeline, N = 3, 4 the lane kernel
   if (variant == kVariantAuto && !two_state(opt) && (n == 2 || n == 5)) variant = kVariantWarpRep;
-  // session o: Adam(W) N = 3 on the warp-specialised kernel (0.933 vs 0.865 lane kernel)
-  if (variant == kVariantAuto && two_state(opt) && n == 3) variant = kVariantWarpSpec;
+  // sessions o/x: Adam(W) N = 1, 3, 5-8 on the warp-specialised kernel (N = 3 0.933-0.944 vs 0.865 lane kernel;
+  // N = 1 0.895 vs 0.864 bulk-copy pipeline; N = 5 / 6 / 7 / 8 0.953 / 0.952 / 0.971 / 0.963 vs 0.92 replica loop)
+  if (variant == kVariantAuto && two_state(opt) && n != 2 && n != 4) variant = kVariantWarpSpec;
   if (variant == kVariantWarpSpec) {
     switch (n) {
       case 1: return launch_stale_warpspec_n<1>(b, hp, opt, num_sms, s);

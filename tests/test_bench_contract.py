@@ -87,8 +87,12 @@ def test_stale_kernel_name_and_launches(monkeypatch):
     assert bench.kernel_name("auto", "adam", 2, 1) == "colocated_laneshfl<stale,adam>"
     assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_bulkpipe<stale>"
     assert bench.kernel_name("auto", "sgd", 5, 1) == "colocated_warprep<stale>"
-    assert bench.kernel_name("auto", "adam", 1, 1) == "colocated_bulkpipe<stale,adam>"
-    assert bench.kernel_name("auto", "adam", 5, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "adam", 1, 1) == "colocated_warpspec<stale,adam>"
+    assert bench.kernel_name("auto", "adam", 7, 1) == "colocated_warpspec<stale,adam>"
+    assert bench.kernel_name("auto", "sgd", 7, 1) == "colocated_wide<stale>"
+    assert bench.kernel_name("auto", "sgd", 1, 1) == "colocated_bulkpipe<stale>"
+    assert bench.kernel_name("auto", "adam", 5, 1) == "colocated_warpspec<stale,adam>"
+    assert bench.kernel_name("auto", "adam", 12, 1) == "colocated_wide<stale>"
     assert bench.kernel_name("auto", "sgd", 6, 1) == "colocated_wide<stale>"
     assert bench.kernel_name("auto", "sgd", 12, 1) == "colocated_wide<stale>"
     args = argparse.Namespace(optimizer="sgd", variant="auto", staleness=1)

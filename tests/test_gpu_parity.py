@@ -298,11 +298,12 @@ def test_warp_specialised_stale(n, optimizer):
 
 
 @pytest.mark.parametrize("n,optimizer,staleness", [(8, "adam", 0), (8, "adamw", 0), (5, "sgd", 0), (5, "asgd", 0),
-                                                   (3, "adam", 1), (3, "adamw", 1), (7, "adam", 0), (6, "adamw", 0)])
+                                                   (3, "adam", 1), (3, "adamw", 1), (7, "adam", 0), (6, "adamw", 0),
+                                                   (1, "adam", 1), (5, "adamw", 1), (6, "adam", 1), (8, "adam", 1)])
 def test_library_default_kernel(n, optimizer, staleness):
-    """The library's own per-N choice (kernel_variant "auto") where sessions o/v moved it: Adam(W) N = 6, 7 (U = 3)
-    and 8 (U = 2) and SGD/ASGD N = 5 to the warp-specialised kernel, the stale Adam(W) N = 3 likewise; 30 steps,
-    several stages per call."""
+    """The library's own per-N choice (kernel_variant "auto") where sessions o/v/x moved it: Adam(W) N = 6, 7 (U = 3)
+    and 8 (U = 2) and SGD/ASGD N = 5 to the warp-specialised kernel, the stale Adam(W) N = 1, 3, 5-8 likewise; 30
+    steps, several stages per call."""
     lr = 1e-3 if optimizer in ("adam", "adamw") else synth.LR
     _run_colocated(n, [100_003, 7, 4096, 1_000_001], 30, "combined", variants=("auto",), many=True,
                    optimizer=optimizer, lr=lr, wd=0.0 if optimizer == "sgd" else 1e-2, staleness=staleness)
