@@ -152,6 +152,34 @@ def test_valid_config_without_gpu_reports_cuda_error(lib):
     assert h.value is None
 
 
+def test_channel_argument_checks_without_gpu(lib):
+    """Activation channels (ea_chan_*): argument validation happens before any CUDA call, every call tolerates a
+    NULL channel, and ea_chan_last_error(NULL) reports the last failed create."""
+    out = ctypes.c_void_p()
+    assert lib.ea_chan_create(0, 2, 1024, 4, ctypes.byref(out)) == binding.EA_EINVAL      # role
+    assert b"role" in lib.ea_chan_last_error(None)
+    assert lib.ea_chan_create(0, 0, 0, 4, ctypes.byref(out)) == binding.EA_EINVAL         # slot_bytes
+    assert lib.ea_chan_create(0, 1, 1024, 0, ctypes.byref(out)) == binding.EA_EINVAL      # slots
+    assert lib.ea_chan_create(0, 0, 1024, 4, None) == binding.EA_EINVAL                   # output
+    assert out.value is None
+    assert lib.ea_chan_send(None, None, 0, None) == binding.EA_EINVAL
+    assert lib.ea_chan_recv(None, None, 0, None) == binding.EA_EINVAL
+    assert lib.ea_chan_export(None, None) == binding.EA_EINVAL
+    assert lib.ea_chan_connect(None, None) == binding.EA_EINVAL
+    assert lib.ea_chan_pair(None, None) == binding.EA_EINVAL
+    assert lib.ea_chan_count(None) == -1
+    assert lib.ea_chan_destroy(None) == binding.EA_OK
+    assert binding.CHAN_HANDLE_BYTES == 80 and binding.IPC_HANDLE_BYTES == 64
+
+
+@pytest.mark.skipif(__import__("torch").cuda.is_available(), reason="checks the no-GPU error path")
+def test_channel_create_without_gpu_reports_cuda_error(lib):
+    out = ctypes.c_void_p()
+    st = lib.ea_chan_create(0, 0, 1024, 4, ctypes.byref(out))
+    assert st in (binding.EA_ECUDA, binding.EA_ENOMEM)
+    assert out.value is None and lib.ea_chan_last_error(None)
+
+
 # ----------------------------------------------------------------- schedule (a9)
 def _oracle(K, M, stage, a):
     return advance_forward_schedule(K, M, stage + 1, a)
